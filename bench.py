@@ -1,0 +1,437 @@
+#!/usr/bin/env python
+"""Benchmark: GNNLab sample+extract hot path on B200 (BASELINE.json metric).
+
+One step = one mini-batch through the whole per-batch path: epoch shuffle
+(a1, at epoch boundaries), k-hop sampling (a2), dedup/relabel into blocks
+(a3), mark (a4) and feature extract (a7) from the PreSC cache (a5/a6 run
+once before the timed region, timed separately like Table 6, PAPER.md
+L468-474).  Workload: configs[1] (ogbn-products-shaped PR, GraphSAGE [25,10],
+batch 8000), synthetic (synth/), alpha = 1.0 (the paper's R% for GSG-PR,
+Table 5); the alpha sweep reports hit rate vs Optimal and seeds/s.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+Under torchrun each rank owns one GPU; batches shard round-robin (batch
+g = i*N + rank); the only collective is the all-reduce of PreSC counts
+(and the max-over-ranks timing).  Rank 0 prints ONE JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synth  # noqa: E402
+
+METRIC = "sample+extract seeds/sec at 1/2/4/8 B200; cache hit rate vs optimal (%)"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=50)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--config", default="PR", choices=list(synth.SHAPES))
+    p.add_argument("--alpha", type=float, default=1.0)
+    p.add_argument("--sweep-steps", type=int, default=10)
+    p.add_argument("--no-sweep", action="store_true")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-seconds", type=float, default=15.0)
+    p.add_argument("--measure-epochs", type=int, default=2)
+    return p.parse_args()
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def workload_name(sh, alpha):
+    samp = (f"k-hop {list(sh.fanouts)}" if sh.sampler == "khop"
+            else f"random walk {len(sh.fanouts)}x(4 walks, len 3, top-{sh.fanouts[0]})")
+    return (f"{sh.name}-shaped synthetic power-law graph (V={sh.V}, E={sh.E}, feat {sh.D}), "
+            f"{samp}, batch {sh.batch}, PreSC#{sh.K}, alpha={alpha}")
+
+
+def read_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.p = None
+        self.path = os.path.join("/tmp", f"glb_clocks_{os.getpid()}.csv")
+
+    def start(self):
+        try:
+            self.f = open(self.path, "w")
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                       "-i", str(self.index), "-lms", "100"], stdout=self.f,
+                                      stderr=subprocess.DEVNULL)
+        except (OSError, FileNotFoundError):
+            self.p = None
+
+    def stop(self):
+        if self.p is None:
+            return None
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.p.kill()
+        self.f.close()
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for line in open(self.path):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                mx = float(parts[2])
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+# ------------------------------------------------------------------------------------------
+def reference_arm(args):
+    """--impl reference: the CPU oracle as it stands (test infrastructure; the one
+    other place bench.py executes oracle/), on this arm's workload/metric."""
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return
+    import oracle
+    sh = synth.SHAPES[args.config]
+    g = synth.make_graph(sh)
+    go = oracle.GraphOracle(g.indptr, g.indices, g.features)
+    nb = math.ceil(sh.n_train / sh.batch)
+    steps = []
+    batches = {}
+
+    def run(i):
+        e = sh.K + i // nb
+        b = i % nb
+        if e not in batches:
+            batches[e] = oracle.epoch_batches(g.train, sh.batch, g.seed, e)
+        seeds = batches[e][b]
+        t0 = time.perf_counter()
+        s = go.sample(sh.sampler, seeds, sh.fanouts, g.seed, e, b)
+        go.extract(s.uniq)
+        return time.perf_counter() - t0, len(seeds)
+
+    for i in range(args.warmup):
+        run(i)
+    tot_t, tot_s = 0.0, 0
+    for i in range(args.warmup, args.warmup + args.steps):
+        t, n = run(i)
+        tot_t += t
+        tot_s += n
+        steps.append(t)
+    v = tot_s / tot_t
+    cores = 1
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": "seeds/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_t / args.steps,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+        "data": "synthetic", "config": {"workload": workload_name(sh, args.alpha)},
+        "cpu_baseline": {"value": v, "unit": "seeds/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{args.steps} full mini-batches (sample+relabel+extract), "
+                                   f"single-threaded C oracle"},
+        "e2e": {"value": v, "unit": "seeds/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(g, sh, budget_s):
+    """Oracle as it stands, timed on this host (rank 0, N=1), bounded sample."""
+    import oracle
+    go = oracle.GraphOracle(g.indptr, g.indices, g.features)
+    bs = oracle.epoch_batches(g.train, sh.batch, g.seed, sh.K)
+    t_tot, seeds, nb = 0.0, 0, 0
+    while t_tot < budget_s and nb < len(bs):
+        t0 = time.perf_counter()
+        s = go.sample(sh.sampler, bs[nb], sh.fanouts, g.seed, sh.K, nb)
+        go.extract(s.uniq)
+        t_tot += time.perf_counter() - t0
+        seeds += len(bs[nb])
+        nb += 1
+    return {"value": seeds / t_tot, "unit": "seeds/s", "cores": 1, "kind": "oracle",
+            "sample": f"{nb} mini-batches of epoch {sh.K} (sample+relabel+extract, "
+                      f"{seeds} seeds, {t_tot:.1f} s), single-threaded C oracle"}
+
+
+# ------------------------------------------------------------------------------------------
+def main():
+    args = parse()
+    if args.impl == "reference":
+        return reference_arm(args)
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_eurosys_yangtswycyz22_b200 as glb
+
+    world, rank, local = dist_env()
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    sh = synth.SHAPES[args.config]
+
+    t0 = time.perf_counter()
+    g = synth.make_graph(sh)
+    t_gen = time.perf_counter() - t0
+
+    ctx = glb.Context(local)
+    stream = torch.cuda.current_stream(dev)
+    ctx.set_stream(stream)
+    t0 = time.perf_counter()
+    ctx.load_graph(g.indptr, g.indices, g.features)
+    t_load = time.perf_counter() - t0
+    kind = sh.sampler
+    if kind == "khop":
+        ctx.set_sampler("khop", fanouts=sh.fanouts, max_batch=sh.batch)
+    else:
+        ctx.set_sampler("rwalk", layers=len(sh.fanouts), walks=synth.RW_WALKS,
+                        walk_len=synth.RW_LEN, topk=sh.fanouts[0], max_batch=sh.batch)
+    ctx.set_train_set(g.train, sh.batch, g.seed)
+    nb = ctx.num_batches
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    # ---- preprocessing (Table 6 analog): PreSC#K and load_cache
+    barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    ctx.presample(sh.K, rank, world)
+    if world > 1:
+        dist.all_reduce(ctx.counts_tensor(glb.COUNT_PRESAMPLE))  # u32 sums (< 2^31)
+    torch.cuda.synchronize()
+    t_pre = time.perf_counter() - t0
+    t0 = time.perf_counter()
+    ctx.build_cache(args.alpha)
+    torch.cuda.synchronize()
+    t_cache = time.perf_counter() - t0
+
+    ub = sh.batch
+    for k in sh.fanouts:
+        ub = min(ub * (1 + k), sh.V)
+    out = torch.empty((ub, sh.D), dtype=torch.float32, device=dev)
+
+    def batch_of(i):
+        gidx = i * world + rank
+        return sh.K + gidx // nb, gidx % nb
+
+    def n_seeds(b):
+        return min(sh.batch, sh.n_train - b * sh.batch)
+
+    # ---- warmup
+    for i in range(args.warmup):
+        e, b = batch_of(i)
+        ctx.sample_batch(e, b)
+        ctx.extract_sample(out)
+    torch.cuda.synchronize()
+
+    # ---- timed region: device time, CUDA events on the launching stream
+    steps = list(range(args.warmup, args.warmup + args.steps))
+    ev_x = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+            for _ in steps]
+    clocks = Clocks(local)
+    launches0 = ctx.launches
+    barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    t_start = torch.cuda.Event(enable_timing=True)
+    t_end = torch.cuda.Event(enable_timing=True)
+    t_start.record(stream)
+    seeds_done = 0
+    for j, i in enumerate(steps):
+        e, b = batch_of(i)
+        ctx.sample_batch(e, b)
+        ev_x[j][0].record(stream)
+        ctx.extract_sample(out)
+        ev_x[j][1].record(stream)
+        seeds_done += n_seeds(b)
+    t_end.record(stream)
+    torch.cuda.synchronize()
+    barrier()
+    clk = clocks.stop()
+    launches = ctx.launches - launches0
+    elapsed_ms = t_start.elapsed_time(t_end)
+    x_ms = [a.elapsed_time(bb) for a, bb in ev_x]
+    el = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
+    tot = torch.tensor([float(seeds_done)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(el, op=dist.ReduceOp.MAX)
+        dist.all_reduce(tot)
+    elapsed_max = float(el.item())
+    value = float(tot.item()) / (elapsed_max / 1e3)
+
+    # ---- replay (untimed) to count the units each timed launch processed
+    nL, hits, misses = [], [], []
+    for i in steps:
+        e, b = batch_of(i)
+        ctx.sample_batch(e, b)
+        s = ctx.sample_result()
+        st = ctx.extract_sample(out, stats=True)
+        nL.append(s.sizes[-1])
+        hits.append(st["hits"])
+        misses.append(st["misses"])
+    D = sh.D
+    # algorithmic HBM bytes of the extract launch: per row read (hit: cache row from
+    # HBM) + write of the out row + the 8-byte (dst, src) work-list entry.
+    hbm_bytes = [h * (2 * 4 * D + 8) + m * (4 * D + 8) for h, m in zip(hits, misses)]
+    ach_gbs = statistics.mean(bb / (t * 1e-3) for bb, t in zip(hbm_bytes, x_ms)) / 1e9
+    peak, peak_src = read_peaks()
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        tj = json.load(open(tp))
+        key = f"{sh.name}:{args.alpha}"
+        if key in tj:
+            traffic = tj[key]
+
+    # ---- e2e through the public API with host buffers (pinned seeds H2D, sizes/stats D2H)
+    e2e_steps = steps[: max(1, min(len(steps), 20))]
+    host_seeds = {}
+    for i in e2e_steps:
+        e, b = batch_of(i)
+        if e not in host_seeds:
+            ctx.shuffle(e)
+            host_seeds[e] = ctx.permutation(sh.n_train)
+    pinned = {i: torch.from_numpy(host_seeds[batch_of(i)[0]][batch_of(i)[1] * sh.batch:
+                                                       batch_of(i)[1] * sh.batch + n_seeds(batch_of(i)[1])].copy()
+                                  ).pin_memory() for i in e2e_steps}
+    barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    e2e_seeds = 0
+    for i in e2e_steps:
+        e, b = batch_of(i)
+        ctx.sample(pinned[i].numpy(), seed=g.seed, epoch=e, batch=b)  # H2D seeds, D2H sizes
+        ctx.extract_sample(out, stats=True)                           # D2H hit/miss counts
+        e2e_seeds += n_seeds(b)
+    torch.cuda.synchronize()
+    e2e_t = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
+    e2e_n = torch.tensor([float(e2e_seeds)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(e2e_n)
+    e2e_val = float(e2e_n.item()) / float(e2e_t.item())
+    h2d = 4 * statistics.mean(n_seeds(batch_of(i)[1]) for i in e2e_steps)
+    d2h = 160 + 16  # DevState sizes record + 2 x u64 hit/miss counts
+
+    # ---- hit rate vs Optimal (accesses recorded over measured epochs, untimed)
+    result_hit = None
+    sweep = []
+    if not args.no_sweep:
+        ctx.reset_counts(glb.COUNT_ACCESS)
+        ctx.set_count_mode(glb.COUNT_ACCESS)
+        for e in range(sh.K, sh.K + args.measure_epochs):
+            for b in range(rank, nb, world):
+                ctx.sample_batch(e, b)
+        ctx.set_count_mode(glb.COUNT_NONE)
+        ctx.sync()
+        if world > 1:
+            dist.all_reduce(ctx.counts_tensor(glb.COUNT_ACCESS))
+        for a in sorted(set(sh.alphas) | {args.alpha}):
+            ctx.build_cache(a)
+            hs = ctx.hit_stats()
+            H = hs["hits"] / hs["total"] if hs["total"] else 0.0
+            Hs = hs["optimal_hits"] / hs["total"] if hs["total"] else 0.0
+            # timed seeds/s at this alpha (short run)
+            torch.cuda.synchronize()
+            s0 = torch.cuda.Event(enable_timing=True)
+            s1 = torch.cuda.Event(enable_timing=True)
+            s0.record(stream)
+            sd = 0
+            for i in range(args.sweep_steps):
+                e, b = batch_of(i)
+                ctx.sample_batch(e, b)
+                ctx.extract_sample(out)
+                sd += n_seeds(b)
+            s1.record(stream)
+            torch.cuda.synchronize()
+            ms = s0.elapsed_time(s1)
+            sweep.append({"alpha": a, "cache_rows": hs["cache_rows"], "hit_rate": H,
+                          "optimal_hit_rate": Hs,
+                          "presc_vs_optimal_pct": (100.0 * H / Hs) if Hs > 0 else None,
+                          "seeds_per_s": sd * world / (ms / 1e3)})
+            if a == args.alpha:
+                result_hit = sweep[-1]
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(g, sh, args.cpu_seconds)
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": "seeds/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": elapsed_max / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "config": {"workload": workload_name(sh, args.alpha), "shape": sh.name,
+                       "V": sh.V, "E": sh.E, "feat_dim": sh.D, "batch": sh.batch,
+                       "fanouts": list(sh.fanouts), "sampler": sh.sampler, "alpha": args.alpha,
+                       "presample_K": sh.K, "parallelism": f"dp{world}",
+                       "l2": "inputs larger than L2 (CSR %.2f GB, feature cache %.2f GB vs 126 MB L2)"
+                             % ((8 * (sh.V + 1) + 4 * sh.E) / 1e9, 4 * sh.D * sh.V * args.alpha / 1e9)},
+            "roofline": {"kernel": "k_gather (extract a7)", "bound": "hbm", "achieved": ach_gbs,
+                         "peak": peak, "unit": "GB/s", "frac": ach_gbs / peak, "traffic": traffic,
+                         "peak_source": peak_src,
+                         "extract_ms_per_step": statistics.mean(x_ms),
+                         "extract_share_of_step": statistics.mean(x_ms) / (elapsed_max / args.steps),
+                         "algorithmic_bytes_per_launch": statistics.mean(hbm_bytes)},
+            "cpu_baseline": cpu,
+            "e2e": {"value": e2e_val, "unit": "seeds/s", "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": d2h, "steps": len(e2e_steps),
+                    "api": "glb_sample(host seeds, sync) + glb_extract_sample + stats"},
+            "gpu_launches": launches,
+            "clocks": clk,
+            "hit_rate": result_hit,
+            "alpha_sweep": sweep,
+            "units": {"mean_n_L": statistics.mean(nL), "mean_hits": statistics.mean(hits),
+                      "mean_misses": statistics.mean(misses)},
+            "preprocess_s": {"generate_inputs": t_gen, "load_graph": t_load,
+                             "presample": t_pre, "build_cache": t_cache},
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

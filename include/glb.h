@@ -1,0 +1,181 @@
+/*
+ * glb.h -- C-ABI of the B200-native GNNLab sample+extract hot path.
+ *
+ * Paper: GNNLab: A Factored System for Sample-based GNN Training over GPUs
+ * (EuroSys'22), text at PAPER.md.  Citations "L<n> §<s>" point into it;
+ * "reading Qn" points at DESIGN.md "Readings" (ambiguities resolved).
+ *
+ * One glb_ctx per (process, GPU).  Plain pointers and sizes only, no torch
+ * types.  All functions return a glb_status (0 = OK, < 0 = error) and never
+ * throw or abort; glb_last_error() returns a detail string.  Unless stated,
+ * calls are asynchronous on the ctx stream (glb_set_stream) and a device
+ * pointer argument must stay valid until the stream reaches the call.
+ * Calls on one ctx are not re-entrant.  After GLB_ECUDA the ctx is poisoned
+ * (every later call returns GLB_ECUDA); destroy it.
+ *
+ * Device memory owned by the ctx (topology copy, relabel tables, cache,
+ * sample buffers) is allocated with cudaMalloc on ctx->device and freed by
+ * glb_destroy.  Host feature memory is BORROWED: glb_load_graph registers it
+ * (cudaHostRegisterMapped|Portable) and glb_destroy unregisters it; the
+ * caller keeps it alive until then.
+ */
+#ifndef GLB_H
+#define GLB_H
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct glb_ctx glb_ctx;
+typedef int32_t glb_status;
+
+enum {
+  GLB_OK = 0,
+  GLB_EINVAL = -1,  /* bad argument: bad CSR, duplicate seed, id >= V, fanout 0, alpha not in [0,1] */
+  GLB_ENOMEM = -2,  /* allocation failed, or a batch exceeds the capacity set by glb_set_sampler */
+  GLB_ECUDA = -3,   /* CUDA runtime error (ctx poisoned) */
+  GLB_ESTATE = -4,  /* call out of order (e.g. sample before load_graph) */
+  GLB_ERANGE = -5   /* epoch >= 2^16 or hop >= 2^8 (RNG counter field widths, reading Q4) */
+};
+
+/* sampler kinds */
+enum {
+  GLB_KHOP_UNIFORM = 0, /* k-hop uniform neighbourhood sampling (L67, Fig 7) */
+  GLB_RANDOM_WALK = 1   /* PinSAGE random walks: "5 neighbors from 4 paths of length 3" (L353) */
+};
+
+/* visit-count recording targets (glb_set_count_mode) */
+enum {
+  GLB_COUNT_NONE = 0,
+  GLB_COUNT_PRESAMPLE = 1, /* PreSC hotness counts h_v (L333 §6.3) */
+  GLB_COUNT_ACCESS = 2     /* measured-epoch accesses, for hit rate / Optimal (L148 fn4) */
+};
+
+#define GLB_MAX_HOPS 8
+
+/* ------------------------------------------------------------------ ctx */
+const char* glb_last_error(const glb_ctx* ctx); /* ctx may be NULL (creation errors) */
+glb_status glb_create(int device, glb_ctx** out);
+glb_status glb_destroy(glb_ctx* ctx);
+/* Run every later call on this stream (cudaStream_t; e.g. torch.cuda.current_stream().cuda_stream).
+ * NULL = the legacy default stream.  A new ctx starts on its own non-blocking stream; callers
+ * that hand device buffers produced on another stream must set that stream (or synchronise). */
+glb_status glb_set_stream(glb_ctx* ctx, void* cuda_stream);
+glb_status glb_sync(glb_ctx* ctx); /* cudaStreamSynchronize + deferred device error check */
+
+/* --------------------------------------------------------------- load(dev, graph) (Fig 9)
+ * indptr: host u64[V+1], indptr[0]=0, non-decreasing, indptr[V]=E.
+ * indices: host u32[E], each < V.  Topology is COPIED into HBM (D1: CSR in GPU
+ * memory, L222/L250).  features: host f32[V][feat_dim] row-major, BORROWED and
+ * registered as mapped pinned memory (D2); may be NULL (sample-only ctx).
+ * Synchronous.  Errors: EINVAL (shape/monotonicity/range), ENOMEM, ECUDA. */
+glb_status glb_load_graph(glb_ctx* ctx, uint64_t num_vertices, uint64_t num_edges,
+                          const uint64_t* indptr, const uint32_t* indices,
+                          const void* features, uint32_t feat_dim);
+
+/* Sampler used by glb_sample_batch / glb_presample, and the capacity of the
+ * per-batch buffers.  kind GLB_KHOP_UNIFORM: fanouts[0..num_hops-1] (hop order
+ * from the seeds, reading Q1).  kind GLB_RANDOM_WALK: num_hops layers, each
+ * keeping rw_topk of rw_walks walks of rw_len steps (fanouts ignored).
+ * max_batch: largest seed count a batch may have.  Synchronous (allocates). */
+glb_status glb_set_sampler(glb_ctx* ctx, int kind, const uint32_t* fanouts, uint32_t num_hops,
+                           uint32_t rw_walks, uint32_t rw_len, uint32_t rw_topk,
+                           uint32_t max_batch);
+
+/* Training set T (host u32[n], distinct, each < V) and mini-batch size B
+ * (L305 §6.2: shuffle T each epoch and divide it; last batch partial).
+ * seed keys every draw of the ctx (shuffle and sampling).  Synchronous. */
+glb_status glb_set_train_set(glb_ctx* ctx, const uint32_t* train, uint64_t n, uint32_t batch_size,
+                             uint64_t seed);
+/* number of mini-batches per epoch = ceil(n / B) */
+glb_status glb_num_batches(const glb_ctx* ctx, uint32_t* out);
+/* a1: device-side epoch permutation (Philox keys + stable radix sort; reading Q9/§8(c).2).
+ * Later glb_sample_batch(epoch, b) calls use it. */
+glb_status glb_shuffle(glb_ctx* ctx, uint32_t epoch);
+/* copy the current epoch permutation to host u32[n] (synchronous; tests) */
+glb_status glb_get_permutation(glb_ctx* ctx, uint32_t* host_out);
+
+/* ---------------------------------------------------------------- samples (a2-a4)
+ * Per-hop blocks, DGL style (reading Q3): block l has dst = lids 0..n_l-1 and
+ * src = lids 0..n_{l+1}-1; uniq[lid] = gid and the first n_l lids are the
+ * frontier of hop l (seeds first, in input order; new vertices in
+ * first-occurrence order, reading Q5).  Device pointers are OWNED BY THE CTX
+ * and valid until the next sample call. */
+typedef struct {
+  uint32_t num_hops;
+  uint32_t num_seeds;
+  const uint32_t* uniq;                   /* device u32[sizes[num_hops]] */
+  uint64_t sizes[GLB_MAX_HOPS + 1];       /* n_0..n_L (host values) */
+  uint64_t nnz[GLB_MAX_HOPS];             /* edges of block l */
+  const uint32_t* indptr[GLB_MAX_HOPS];   /* device u32[n_l+1] */
+  const uint32_t* indices[GLB_MAX_HOPS];  /* device u32[nnz_l], src lids, slot order */
+  const uint32_t* weights[GLB_MAX_HOPS];  /* device u32[nnz_l] visit counts (random walk), else NULL */
+  const int32_t* cache_slot;              /* device i32[sizes[L]]: slot of uniq[i] or -1 (a4 "mark") */
+} glb_blocks;
+
+/* Sample one mini-batch.  seeds: host or device u32[num_seeds] (distinct, < V).
+ * The sampler is the one set by glb_set_sampler; kind GLB_KHOP_UNIFORM may
+ * override its fanouts with (fanouts, num_hops) -- pass NULL/0 to keep them.
+ * Draws are keyed by (seed, epoch, batch, hop, vertex, slot) (reading Q4).
+ * Synchronous: one device->host copy of the sizes.  Errors: EINVAL (dup seed,
+ * id >= V), ENOMEM (num_seeds > max_batch), ERANGE, ESTATE. */
+glb_status glb_sample(glb_ctx* ctx, const uint32_t* seeds, uint32_t num_seeds,
+                      const uint32_t* fanouts, uint32_t num_hops, uint64_t seed, uint32_t epoch,
+                      uint32_t batch, glb_blocks* out);
+
+/* Sample mini-batch `batch` of the current epoch permutation (glb_shuffle) with
+ * the ctx sampler.  ASYNCHRONOUS: no host sync; sizes stay on the device.
+ * Visit counts are recorded per the count mode.  Use glb_sample_result to read
+ * sizes (synchronises), or glb_extract_sample to gather features directly. */
+glb_status glb_sample_batch(glb_ctx* ctx, uint32_t epoch, uint32_t batch);
+glb_status glb_sample_result(glb_ctx* ctx, glb_blocks* out);
+
+/* ---------------------------------------------------------------- PreSC (a5, a6)
+ * GLB_COUNT_PRESAMPLE: every batch-unique vertex of every later sample adds 1 to
+ * counts[v] (reading Q8); GLB_COUNT_ACCESS: adds 1 to access[v]. */
+glb_status glb_set_count_mode(glb_ctx* ctx, int mode);
+glb_status glb_reset_counts(glb_ctx* ctx, int which /* GLB_COUNT_PRESAMPLE | _ACCESS */);
+/* PreSC#K (L333-335 §6.3): sample every batch of epochs 0..K-1 of this rank's
+ * share (batches b with b % world == rank) with recording into counts.
+ * Counts accumulate; allreduce them across ranks before glb_build_cache. */
+glb_status glb_presample(glb_ctx* ctx, uint32_t K, uint32_t rank, uint32_t world);
+/* device pointer of the u32[V] count array (for NCCL allreduce through torch) */
+glb_status glb_counts_device_ptr(glb_ctx* ctx, int which, void** out);
+glb_status glb_get_counts(glb_ctx* ctx, int which, uint32_t* host_out /* V */);
+/* load_cache(hotness_map, alpha) (L301 §6.1): C = floor(alpha*V); rank vertices by
+ * (count desc, gid asc) (reading Q10); slot = rank for the first C; copy their
+ * feature rows from host memory into an HBM cache f32[C][D].  hotness: NULL =
+ * the PreSC counts, else a device u32[V] hotness map (e.g. degree).  Synchronous. */
+glb_status glb_build_cache(glb_ctx* ctx, double alpha, const uint32_t* hotness);
+glb_status glb_get_cache_slots(glb_ctx* ctx, int32_t* host_out /* V */);
+glb_status glb_cache_size(const glb_ctx* ctx, uint64_t* out);
+
+/* Hit-rate statistics over the recorded accesses (GLB_COUNT_ACCESS) for the
+ * current cache: total accesses, accesses served by the cache (H = hits/total),
+ * and the Optimal policy's hits: the C largest access counts (L148 fn4, L339).
+ * Synchronous.  Exact integers. */
+typedef struct { uint64_t total, hits, optimal_hits, cache_rows; } glb_hit_stats;
+glb_status glb_hit_stats_get(glb_ctx* ctx, glb_hit_stats* out);
+
+/* ---------------------------------------------------------------- extract (a7)
+ * extract(features, samples) (Fig 9; L252): out[i,:] = features[vertices[i],:]
+ * for i < n, bytes exact; cache hits read the HBM cache, misses read the
+ * mapped pinned host matrix over PCIe (zero copy).  vertices: device u32[n]
+ * (any ids < V, duplicates allowed); out: device f32[n][D], caller-owned.
+ * stats (nullable, HOST pointer): filled at the next glb_sync. */
+typedef struct { uint64_t hits, misses; } glb_extract_stats;
+glb_status glb_extract(glb_ctx* ctx, const uint32_t* vertices, uint64_t n, void* out,
+                       glb_extract_stats* stats);
+/* Extract the features of the last sample's uniq (out: device f32[>= n_L][D]),
+ * using the marks taken during relabel; no host sync. */
+glb_status glb_extract_sample(glb_ctx* ctx, void* out, glb_extract_stats* stats);
+
+/* launch counter: number of kernels this ctx launched so far (bench evidence) */
+uint64_t glb_kernel_launches(const glb_ctx* ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

@@ -1,0 +1,630 @@
+// capi.cu -- the extern "C" boundary (include/glb.h): context, buffers, and
+// the host-side sequencing of the hot path.  No host sync inside a sampled
+// batch: every size a kernel needs lives in DevState on the device.
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <new>
+
+#include "glb_internal.cuh"
+
+using namespace glb;
+
+namespace {
+
+thread_local std::string g_create_err;
+
+glb_status set_err(glb_ctx* c, glb_status s, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  if (c) c->err = buf;
+  else g_create_err = buf;
+  return s;
+}
+
+glb_status cuda_fail(glb_ctx* c, cudaError_t e, const char* what) {
+  if (c) c->poisoned = true;
+  return set_err(c, GLB_ECUDA, "%s: %s", what, cudaGetErrorString(e));
+}
+
+#define CK(expr)                                          \
+  do {                                                    \
+    cudaError_t e_ = (expr);                              \
+    if (e_ != cudaSuccess) return cuda_fail(c, e_, #expr); \
+  } while (0)
+
+#define ENTER(c)                                                            \
+  do {                                                                      \
+    if (!(c)) return set_err(nullptr, GLB_EINVAL, "null ctx");              \
+    if ((c)->poisoned) return set_err(c, GLB_ECUDA, "ctx poisoned: %s", (c)->err.c_str()); \
+    cudaError_t e0_ = cudaSetDevice((c)->device);                           \
+    if (e0_ != cudaSuccess) return cuda_fail(c, e0_, "cudaSetDevice");     \
+  } while (0)
+
+template <typename T>
+void dfree(T*& p) {
+  if (p) cudaFree((void*)p);
+  p = nullptr;
+}
+
+template <typename T>
+cudaError_t dalloc(T** p, uint64_t count) {
+  *p = nullptr;
+  return cudaMalloc((void**)p, sizeof(T) * (count ? count : 1));
+}
+
+void free_sample_bufs(glb_ctx* c) {
+  SampleBufs& b = c->sb;
+  dfree(b.seeds); dfree(b.uniq); dfree(b.lidslot); dfree(b.picks); dfree(b.pickw);
+  for (int l = 0; l < GLB_MAX_HOPS; ++l) {
+    dfree(b.bindptr[l]); dfree(b.bindices[l]); dfree(b.bweights[l]); dfree(b.status[l]);
+  }
+  dfree(b.hit_dst); dfree(b.hit_src); dfree(b.miss_dst); dfree(b.miss_src);
+  b = SampleBufs();
+  c->sampler_set = false;
+  c->have_sample = false;
+}
+
+void free_graph(glb_ctx* c) {
+  dfree(c->indptr); dfree(c->indices); dfree(c->vmap); dfree(c->lidmap);
+  dfree(c->slot); dfree(c->cache); dfree(c->counts); dfree(c->access);
+  if (c->registered && c->h_features) cudaHostUnregister((void*)c->h_features);
+  c->registered = false;
+  c->h_features = nullptr;
+  c->features_mapped = nullptr;
+  c->V = c->E = 0;
+  c->C = 0;
+  c->D = 0;
+  c->gen = 0;
+  c->have_sample = false;
+}
+
+glb_status check_dev_err(glb_ctx* c, DevState* st) {
+  uint32_t err = 0;
+  CK(cudaMemcpyAsync(&err, &st->err, sizeof(err), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  if (err) {
+    CK(cudaMemsetAsync(&st->err, 0, sizeof(uint32_t), c->stream));
+    if (err & kErrDupSeed) return set_err(c, GLB_EINVAL, "duplicate seed in batch");
+    if (err & kErrRange) return set_err(c, GLB_EINVAL, "vertex id >= V");
+    if (err & kErrBadGraph) return set_err(c, GLB_EINVAL, "invalid CSR");
+    return set_err(c, GLB_EINVAL, "device error 0x%x", err);
+  }
+  return GLB_OK;
+}
+
+// Enqueue one sampled mini-batch (a2/a2' + a3 + a4, and a5 when counting).
+glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, int kind,
+                          const uint32_t* k, uint32_t L, uint64_t seed, uint32_t epoch,
+                          uint32_t batch) {
+  if (epoch > 0xFFFFu) return set_err(c, GLB_ERANGE, "epoch %u >= 2^16", epoch);
+  if (n0 > c->sb.cap_batch) return set_err(c, GLB_ENOMEM, "batch %u > max_batch %u", n0, c->sb.cap_batch);
+  if (L > c->sb.L) return set_err(c, GLB_ENOMEM, "num_hops %u > configured %u", L, c->sb.L);
+  for (uint32_t l = 0; l < L; ++l)
+    if (k[l] > c->sb.k[l]) return set_err(c, GLB_ENOMEM, "fanout %u > configured %u at hop %u", k[l], c->sb.k[l], l);
+  if (c->gen >= 0xFFFFFFF0u) {  // generation wrap: clear the relabel table once
+    CK(cudaMemsetAsync(c->vmap, 0xFF, sizeof(unsigned long long) * c->V, c->stream));
+    c->gen = 0;
+  }
+  c->gen += 1;
+  CK(cudaMemsetAsync(c->st, 0, sizeof(DevState), c->stream));
+  const int mode = c->count_mode;
+  CK(launch_seed_init(c, seeds_dev, n0, mode));
+  for (uint32_t l = 0; l < L; ++l) {
+    if (kind == GLB_KHOP_UNIFORM) CK(launch_khop(c, l, k[l], seed, epoch, batch));
+    else CK(launch_rwalk(c, l, seed, epoch, batch));
+    CK(launch_compact(c, l, k[l], kind == GLB_RANDOM_WALK, mode));
+    CK(launch_remap(c, l));
+  }
+  c->have_sample = true;
+  c->last_L = L;
+  c->last_kind = kind;
+  c->last_n0 = n0;
+  for (uint32_t l = 0; l < L; ++l) c->last_k[l] = k[l];
+  return GLB_OK;
+}
+
+glb_status ensure_perm(glb_ctx* c, uint32_t epoch) {
+  if (c->perm_epoch == (int)epoch) return GLB_OK;
+  return glb_shuffle(c, epoch);
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* glb_last_error(const glb_ctx* ctx) {
+  return ctx ? ctx->err.c_str() : g_create_err.c_str();
+}
+
+uint64_t glb_kernel_launches(const glb_ctx* ctx) { return ctx ? ctx->launches : 0; }
+
+glb_status glb_create(int device, glb_ctx** out) {
+  if (!out) return set_err(nullptr, GLB_EINVAL, "null out");
+  *out = nullptr;
+  int n = 0;
+  cudaError_t e = cudaGetDeviceCount(&n);
+  if (e != cudaSuccess || n == 0) return set_err(nullptr, GLB_ECUDA, "no CUDA device: %s", cudaGetErrorString(e));
+  if (device < 0 || device >= n) return set_err(nullptr, GLB_EINVAL, "device %d out of range", device);
+  glb_ctx* c = new (std::nothrow) glb_ctx();
+  if (!c) return set_err(nullptr, GLB_ENOMEM, "host alloc");
+  c->device = device;
+  if ((e = cudaSetDevice(device)) != cudaSuccess ||
+      (e = cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device)) != cudaSuccess ||
+      (e = cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking)) != cudaSuccess ||
+      (e = cudaMalloc(&c->st, sizeof(DevState))) != cudaSuccess ||
+      (e = cudaMalloc(&c->st_x, sizeof(DevState))) != cudaSuccess ||
+      (e = cudaMalloc(&c->scratch, 4 * sizeof(unsigned long long))) != cudaSuccess ||
+      (e = cudaMalloc(&c->xcount, 2 * sizeof(unsigned long long))) != cudaSuccess ||
+      (e = cudaMallocHost(&c->h_st, sizeof(DevState))) != cudaSuccess ||
+      (e = cudaMallocHost(&c->h_xcount, 2 * sizeof(unsigned long long))) != cudaSuccess ||
+      (e = cudaMemset(c->st, 0, sizeof(DevState))) != cudaSuccess ||
+      (e = cudaMemset(c->st_x, 0, sizeof(DevState))) != cudaSuccess) {
+    glb_status s = set_err(nullptr, GLB_ECUDA, "glb_create: %s", cudaGetErrorString(e));
+    glb_destroy(c);
+    return s;
+  }
+  c->stream = c->own_stream;
+  *out = c;
+  return GLB_OK;
+}
+
+glb_status glb_destroy(glb_ctx* c) {
+  if (!c) return GLB_OK;
+  cudaSetDevice(c->device);
+  if (c->stream) cudaStreamSynchronize(c->stream);
+  free_sample_bufs(c);
+  free_graph(c);
+  dfree(c->xb.hit_dst); dfree(c->xb.hit_src); dfree(c->xb.miss_dst); dfree(c->xb.miss_src);
+  dfree(c->train); dfree(c->perm); dfree(c->shuf_keys); dfree(c->shuf_vals);
+  dfree(c->st); dfree(c->st_x); dfree(c->scratch); dfree(c->xcount);
+  if (c->sort_tmp) cudaFree(c->sort_tmp);
+  if (c->h_st) cudaFreeHost(c->h_st);
+  if (c->h_xcount) cudaFreeHost(c->h_xcount);
+  if (c->own_stream) cudaStreamDestroy(c->own_stream);
+  delete c;
+  return GLB_OK;
+}
+
+glb_status glb_set_stream(glb_ctx* c, void* s) {
+  ENTER(c);
+  c->stream = (cudaStream_t)s;  // NULL = the legacy default stream
+  return GLB_OK;
+}
+
+glb_status glb_sync(glb_ctx* c) {
+  ENTER(c);
+  CK(cudaStreamSynchronize(c->stream));
+  if (c->pending_stats) {
+    c->pending_stats->hits = c->h_xcount[0];
+    c->pending_stats->misses = c->h_xcount[1];
+    c->pending_stats = nullptr;
+  }
+  glb_status s = check_dev_err(c, c->st_x);
+  if (s != GLB_OK) return s;
+  return check_dev_err(c, c->st);
+}
+
+glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* indptr,
+                          const uint32_t* indices, const void* features, uint32_t D) {
+  ENTER(c);
+  if (V == 0 || V >= 0xFFFFFFFFull) return set_err(c, GLB_EINVAL, "V=%llu out of range", (unsigned long long)V);
+  if (!indptr || (E && !indices)) return set_err(c, GLB_EINVAL, "null CSR");
+  if (indptr[0] != 0 || indptr[V] != E) return set_err(c, GLB_EINVAL, "indptr[0]!=0 or indptr[V]!=E");
+  if (features && D == 0) return set_err(c, GLB_EINVAL, "feat_dim 0");
+  CK(cudaStreamSynchronize(c->stream));
+  free_graph(c);
+  free_sample_bufs(c);
+  c->V = V;
+  c->E = E;
+  CK(dalloc(&c->indptr, V + 1));
+  CK(dalloc(&c->indices, E));
+  CK(dalloc(&c->vmap, V));
+  CK(dalloc(&c->lidmap, V));
+  CK(dalloc(&c->slot, V));
+  CK(dalloc(&c->counts, V));
+  CK(dalloc(&c->access, V));
+  CK(cudaMemcpy(c->indptr, indptr, sizeof(uint64_t) * (V + 1), cudaMemcpyHostToDevice));
+  if (E) CK(cudaMemcpy(c->indices, indices, sizeof(uint32_t) * E, cudaMemcpyHostToDevice));
+  CK(cudaMemsetAsync(c->vmap, 0xFF, sizeof(unsigned long long) * V, c->stream));
+  CK(cudaMemsetAsync(c->slot, 0xFF, sizeof(int32_t) * V, c->stream));
+  CK(cudaMemsetAsync(c->counts, 0, sizeof(uint32_t) * V, c->stream));
+  CK(cudaMemsetAsync(c->access, 0, sizeof(uint32_t) * V, c->stream));
+  CK(cudaMemsetAsync(c->st, 0, sizeof(DevState), c->stream));
+  CK(launch_validate_graph(c));
+  glb_status s = check_dev_err(c, c->st);
+  if (s != GLB_OK) {
+    free_graph(c);
+    return s;
+  }
+  if (features) {
+    const size_t bytes = (size_t)V * D * sizeof(float);
+    cudaError_t e = cudaHostRegister((void*)features, bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+    if (e == cudaErrorHostMemoryAlreadyRegistered) {
+      (void)cudaGetLastError();
+      c->registered = false;
+    } else if (e != cudaSuccess) {
+      (void)cudaGetLastError();
+      free_graph(c);
+      return set_err(c, GLB_ENOMEM, "cudaHostRegister(%zu bytes): %s", bytes, cudaGetErrorString(e));
+    } else {
+      c->registered = true;
+    }
+    void* dp = nullptr;
+    CK(cudaHostGetDevicePointer(&dp, (void*)features, 0));
+    c->h_features = features;
+    c->features_mapped = (const float*)dp;
+    c->D = D;
+  }
+  return GLB_OK;
+}
+
+glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32_t L,
+                           uint32_t walks, uint32_t len, uint32_t topk, uint32_t max_batch) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "set_sampler before load_graph");
+  if (L > GLB_MAX_HOPS) return set_err(c, GLB_EINVAL, "num_hops %u > %d", L, GLB_MAX_HOPS);
+  uint32_t k[GLB_MAX_HOPS] = {};
+  if (kind == GLB_KHOP_UNIFORM) {
+    if (L && !fanouts) return set_err(c, GLB_EINVAL, "null fanouts");
+    for (uint32_t l = 0; l < L; ++l) {
+      if (fanouts[l] == 0 || fanouts[l] > (uint32_t)kMaxFanout)
+        return set_err(c, GLB_EINVAL, "fanout %u not in [1,%d]", fanouts[l], kMaxFanout);
+      k[l] = fanouts[l];
+    }
+  } else if (kind == GLB_RANDOM_WALK) {
+    if (walks == 0 || walks > 32 || len == 0 || len > (uint32_t)kMaxWalkLen || topk == 0 || topk > 32)
+      return set_err(c, GLB_EINVAL, "random walk needs walks in [1,32], len in [1,%d], topk in [1,32]", kMaxWalkLen);
+    for (uint32_t l = 0; l < L; ++l) k[l] = topk;
+  } else {
+    return set_err(c, GLB_EINVAL, "unknown sampler kind %d", kind);
+  }
+  CK(cudaStreamSynchronize(c->stream));
+  free_sample_bufs(c);
+  SampleBufs& b = c->sb;
+  b.cap_batch = max_batch;
+  b.L = L;
+  b.ub[0] = max_batch < c->V ? max_batch : c->V;
+  uint64_t pos = b.ub[0], maxflat = 1;
+  for (uint32_t l = 0; l < L; ++l) {
+    b.k[l] = k[l];
+    const uint64_t flat = b.ub[l] * k[l];
+    if (flat >= (1ull << 31)) return set_err(c, GLB_ENOMEM, "hop %u capacity %llu >= 2^31", l, (unsigned long long)flat);
+    pos += flat;
+    maxflat = flat > maxflat ? flat : maxflat;
+    const uint64_t nx = b.ub[l] * (1ull + k[l]);
+    b.ub[l + 1] = nx < c->V ? nx : c->V;
+  }
+  if (pos >= 0xFFFFFFFFull) return set_err(c, GLB_ENOMEM, "relabel positions overflow 2^32");
+  const uint64_t un = b.ub[L] > max_batch ? b.ub[L] : max_batch;
+  CK(dalloc(&b.seeds, max_batch));
+  CK(dalloc(&b.uniq, un));
+  CK(dalloc(&b.lidslot, un));
+  CK(dalloc(&b.picks, maxflat));
+  if (kind == GLB_RANDOM_WALK) CK(dalloc(&b.pickw, maxflat));
+  for (uint32_t l = 0; l < L; ++l) {
+    const uint64_t flat = b.ub[l] * k[l];
+    CK(dalloc(&b.bindptr[l], b.ub[l] + 1));
+    CK(dalloc(&b.bindices[l], flat));
+    if (kind == GLB_RANDOM_WALK) CK(dalloc(&b.bweights[l], flat));
+    b.ntiles[l] = (flat + kCompactTile - 1) / kCompactTile;
+    CK(dalloc(&b.status[l], b.ntiles[l]));
+  }
+  CK(dalloc(&b.hit_dst, un));
+  CK(dalloc(&b.hit_src, un));
+  CK(dalloc(&b.miss_dst, un));
+  CK(dalloc(&b.miss_src, un));
+  c->kind = kind;
+  c->L = L;
+  for (uint32_t l = 0; l < L; ++l) c->fanouts[l] = k[l];
+  c->rw_walks = walks;
+  c->rw_len = len;
+  c->rw_topk = topk;
+  c->sampler_set = true;
+  return GLB_OK;
+}
+
+glb_status glb_set_train_set(glb_ctx* c, const uint32_t* train, uint64_t n, uint32_t B,
+                             uint64_t seed) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "set_train_set before load_graph");
+  if (B == 0 || (n && !train) || n >= 0xFFFFFFFFull) return set_err(c, GLB_EINVAL, "bad train set");
+  for (uint64_t i = 0; i < n; ++i)
+    if (train[i] >= c->V) return set_err(c, GLB_EINVAL, "train id %u >= V", train[i]);
+  CK(cudaStreamSynchronize(c->stream));
+  dfree(c->train); dfree(c->perm); dfree(c->shuf_keys); dfree(c->shuf_vals);
+  CK(dalloc(&c->train, n));
+  CK(dalloc(&c->perm, n));
+  CK(dalloc(&c->shuf_keys, 2 * n));
+  CK(dalloc(&c->shuf_vals, 2 * n));
+  if (n) CK(cudaMemcpy(c->train, train, sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
+  c->n_train = n;
+  c->batch_size = B;
+  c->seed = seed;
+  c->train_set = true;
+  c->perm_epoch = -1;
+  return GLB_OK;
+}
+
+glb_status glb_num_batches(const glb_ctx* c, uint32_t* out) {
+  if (!c || !out) return GLB_EINVAL;
+  if (!c->train_set) return GLB_ESTATE;
+  *out = (uint32_t)((c->n_train + c->batch_size - 1) / c->batch_size);
+  return GLB_OK;
+}
+
+glb_status glb_shuffle(glb_ctx* c, uint32_t epoch) {
+  ENTER(c);
+  if (!c->train_set) return set_err(c, GLB_ESTATE, "shuffle before set_train_set");
+  if (epoch > 0xFFFFu) return set_err(c, GLB_ERANGE, "epoch %u >= 2^16", epoch);
+  const uint64_t n = c->n_train;
+  unsigned long long* kout = nullptr;
+  uint32_t* vout = nullptr;
+  CK(launch_shuffle_keys(c, epoch, c->shuf_keys, c->shuf_vals));
+  CK(radix_sort_pairs_u64(c, c->shuf_keys, c->shuf_vals, c->shuf_keys + n, c->shuf_vals + n, n, 64,
+                          &kout, &vout));
+  CK(launch_permute(c, c->train, vout, n, c->perm));
+  c->perm_epoch = (int)epoch;
+  return GLB_OK;
+}
+
+glb_status glb_get_permutation(glb_ctx* c, uint32_t* host_out) {
+  ENTER(c);
+  if (c->perm_epoch < 0) return set_err(c, GLB_ESTATE, "no permutation yet");
+  CK(cudaMemcpyAsync(host_out, c->perm, sizeof(uint32_t) * c->n_train, cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  return GLB_OK;
+}
+
+glb_status glb_sample_result(glb_ctx* c, glb_blocks* out) {
+  ENTER(c);
+  if (!c->have_sample) return set_err(c, GLB_ESTATE, "no sample");
+  CK(cudaMemcpyAsync(c->h_st, c->st, sizeof(DevState), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  const DevState& h = *c->h_st;
+  if (h.err) {
+    CK(cudaMemsetAsync(&c->st->err, 0, sizeof(uint32_t), c->stream));
+    if (h.err & kErrDupSeed) return set_err(c, GLB_EINVAL, "duplicate seed in batch");
+    if (h.err & kErrRange) return set_err(c, GLB_EINVAL, "seed id >= V");
+    return set_err(c, GLB_EINVAL, "device error 0x%x", h.err);
+  }
+  if (!out) return GLB_OK;
+  memset(out, 0, sizeof(*out));
+  out->num_hops = c->last_L;
+  out->num_seeds = c->last_n0;
+  out->uniq = c->sb.uniq;
+  out->cache_slot = c->sb.lidslot;
+  for (uint32_t l = 0; l <= c->last_L; ++l) out->sizes[l] = h.n[l];
+  for (uint32_t l = 0; l < c->last_L; ++l) {
+    out->nnz[l] = h.nnz[l];
+    out->indptr[l] = c->sb.bindptr[l];
+    out->indices[l] = c->sb.bindices[l];
+    out->weights[l] = c->last_kind == GLB_RANDOM_WALK ? c->sb.bweights[l] : nullptr;
+  }
+  return GLB_OK;
+}
+
+glb_status glb_sample(glb_ctx* c, const uint32_t* seeds, uint32_t n0, const uint32_t* fanouts,
+                      uint32_t L, uint64_t seed, uint32_t epoch, uint32_t batch, glb_blocks* out) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "sample before load_graph");
+  if (!c->sampler_set) return set_err(c, GLB_ESTATE, "sample before set_sampler");
+  if (n0 && !seeds) return set_err(c, GLB_EINVAL, "null seeds");
+  const uint32_t* k = c->fanouts;
+  if (c->kind == GLB_KHOP_UNIFORM && fanouts) {
+    for (uint32_t l = 0; l < L; ++l)
+      if (fanouts[l] == 0) return set_err(c, GLB_EINVAL, "fanout 0");
+    k = fanouts;
+  } else {
+    L = c->L;
+  }
+  if (n0 > c->sb.cap_batch) return set_err(c, GLB_ENOMEM, "batch %u > max_batch %u", n0, c->sb.cap_batch);
+  const uint32_t* sd = seeds;
+  cudaPointerAttributes at;
+  const bool on_dev = n0 && cudaPointerGetAttributes(&at, seeds) == cudaSuccess &&
+                      at.type == cudaMemoryTypeDevice;
+  (void)cudaGetLastError();
+  if (!on_dev) {
+    if (n0) CK(cudaMemcpyAsync(c->sb.seeds, seeds, sizeof(uint32_t) * n0, cudaMemcpyHostToDevice, c->stream));
+    sd = c->sb.seeds;
+  }
+  glb_status s = enqueue_sample(c, sd, n0, c->kind, k, L, seed, epoch, batch);
+  if (s != GLB_OK) return s;
+  return glb_sample_result(c, out);
+}
+
+glb_status glb_sample_batch(glb_ctx* c, uint32_t epoch, uint32_t b) {
+  ENTER(c);
+  if (!c->V || !c->sampler_set || !c->train_set) return set_err(c, GLB_ESTATE, "sample_batch needs graph, sampler, train set");
+  const uint64_t nb = (c->n_train + c->batch_size - 1) / c->batch_size;
+  if (b >= nb) return set_err(c, GLB_EINVAL, "batch %u >= %llu", b, (unsigned long long)nb);
+  if (epoch > 0xFFFFu) return set_err(c, GLB_ERANGE, "epoch %u >= 2^16", epoch);
+  glb_status s = ensure_perm(c, epoch);
+  if (s != GLB_OK) return s;
+  const uint64_t lo = (uint64_t)b * c->batch_size;
+  const uint64_t hi = lo + c->batch_size < c->n_train ? lo + c->batch_size : c->n_train;
+  return enqueue_sample(c, c->perm + lo, (uint32_t)(hi - lo), c->kind, c->fanouts, c->L, c->seed,
+                        epoch, b);
+}
+
+glb_status glb_set_count_mode(glb_ctx* c, int mode) {
+  ENTER(c);
+  if (mode < GLB_COUNT_NONE || mode > GLB_COUNT_ACCESS) return set_err(c, GLB_EINVAL, "bad count mode");
+  c->count_mode = mode;
+  return GLB_OK;
+}
+
+glb_status glb_reset_counts(glb_ctx* c, int which) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "no graph");
+  uint32_t* p = which == GLB_COUNT_PRESAMPLE ? c->counts : which == GLB_COUNT_ACCESS ? c->access : nullptr;
+  if (!p) return set_err(c, GLB_EINVAL, "bad count target");
+  CK(cudaMemsetAsync(p, 0, sizeof(uint32_t) * c->V, c->stream));
+  return GLB_OK;
+}
+
+glb_status glb_presample(glb_ctx* c, uint32_t K, uint32_t rank, uint32_t world) {
+  ENTER(c);
+  if (!c->V || !c->sampler_set || !c->train_set) return set_err(c, GLB_ESTATE, "presample needs graph, sampler, train set");
+  if (world == 0 || rank >= world) return set_err(c, GLB_EINVAL, "bad rank/world");
+  const int saved = c->count_mode;
+  c->count_mode = GLB_COUNT_PRESAMPLE;
+  const uint32_t nb = (uint32_t)((c->n_train + c->batch_size - 1) / c->batch_size);
+  glb_status s = GLB_OK;
+  for (uint32_t e = 0; e < K && s == GLB_OK; ++e)
+    for (uint32_t b = rank; b < nb && s == GLB_OK; b += world) s = glb_sample_batch(c, e, b);
+  c->count_mode = saved;
+  if (s != GLB_OK) return s;
+  c->have_sample = false;
+  return check_dev_err(c, c->st);
+}
+
+glb_status glb_counts_device_ptr(glb_ctx* c, int which, void** out) {
+  ENTER(c);
+  if (!out) return set_err(c, GLB_EINVAL, "null out");
+  *out = which == GLB_COUNT_PRESAMPLE ? (void*)c->counts : which == GLB_COUNT_ACCESS ? (void*)c->access : nullptr;
+  return *out ? GLB_OK : set_err(c, GLB_EINVAL, "bad count target");
+}
+
+glb_status glb_get_counts(glb_ctx* c, int which, uint32_t* host_out) {
+  void* p = nullptr;
+  glb_status s = glb_counts_device_ptr(c, which, &p);
+  if (s != GLB_OK) return s;
+  CK(cudaMemcpyAsync(host_out, p, sizeof(uint32_t) * c->V, cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  return GLB_OK;
+}
+
+glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "build_cache before load_graph");
+  if (!(alpha >= 0.0 && alpha <= 1.0)) return set_err(c, GLB_EINVAL, "alpha %g not in [0,1]", alpha);
+  const uint64_t V = c->V;
+  uint64_t C = (uint64_t)std::floor(alpha * (double)V);
+  if (C > V) C = V;
+  const uint32_t* hot = hotness ? hotness : c->counts;
+  uint32_t* tmp = nullptr;
+  CK(dalloc(&tmp, 4 * V));
+  uint32_t *k0 = tmp, *v0 = tmp + V, *k1 = tmp + 2 * V, *v1 = tmp + 3 * V;
+  uint32_t* dmax = (uint32_t*)c->scratch;
+  CK(cudaMemsetAsync(dmax, 0, sizeof(uint32_t), c->stream));
+  CK(launch_max_u32(c, hot, V, dmax));
+  uint32_t maxc = 0;
+  CK(cudaMemcpyAsync(&maxc, dmax, sizeof(uint32_t), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  int bits = 0;
+  while (bits < 32 && (maxc >> bits)) ++bits;
+  CK(launch_rank_keys(c, hot, maxc, k0, v0));
+  uint32_t *ko = nullptr, *order = nullptr;
+  CK(radix_sort_pairs_u32(c, k0, v0, k1, v1, V, bits, &ko, &order));
+  CK(cudaMemsetAsync(c->slot, 0xFF, sizeof(int32_t) * V, c->stream));
+  CK(launch_assign_slots(c, order, C));
+  dfree(c->cache);
+  c->C = C;
+  if (c->features_mapped && C) {
+    CK(dalloc(&c->cache, C * (uint64_t)c->D));
+    // cache rows come over PCIe from the mapped host matrix (zero copy)
+    CK(launch_gather(c, c->cache, nullptr, c->features_mapped, nullptr, nullptr, nullptr, order,
+                     nullptr, 0, C));
+  }
+  CK(cudaStreamSynchronize(c->stream));
+  cudaFree(tmp);
+  c->have_sample = false;  // marks of an earlier sample refer to the old cache
+  return GLB_OK;
+}
+
+glb_status glb_get_cache_slots(glb_ctx* c, int32_t* host_out) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "no graph");
+  CK(cudaMemcpyAsync(host_out, c->slot, sizeof(int32_t) * c->V, cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  return GLB_OK;
+}
+
+glb_status glb_cache_size(const glb_ctx* c, uint64_t* out) {
+  if (!c || !out) return GLB_EINVAL;
+  *out = c->C;
+  return GLB_OK;
+}
+
+glb_status glb_hit_stats_get(glb_ctx* c, glb_hit_stats* out) {
+  ENTER(c);
+  if (!c->V || !out) return set_err(c, GLB_ESTATE, "no graph");
+  unsigned long long h3[3];
+  CK(cudaMemsetAsync(c->scratch, 0, 3 * sizeof(unsigned long long), c->stream));
+  CK(launch_hit_stats(c, c->scratch));
+  CK(cudaMemcpyAsync(h3, c->scratch, sizeof(h3), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  out->total = h3[0];
+  out->hits = h3[1];
+  out->cache_rows = c->C;
+  const uint32_t mx = (uint32_t)h3[2];
+  unsigned long long* bins = nullptr;
+  CK(dalloc(&bins, (uint64_t)mx + 1));
+  CK(cudaMemsetAsync(bins, 0, sizeof(unsigned long long) * ((uint64_t)mx + 1), c->stream));
+  CK(launch_value_hist(c, c->access, c->V, bins, mx + 1));
+  unsigned long long* hb = new (std::nothrow) unsigned long long[(uint64_t)mx + 1];
+  if (!hb) { cudaFree(bins); return set_err(c, GLB_ENOMEM, "host alloc"); }
+  CK(cudaMemcpyAsync(hb, bins, sizeof(unsigned long long) * ((uint64_t)mx + 1), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  cudaFree(bins);
+  // Optimal policy: the C largest access counts (L148 fn4)
+  uint64_t left = c->C, opt = 0;
+  for (uint64_t x = mx; x >= 1 && left; --x) {
+    const uint64_t take = hb[x] < left ? hb[x] : left;
+    opt += take * x;
+    left -= take;
+  }
+  delete[] hb;
+  out->optimal_hits = opt;
+  return GLB_OK;
+}
+
+glb_status glb_extract(glb_ctx* c, const uint32_t* vertices, uint64_t n, void* out,
+                       glb_extract_stats* stats) {
+  ENTER(c);
+  if (!c->V || !c->features_mapped) return set_err(c, GLB_ESTATE, "extract needs a graph with features");
+  if (n && (!vertices || !out)) return set_err(c, GLB_EINVAL, "null pointer");
+  if (n >= 0xFFFFFFFFull) return set_err(c, GLB_EINVAL, "n too large");
+  if (n > c->xb.cap) {
+    CK(cudaStreamSynchronize(c->stream));
+    dfree(c->xb.hit_dst); dfree(c->xb.hit_src); dfree(c->xb.miss_dst); dfree(c->xb.miss_src);
+    c->xb.cap = 0;
+    CK(dalloc(&c->xb.hit_dst, n));
+    CK(dalloc(&c->xb.hit_src, n));
+    CK(dalloc(&c->xb.miss_dst, n));
+    CK(dalloc(&c->xb.miss_src, n));
+    c->xb.cap = n;
+  }
+  CK(cudaMemsetAsync(&c->st_x->nhit, 0, 2 * sizeof(uint32_t), c->stream));
+  if (n) CK(launch_mark(c, vertices, n));
+  CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->xb.hit_dst, c->xb.hit_src,
+                   c->xb.miss_dst, c->xb.miss_src, &c->st_x->nhit, 0, 0));
+  if (stats) {
+    CK(cudaMemcpyAsync(c->h_xcount, c->xcount, 2 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
+    c->pending_stats = stats;
+  }
+  return GLB_OK;
+}
+
+glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
+  ENTER(c);
+  if (!c->have_sample) return set_err(c, GLB_ESTATE, "extract_sample without a current sample");
+  if (!c->features_mapped) return set_err(c, GLB_ESTATE, "graph loaded without features");
+  if (!out) return set_err(c, GLB_EINVAL, "null out");
+  CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_dst, c->sb.hit_src,
+                   c->sb.miss_dst, c->sb.miss_src, &c->st->nhit, 0, 0));
+  if (stats) {
+    CK(cudaMemcpyAsync(c->h_xcount, c->xcount, 2 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
+    c->pending_stats = stats;
+  }
+  return GLB_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,210 @@
+// glb_internal.cuh -- internal declarations of the B200 sample+extract library.
+// Not part of the ABI (see include/glb.h).  Shares nothing with oracle/.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "glb.h"
+
+namespace glb {
+
+constexpr uint32_t kEmpty = 0xFFFFFFFFu;
+constexpr int kThreads = 256;          // block size of every grid-stride kernel
+constexpr int kCompactItems = 8;       // flat positions per thread in a compaction tile
+constexpr int kCompactTile = kThreads * kCompactItems;
+constexpr int kMaxFanout = 1024;
+constexpr int kMaxWalkLen = 8;
+
+// RNG domains (reading Q4): counter word 3 = epoch<<16 | hop<<8 | domain
+enum : uint32_t { kDomShuffle = 1, kDomKhop = 2, kDomRwalk = 3 };
+
+// device error bits (DevState::err)
+enum : uint32_t { kErrDupSeed = 1u, kErrRange = 2u, kErrCapacity = 4u, kErrBadGraph = 8u };
+
+// Per-batch device state.  Sizes live here so no kernel needs a host sync.
+struct DevState {
+  uint32_t n[GLB_MAX_HOPS + 1];     // frontier sizes n_0..n_L
+  uint32_t nnz[GLB_MAX_HOPS];       // block edge counts
+  uint32_t base[GLB_MAX_HOPS + 1];  // first flat position of hop l (relabel order)
+  uint32_t tile_ctr[GLB_MAX_HOPS];  // dynamic tile ids of the compaction scans
+  uint32_t nhit, nmiss;             // extract work lists (marks)
+  uint32_t err;
+  uint32_t pad;
+};
+
+// Counter-based RNG: Philox4x32-10 (Random123 constants).
+__device__ __forceinline__ uint4 philox10(uint4 c, uint32_t k0, uint32_t k1) {
+#pragma unroll
+  for (int r = 0; r < 10; ++r) {
+    if (r) {
+      k0 += 0x9E3779B9u;
+      k1 += 0xBB67AE85u;
+    }
+    const uint32_t hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
+    const uint32_t hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
+    c = make_uint4(hi1 ^ c.y ^ k0, lo1, hi0 ^ c.w ^ k1, lo0);
+  }
+  return c;
+}
+__device__ __forceinline__ uint32_t ctr3(uint32_t epoch, uint32_t hop, uint32_t dom) {
+  return ((epoch & 0xFFFFu) << 16) | ((hop & 0xFFu) << 8) | (dom & 0xFFu);
+}
+__device__ __forceinline__ uint64_t draw64(uint64_t seed, uint32_t c0, uint32_t c1, uint32_t c2,
+                                           uint32_t c3, uint32_t half) {
+  const uint4 w = philox10(make_uint4(c0, c1, c2, c3), (uint32_t)seed, (uint32_t)(seed >> 32));
+  return half ? (((uint64_t)w.w << 32) | w.z) : (((uint64_t)w.y << 32) | w.x);
+}
+// floor(r * n / 2^64)
+__device__ __forceinline__ uint32_t bounded(uint64_t r, uint32_t n) {
+  return (uint32_t)__umul64hi(r, (uint64_t)n);
+}
+
+// Relabel table entry: ((0xFFFFFFFF - gen) << 32) | position.  Within one
+// generation atomicMin keeps the first position; a newer generation is always
+// smaller, so stale entries never need clearing.
+__device__ __forceinline__ uint64_t enc_pos(uint32_t gen, uint32_t pos) {
+  return ((uint64_t)(0xFFFFFFFFu - gen) << 32) | pos;
+}
+
+struct SampleBufs {
+  uint32_t cap_batch = 0;
+  uint32_t L = 0;
+  uint64_t ub[GLB_MAX_HOPS + 1] = {};
+  uint32_t k[GLB_MAX_HOPS] = {};      // slots per frontier vertex (fanout or topk)
+  uint32_t* seeds = nullptr;          // u32[cap_batch]
+  uint32_t* uniq = nullptr;           // u32[ub[L]]
+  int32_t* lidslot = nullptr;         // i32[ub[L]]  (a4 marks)
+  uint32_t* picks = nullptr;          // u32[max ub[l]*k[l]]
+  uint32_t* pickw = nullptr;          // u32[...] random-walk counts
+  uint32_t* bindptr[GLB_MAX_HOPS] = {};
+  uint32_t* bindices[GLB_MAX_HOPS] = {};
+  uint32_t* bweights[GLB_MAX_HOPS] = {};
+  unsigned long long* status[GLB_MAX_HOPS] = {};
+  uint64_t ntiles[GLB_MAX_HOPS] = {};
+  uint32_t* hit_dst = nullptr;        // extract work lists
+  uint32_t* hit_src = nullptr;
+  uint32_t* miss_dst = nullptr;
+  uint32_t* miss_src = nullptr;
+};
+
+struct ExtractBufs {
+  uint64_t cap = 0;
+  uint32_t* hit_dst = nullptr;
+  uint32_t* hit_src = nullptr;
+  uint32_t* miss_dst = nullptr;
+  uint32_t* miss_src = nullptr;
+};
+
+}  // namespace glb
+
+struct glb_ctx {
+  int device = 0;
+  cudaStream_t own_stream = nullptr;
+  cudaStream_t stream = nullptr;
+  int num_sms = 148;
+  bool poisoned = false;
+  std::string err;
+  uint64_t launches = 0;
+
+  // graph (D1, D2)
+  uint64_t V = 0, E = 0;
+  uint64_t* indptr = nullptr;
+  uint32_t* indices = nullptr;
+  const void* h_features = nullptr;
+  const float* features_mapped = nullptr;  // device alias of the registered host matrix
+  bool registered = false;
+  uint32_t D = 0;
+
+  // relabel tables (D6): direct-address over gids
+  unsigned long long* vmap = nullptr;  // u64[V]
+  uint32_t* lidmap = nullptr;          // u32[V]
+  uint32_t gen = 0;
+
+  // cache (D3, D4, D5)
+  int32_t* slot = nullptr;     // i32[V]
+  float* cache = nullptr;      // f32[C][D]
+  uint64_t C = 0;
+  uint32_t* counts = nullptr;  // u32[V] PreSC hotness
+  uint32_t* access = nullptr;  // u32[V] measured accesses
+  int count_mode = GLB_COUNT_NONE;
+
+  // sampler config
+  bool sampler_set = false;
+  int kind = GLB_KHOP_UNIFORM;
+  uint32_t L = 0;
+  uint32_t fanouts[GLB_MAX_HOPS] = {};
+  uint32_t rw_walks = 4, rw_len = 3, rw_topk = 5;
+  glb::SampleBufs sb;
+  glb::ExtractBufs xb;
+
+  // training set (D9)
+  uint32_t* train = nullptr;
+  uint32_t* perm = nullptr;
+  uint64_t n_train = 0;
+  uint32_t batch_size = 0;
+  uint64_t seed = 0;
+  bool train_set = false;
+  int perm_epoch = -1;
+
+  // last sample
+  bool have_sample = false;
+  uint32_t last_L = 0;
+  uint32_t last_k[GLB_MAX_HOPS] = {};
+  int last_kind = 0;
+  uint32_t last_n0 = 0;
+
+  glb::DevState* st = nullptr;    // device: current sample
+  glb::DevState* h_st = nullptr;  // pinned mirror
+  glb::DevState* st_x = nullptr;  // device: generic glb_extract (mark lists, errors)
+  unsigned long long* scratch = nullptr;  // device [4] u64 reductions
+  // shuffle scratch
+  unsigned long long* shuf_keys = nullptr;
+  uint32_t* shuf_vals = nullptr;
+  glb_extract_stats* pending_stats = nullptr;
+  unsigned long long* xcount = nullptr;      // device [2] hits/misses of the last extract
+  unsigned long long* h_xcount = nullptr;    // pinned mirror
+
+  // radix sort scratch
+  void* sort_tmp = nullptr;
+  size_t sort_tmp_bytes = 0;
+};
+
+namespace glb {
+
+// ---- launchers (defined in the .cu files) ----
+cudaError_t launch_validate_graph(glb_ctx* c);
+cudaError_t launch_seed_init(glb_ctx* c, const uint32_t* seeds, uint32_t n0, int count_mode);
+cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch,
+                        uint32_t batch);
+cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch, uint32_t batch);
+cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, int count_mode);
+cudaError_t launch_remap(glb_ctx* c, uint32_t hop);
+cudaError_t launch_mark(glb_ctx* c, const uint32_t* vertices, uint64_t n);
+cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const float* src_miss,
+                          const uint32_t* hit_dst, const uint32_t* hit_src,
+                          const uint32_t* miss_dst, const uint32_t* miss_src,
+                          const uint32_t* dev_counts /* [nhit, nmiss] on device or null */,
+                          uint64_t nhit_host, uint64_t nmiss_host);
+cudaError_t launch_shuffle_keys(glb_ctx* c, uint32_t epoch, unsigned long long* keys, uint32_t* vals);
+cudaError_t radix_sort_pairs_u64(glb_ctx* c, unsigned long long* keys, uint32_t* vals,
+                                 unsigned long long* keys_alt, uint32_t* vals_alt, uint64_t n,
+                                 int bits, unsigned long long** keys_out, uint32_t** vals_out);
+cudaError_t radix_sort_pairs_u32(glb_ctx* c, uint32_t* keys, uint32_t* vals, uint32_t* keys_alt,
+                                 uint32_t* vals_alt, uint64_t n, int bits, uint32_t** keys_out,
+                                 uint32_t** vals_out);
+cudaError_t launch_permute(glb_ctx* c, const uint32_t* table, const uint32_t* idx, uint64_t n,
+                           uint32_t* out);
+cudaError_t launch_max_u32(glb_ctx* c, const uint32_t* a, uint64_t n, uint32_t* out_dev);
+cudaError_t launch_rank_keys(glb_ctx* c, const uint32_t* hot, uint32_t maxc, uint32_t* keys,
+                             uint32_t* vals);
+cudaError_t launch_assign_slots(glb_ctx* c, const uint32_t* order, uint64_t C);
+cudaError_t launch_hit_stats(glb_ctx* c, unsigned long long* out3 /* total,hits,max */);
+cudaError_t launch_value_hist(glb_ctx* c, const uint32_t* a, uint64_t n, unsigned long long* bins,
+                              uint32_t nbins);
+
+inline void count_launch(glb_ctx* c, int n = 1) { c->launches += (uint64_t)n; }
+
+}  // namespace glb

@@ -1,0 +1,598 @@
+// sample.cu -- a2 (k-hop uniform), a2' (random walk), a3 (dedup + relabel into
+// blocks) and a4 (mark) for sm_100a.
+//
+// Paper: k-hop sampling "uniformly selects ... neighbors for each vertex"
+// (§2, Fig 7), "a variant of the Fisher-Yates
+// algorithm ... GPU-friendly since the workload is more balanced for each
+// vertex" (L410 §7.3); samples are "deduplicated and reassigned with
+// consecutive IDs (starting from 0)" (L67, L250 §5.2); cached vertices are
+// marked during Sample (L252).
+//
+// Design:
+//  * k_khop: G lanes per frontier vertex (G = next_pow2(fanout) <= 32), one
+//    lane per slot.  Floyd's draws are independent per slot (counter-based
+//    RNG), so every lane computes its t_s at once; the sequential "t already
+//    chosen?" test is resolved exactly with __match_any_sync + a short
+//    fixed-point over the j-chain (proof in DESIGN.md).
+//  * relabel: direct-address table vmap[gid] = (~gen << 32 | first position),
+//    one atomicMin per pick (filtered by a plain read and a warp match), then a
+//    single-pass decoupled-look-back scan over the padded (vertex, slot) array
+//    assigns new lids in first-occurrence order and builds the block CSR.
+#include <cuda_runtime.h>
+
+#include "glb_internal.cuh"
+
+namespace glb {
+
+namespace {
+
+constexpr unsigned kFull = 0xFFFFFFFFu;
+
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+
+// Warp-aggregated append of (dst, src) to a list whose length lives at *ctr.
+__device__ __forceinline__ void warp_append(bool pred, uint32_t* ctr, uint32_t* dst_list,
+                                            uint32_t* src_list, uint32_t dst, uint32_t src) {
+  const uint32_t m = __ballot_sync(kFull, pred);
+  if (!m) return;
+  const int lane = threadIdx.x & 31;
+  const int leader = __ffs(m) - 1;
+  uint32_t base = 0;
+  if (lane == leader) base = atomicAdd(ctr, (uint32_t)__popc(m));
+  base = __shfl_sync(kFull, base, leader);
+  if (pred) {
+    const uint32_t r = base + __popc(m & lanemask_lt());
+    dst_list[r] = dst;
+    src_list[r] = src;
+  }
+}
+
+// Insert one pick into the relabel table: keep the smallest position of this
+// generation.  Values only decrease over time, so a (possibly stale) read that
+// is already <= e proves the atomic would be a no-op.
+__device__ __forceinline__ void vmap_insert(unsigned long long* vmap, uint32_t u,
+                                            unsigned long long e) {
+  const unsigned long long old = __ldcg(vmap + u);
+  if (old > e) atomicMin(vmap + u, e);
+}
+
+struct MarkArgs {
+  const int32_t* slot;
+  int32_t* lidslot;
+  uint32_t* hit_dst;
+  uint32_t* hit_src;
+  uint32_t* miss_dst;
+  uint32_t* miss_src;
+  uint32_t* count;  // nullable visit-count target
+};
+
+struct StatusArgs {  // look-back status arrays to clear for this batch
+  unsigned long long* p[GLB_MAX_HOPS];
+  uint32_t n[GLB_MAX_HOPS];
+  uint32_t L;
+};
+
+// ---------------------------------------------------------------- seeds
+__global__ void __launch_bounds__(kThreads)
+    k_seed_init(const uint32_t* __restrict__ seeds, uint32_t n0, uint64_t V, DevState* st,
+                uint32_t* __restrict__ uniq, unsigned long long* vmap, uint32_t* lidmap,
+                uint32_t gen, MarkArgs mk, StatusArgs za) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    st->n[0] = n0;
+    st->base[0] = n0;
+  }
+  const uint32_t stride = gridDim.x * blockDim.x;
+  for (uint32_t l = 0; l < za.L; ++l)
+    for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < za.n[l]; i += stride) za.p[l][i] = 0ull;
+  // warp-uniform loop bound so that warp_append's ballots see the whole warp
+  for (uint32_t i0 = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); i0 < n0; i0 += stride) {
+    const uint32_t i = i0 + (threadIdx.x & 31);
+    bool act = i < n0;
+    uint32_t u = 0;
+    int32_t s = -1;
+    if (act) {
+      u = seeds[i];
+      if (u >= V) {
+        atomicOr(&st->err, kErrRange);
+        u = 0;  // keep later kernels in bounds; the batch is reported invalid
+      }
+      uniq[i] = u;
+      atomicMin(vmap + u, enc_pos(gen, i));
+      lidmap[u] = i;
+      s = __ldg(mk.slot + u);
+      mk.lidslot[i] = s;
+      if (mk.count) atomicAdd(mk.count + u, 1u);
+    }
+    warp_append(act && s >= 0, &st->nhit, mk.hit_dst, mk.hit_src, i, (uint32_t)s);
+    warp_append(act && s < 0, &st->nmiss, mk.miss_dst, mk.miss_src, i, u);
+  }
+}
+
+// ---------------------------------------------------------------- k-hop (G lanes / vertex)
+template <int G>
+__global__ void __launch_bounds__(kThreads)
+    k_khop(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch, uint32_t gen,
+           const DevState* __restrict__ st, DevState* st_w, const uint64_t* __restrict__ indptr,
+           const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
+           unsigned long long* vmap, uint32_t* __restrict__ picks) {
+  const uint32_t n_l = st->n[hop];
+  const uint32_t base = st->base[hop];
+  const uint32_t c3 = ctr3(epoch, hop, kDomKhop);
+  const int lane = threadIdx.x & 31;
+  const uint32_t s = lane & (G - 1);
+  const int gbase = lane & ~(G - 1);
+  constexpr uint32_t kGroupsPerWarp = 32 / G;
+  const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t w0 = warp_global * kGroupsPerWarp; w0 < n_l; w0 += nwarps * kGroupsPerWarp) {
+    const uint32_t d = w0 + lane / G;
+    const bool active = d < n_l;
+    uint32_t v = 0, deg = 0;
+    uint64_t lo = 0;
+    if (active) {
+      v = uniq[d];
+      lo = indptr[v];
+      deg = (uint32_t)(indptr[v + 1] - lo);
+      if (hop == 0 && s == 0 && __ldcg(vmap + v) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
+    }
+    const bool big = active && deg > k;
+    const bool part = big && s < k;  // lane draws a Floyd candidate
+    uint32_t t = 0, j = 0;
+    if (part) {
+      j = deg - k + s;
+      t = bounded(draw64(seed, v, s >> 1, batch, c3, s & 1u), j + 1);
+    }
+    // D1: an earlier slot of the same vertex drew the same t
+    const unsigned long long key =
+        part ? (((unsigned long long)(lane / G) << 32) | t) : ((1ull << 63) | (unsigned)lane);
+    const uint32_t eq = __match_any_sync(kFull, key);
+    const bool d1 = (eq & lanemask_lt()) != 0;
+    // j-chain: t equals j_{s'} (s' < s), which is taken iff slot s' was displaced
+    const bool inr = part && t >= deg - k && t < j;
+    const int ref = inr ? gbase + (int)(t - (deg - k)) : lane;
+    bool disp = d1;
+    for (;;) {
+      const bool r = __shfl_sync(kFull, disp, ref);
+      const bool nd = d1 || (inr && r);
+      const bool done = __ballot_sync(kFull, nd) == __ballot_sync(kFull, disp);
+      disp = nd;
+      if (done) break;
+    }
+    uint32_t sel = kEmpty;
+    if (big) {
+      if (s < k) sel = disp ? j : t;
+    } else if (active && s < deg) {
+      sel = s;
+    }
+    uint32_t u = kEmpty;
+    if (sel != kEmpty) u = __ldg(indices + lo + sel);
+    if (active && s < k) picks[(size_t)d * k + s] = u;
+    // one atomic per distinct gid per warp (lowest lane = smallest position)
+    const unsigned long long ukey = (u != kEmpty) ? (unsigned long long)u : ((1ull << 32) | (unsigned)lane);
+    const uint32_t peers = __match_any_sync(kFull, ukey);
+    if (u != kEmpty && (peers & lanemask_lt()) == 0)
+      vmap_insert(vmap, u, enc_pos(gen, base + d * k + s));
+  }
+}
+
+// Fanout > 32: one warp per vertex, Floyd run sequentially by lane 0 in shared memory.
+__global__ void __launch_bounds__(kThreads)
+    k_khop_wide(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch,
+                uint32_t gen, const DevState* __restrict__ st, DevState* st_w,
+                const uint64_t* __restrict__ indptr, const uint32_t* __restrict__ indices,
+                const uint32_t* __restrict__ uniq, unsigned long long* vmap,
+                uint32_t* __restrict__ picks) {
+  __shared__ uint32_t chosen[kThreads / 32][kMaxFanout];
+  const uint32_t n_l = st->n[hop];
+  const uint32_t base = st->base[hop];
+  const uint32_t c3 = ctr3(epoch, hop, kDomKhop);
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5;
+  const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  uint32_t* ch = chosen[wib];
+  for (uint32_t d = warp_global; d < n_l; d += nwarps) {
+    const uint32_t v = uniq[d];
+    const uint64_t lo = indptr[v];
+    const uint32_t deg = (uint32_t)(indptr[v + 1] - lo);
+    if (hop == 0 && lane == 0 && __ldcg(vmap + v) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
+    if (deg > k) {
+      if (lane == 0) {
+        for (uint32_t s = 0; s < k; ++s) {
+          const uint32_t j = deg - k + s;
+          const uint32_t t = bounded(draw64(seed, v, s >> 1, batch, c3, s & 1u), j + 1);
+          bool taken = false;
+          for (uint32_t q = 0; q < s; ++q) taken |= (ch[q] == t);
+          ch[s] = taken ? j : t;
+        }
+      }
+      __syncwarp();
+    }
+    for (uint32_t s = lane; s < k; s += 32) {
+      uint32_t sel = kEmpty;
+      if (deg > k) sel = ch[s];
+      else if (s < deg) sel = s;
+      const uint32_t u = sel != kEmpty ? __ldg(indices + lo + sel) : kEmpty;
+      picks[(size_t)d * k + s] = u;
+      if (u != kEmpty) vmap_insert(vmap, u, enc_pos(gen, base + d * k + s));
+    }
+    __syncwarp();
+  }
+}
+
+// ---------------------------------------------------------------- random walk
+// PinSAGE (L209, L353): G >= walks lanes per frontier vertex, one walk per lane.
+template <int G>
+__global__ void __launch_bounds__(kThreads)
+    k_rwalk(uint32_t hop, uint32_t walks, uint32_t len, uint32_t topk, uint64_t seed,
+            uint32_t epoch, uint32_t batch, uint32_t gen, const DevState* __restrict__ st,
+            DevState* st_w, const uint64_t* __restrict__ indptr,
+            const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
+            unsigned long long* vmap, uint32_t* __restrict__ picks, uint32_t* __restrict__ pickw) {
+  const uint32_t n_l = st->n[hop];
+  const uint32_t base = st->base[hop];
+  const uint32_t c3 = ctr3(epoch, hop, kDomRwalk);
+  const int lane = threadIdx.x & 31;
+  const uint32_t w = lane & (G - 1);
+  const int gbase = lane & ~(G - 1);
+  constexpr uint32_t kGroupsPerWarp = 32 / G;
+  const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t w0 = warp_global * kGroupsPerWarp; w0 < n_l; w0 += nwarps * kGroupsPerWarp) {
+    const uint32_t d = w0 + lane / G;
+    const bool active = d < n_l;
+    uint32_t v = 0;
+    uint32_t vis[kMaxWalkLen];
+#pragma unroll
+    for (int t = 0; t < kMaxWalkLen; ++t) vis[t] = kEmpty;
+    if (active) {
+      v = uniq[d];
+      if (hop == 0 && w == 0 && __ldcg(vmap + v) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
+      if (w < walks) {
+        uint32_t cur = v;
+#pragma unroll
+        for (int t = 0; t < kMaxWalkLen; ++t) {
+          if ((uint32_t)t < len) {
+            const uint64_t b = indptr[cur];
+            const uint32_t deg = (uint32_t)(indptr[cur + 1] - b);
+            if (deg == 0) break;
+            const uint64_t r = draw64(seed, v, (w << 8) | ((uint32_t)t >> 1), batch, c3, t & 1);
+            cur = __ldg(indices + b + bounded(r, deg));
+            if (cur != v) vis[t] = cur;
+          }
+        }
+      }
+    }
+    // visit counts and first occurrences over the group's walks*len entries
+    uint32_t cnt[kMaxWalkLen];
+    bool first[kMaxWalkLen];
+#pragma unroll
+    for (int t = 0; t < kMaxWalkLen; ++t) { cnt[t] = 0; first[t] = true; }
+    for (uint32_t src = 0; src < G; ++src) {
+#pragma unroll
+      for (int tt = 0; tt < kMaxWalkLen; ++tt) {
+        const uint32_t x = __shfl_sync(kFull, vis[tt], gbase + src);
+#pragma unroll
+        for (int t = 0; t < kMaxWalkLen; ++t) {
+          if (vis[t] != kEmpty && x == vis[t]) {
+            ++cnt[t];
+            if (src * kMaxWalkLen + tt < w * kMaxWalkLen + t) first[t] = false;
+          }
+        }
+      }
+    }
+    // rank of each distinct visited vertex by (count desc, gid asc)
+    uint32_t rank[kMaxWalkLen];
+    uint32_t ndist = 0;
+#pragma unroll
+    for (int t = 0; t < kMaxWalkLen; ++t) rank[t] = 0;
+    for (uint32_t src = 0; src < G; ++src) {
+#pragma unroll
+      for (int tt = 0; tt < kMaxWalkLen; ++tt) {
+        const uint32_t x = __shfl_sync(kFull, vis[tt], gbase + src);
+        const uint32_t xc = __shfl_sync(kFull, cnt[tt], gbase + src);
+        const bool xf = __shfl_sync(kFull, first[tt], gbase + src);
+        if (x != kEmpty && xf) {
+          ++ndist;
+#pragma unroll
+          for (int t = 0; t < kMaxWalkLen; ++t)
+            if (vis[t] != kEmpty && first[t] && (xc > cnt[t] || (xc == cnt[t] && x < vis[t])))
+              ++rank[t];
+        }
+      }
+    }
+    if (active) {
+      for (uint32_t r = w; r < topk; r += G)
+        if (r >= ndist) picks[(size_t)d * topk + r] = kEmpty;
+#pragma unroll
+      for (int t = 0; t < kMaxWalkLen; ++t) {
+        if (vis[t] != kEmpty && first[t] && rank[t] < topk) {
+          const uint32_t f = d * topk + rank[t];
+          picks[f] = vis[t];
+          pickw[f] = cnt[t];
+          vmap_insert(vmap, vis[t], enc_pos(gen, base + f));
+        }
+      }
+    }
+  }
+}
+
+// ---------------------------------------------------------------- compaction scan
+// Status word of the decoupled look-back: [flag:2][new:31][valid:31].
+constexpr unsigned long long kFlagAgg = 1ull << 62;
+constexpr unsigned long long kFlagInc = 2ull << 62;
+constexpr unsigned long long kValMask = (1ull << 62) - 1;
+
+__device__ __forceinline__ unsigned long long pack_status(unsigned long long flag,
+                                                          unsigned long long pair) {
+  // pair = new << 32 | valid
+  return flag | ((pair >> 32) << 31) | (pair & 0x7FFFFFFFull);
+}
+__device__ __forceinline__ unsigned long long unpack_pair(unsigned long long w) {
+  w &= kValMask;
+  return ((w >> 31) << 32) | (w & 0x7FFFFFFFull);
+}
+
+__device__ __forceinline__ unsigned long long warp_incl_scan64(unsigned long long x) {
+  const int lane = threadIdx.x & 31;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long y = __shfl_up_sync(kFull, x, o);
+    if (lane >= o) x += y;
+  }
+  return x;
+}
+__device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(kFull, x, o);
+  return x;
+}
+
+template <bool W>
+__global__ void __launch_bounds__(kThreads)
+    k_compact(uint32_t hop, uint32_t k, uint32_t gen, DevState* st,
+              const uint32_t* __restrict__ picks, const uint32_t* __restrict__ pickw,
+              const unsigned long long* __restrict__ vmap, uint32_t* __restrict__ lidmap,
+              uint32_t* __restrict__ uniq, uint32_t* __restrict__ bindptr,
+              uint32_t* __restrict__ bindices, uint32_t* __restrict__ bweights,
+              unsigned long long* status, MarkArgs mk) {
+  __shared__ uint32_t s_tile;
+  __shared__ unsigned long long s_warp[kThreads / 32];
+  __shared__ unsigned long long s_excl;
+  const uint32_t n_l = st->n[hop];
+  const uint32_t base = st->base[hop];
+  const uint32_t flat = n_l * k;
+  const uint32_t ntiles = (flat + kCompactTile - 1) / kCompactTile;
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  if (flat == 0) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      st->n[hop + 1] = n_l;
+      st->nnz[hop] = 0;
+      st->base[hop + 1] = base;
+      bindptr[n_l] = 0;
+      if (n_l == 0) bindptr[0] = 0;
+    }
+    return;
+  }
+  for (;;) {
+    if (threadIdx.x == 0) s_tile = atomicAdd(&st->tile_ctr[hop], 1u);
+    __syncthreads();
+    const uint32_t tile = s_tile;
+    if (tile >= ntiles) break;
+    const uint32_t f0 = tile * kCompactTile + threadIdx.x * kCompactItems;
+    uint32_t u[kCompactItems];
+    uint32_t flags = 0;  // bit i: valid, bit 16+i: new
+#pragma unroll
+    for (int i = 0; i < kCompactItems; ++i) {
+      const uint32_t f = f0 + i;
+      u[i] = f < flat ? picks[f] : kEmpty;
+    }
+#pragma unroll
+    for (int i = 0; i < kCompactItems; ++i) {
+      if (u[i] != kEmpty) {
+        flags |= 1u << i;
+        if (__ldg(vmap + u[i]) == enc_pos(gen, base + f0 + i)) flags |= 1u << (16 + i);
+      }
+    }
+    const unsigned long long mine =
+        ((unsigned long long)__popc(flags >> 16) << 32) | (unsigned)__popc(flags & 0xFFFFu);
+    // block exclusive scan of (new, valid)
+    const unsigned long long incl = warp_incl_scan64(mine);
+    if (lane == 31) s_warp[wid] = incl;
+    __syncthreads();
+    if (wid == 0) {
+      unsigned long long x = lane < kThreads / 32 ? s_warp[lane] : 0ull;
+      const unsigned long long xi = warp_incl_scan64(x);
+      if (lane < kThreads / 32) s_warp[lane] = xi - x;  // exclusive warp offsets
+      const unsigned long long agg = __shfl_sync(kFull, xi, kThreads / 32 - 1);
+      // decoupled look-back
+      unsigned long long excl = 0;
+      if (tile == 0) {
+        if (lane == 0) atomicExch(status + 0, pack_status(kFlagInc, agg));
+      } else {
+        if (lane == 0) atomicExch(status + tile, pack_status(kFlagAgg, agg));
+        long long idx = (long long)tile - 1;
+        for (;;) {
+          const long long jx = idx - lane;
+          unsigned long long wv = kFlagInc;
+          if (jx >= 0) {
+            do {
+              wv = *((volatile unsigned long long*)(status + jx));
+            } while ((wv >> 62) == 0);
+          }
+          const uint32_t incm = __ballot_sync(kFull, (wv >> 62) == 2);
+          if (incm) {
+            const int firsti = __ffs(incm) - 1;
+            excl += warp_sum64(lane <= firsti ? unpack_pair(wv) : 0ull);
+            break;
+          }
+          excl += warp_sum64(unpack_pair(wv));
+          idx -= 32;
+        }
+        if (lane == 0) atomicExch(status + tile, pack_status(kFlagInc, excl + agg));
+      }
+      if (lane == 0) {
+        s_excl = excl;
+        if (tile == ntiles - 1) {
+          const unsigned long long tot = excl + agg;
+          const uint32_t nnew = (uint32_t)(tot >> 32), nval = (uint32_t)tot;
+          st->n[hop + 1] = n_l + nnew;
+          st->nnz[hop] = nval;
+          st->base[hop + 1] = base + flat;
+          bindptr[n_l] = nval;
+        }
+      }
+    }
+    __syncthreads();
+    unsigned long long run = s_excl + s_warp[wid] + (incl - mine);
+    uint32_t d = f0 / k, s = f0 - d * k;
+#pragma unroll
+    for (int i = 0; i < kCompactItems; ++i) {
+      const uint32_t f = f0 + i;
+      const uint32_t ev = (uint32_t)run, en = (uint32_t)(run >> 32);
+      const bool valid = (flags >> i) & 1u;
+      const bool isnew = (flags >> (16 + i)) & 1u;
+      if (f < flat) {
+        if (s == 0) bindptr[d] = ev;
+        if (valid) {
+          bindices[ev] = u[i];  // gid; k_remap turns it into a lid
+          if (W) bweights[ev] = pickw[f];
+        }
+      }
+      int32_t sl = -1;
+      const uint32_t lid = n_l + en;
+      if (isnew) {
+        uniq[lid] = u[i];
+        lidmap[u[i]] = lid;
+        sl = __ldg(mk.slot + u[i]);
+        mk.lidslot[lid] = sl;
+        if (mk.count) atomicAdd(mk.count + u[i], 1u);
+      }
+      warp_append(isnew && sl >= 0, &st->nhit, mk.hit_dst, mk.hit_src, lid, (uint32_t)sl);
+      warp_append(isnew && sl < 0, &st->nmiss, mk.miss_dst, mk.miss_src, lid, u[i]);
+      run += ((unsigned long long)isnew << 32) | (unsigned)valid;
+      if (++s == k) { s = 0; ++d; }
+    }
+    __syncthreads();
+  }
+}
+
+__global__ void __launch_bounds__(kThreads)
+    k_remap(uint32_t hop, const DevState* __restrict__ st, const uint32_t* __restrict__ lidmap,
+            uint32_t* __restrict__ bindices) {
+  const uint32_t nnz = st->nnz[hop];
+  for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x)
+    bindices[e] = __ldg(lidmap + bindices[e]);
+}
+
+__global__ void k_validate(const uint64_t* __restrict__ indptr, const uint32_t* __restrict__ indices,
+                           uint64_t V, uint64_t E, DevState* st) {
+  const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t t0 = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  bool bad = false;
+  for (uint64_t i = t0; i < V; i += stride) bad |= indptr[i + 1] < indptr[i];
+  if (t0 == 0) bad |= indptr[0] != 0 || indptr[V] != E;
+  for (uint64_t e = t0; e < E; e += stride) bad |= indices[e] >= V;
+  if (bad) atomicOr(&st->err, kErrBadGraph);
+}
+
+inline int grid_for(glb_ctx* c, int per_sm = 8) { return c->num_sms * per_sm; }
+
+MarkArgs mark_args(glb_ctx* c, int count_mode) {
+  MarkArgs m;
+  m.slot = c->slot;
+  m.lidslot = c->sb.lidslot;
+  m.hit_dst = c->sb.hit_dst;
+  m.hit_src = c->sb.hit_src;
+  m.miss_dst = c->sb.miss_dst;
+  m.miss_src = c->sb.miss_src;
+  m.count = count_mode == GLB_COUNT_PRESAMPLE ? c->counts
+            : count_mode == GLB_COUNT_ACCESS  ? c->access
+                                              : nullptr;
+  return m;
+}
+
+}  // namespace
+
+cudaError_t launch_validate_graph(glb_ctx* c) {
+  k_validate<<<grid_for(c), kThreads, 0, c->stream>>>(c->indptr, c->indices, c->V, c->E, c->st);
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_seed_init(glb_ctx* c, const uint32_t* seeds, uint32_t n0, int count_mode) {
+  int blocks = (int)((n0 + kThreads - 1) / kThreads);
+  if (blocks < 1) blocks = 1;
+  if (blocks > grid_for(c)) blocks = grid_for(c);
+  StatusArgs za = {};
+  za.L = c->sb.L;
+  for (uint32_t l = 0; l < c->sb.L; ++l) {
+    za.p[l] = c->sb.status[l];
+    za.n[l] = (uint32_t)c->sb.ntiles[l];
+  }
+  k_seed_init<<<blocks, kThreads, 0, c->stream>>>(seeds, n0, c->V, c->st, c->sb.uniq, c->vmap,
+                                                  c->lidmap, c->gen, mark_args(c, count_mode), za);
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch,
+                        uint32_t batch) {
+  const int grid = grid_for(c);
+  const SampleBufs& b = c->sb;
+#define GLB_KHOP_ARGS                                                                  \
+  hop, k, seed, epoch, batch, c->gen, c->st, c->st, c->indptr, c->indices, b.uniq, c->vmap, \
+      b.picks
+  if (k <= 4) k_khop<4><<<grid, kThreads, 0, c->stream>>>(GLB_KHOP_ARGS);
+  else if (k <= 8) k_khop<8><<<grid, kThreads, 0, c->stream>>>(GLB_KHOP_ARGS);
+  else if (k <= 16) k_khop<16><<<grid, kThreads, 0, c->stream>>>(GLB_KHOP_ARGS);
+  else if (k <= 32) k_khop<32><<<grid, kThreads, 0, c->stream>>>(GLB_KHOP_ARGS);
+  else k_khop_wide<<<grid, kThreads, 0, c->stream>>>(GLB_KHOP_ARGS);
+#undef GLB_KHOP_ARGS
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch, uint32_t batch) {
+  const int grid = grid_for(c);
+  const SampleBufs& b = c->sb;
+#define GLB_RW_ARGS                                                                          \
+  hop, c->rw_walks, c->rw_len, c->rw_topk, seed, epoch, batch, c->gen, c->st, c->st, c->indptr, \
+      c->indices, b.uniq, c->vmap, b.picks, b.pickw
+  const uint32_t w = c->rw_walks;
+  if (w <= 1) k_rwalk<1><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
+  else if (w <= 2) k_rwalk<2><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
+  else if (w <= 4) k_rwalk<4><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
+  else if (w <= 8) k_rwalk<8><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
+  else if (w <= 16) k_rwalk<16><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
+  else k_rwalk<32><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
+#undef GLB_RW_ARGS
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, int count_mode) {
+  const SampleBufs& b = c->sb;
+  const int grid = grid_for(c, 4);
+  if (weighted)
+    k_compact<true><<<grid, kThreads, 0, c->stream>>>(
+        hop, k, c->gen, c->st, b.picks, b.pickw, c->vmap, c->lidmap, b.uniq, b.bindptr[hop],
+        b.bindices[hop], b.bweights[hop], b.status[hop], mark_args(c, count_mode));
+  else
+    k_compact<false><<<grid, kThreads, 0, c->stream>>>(
+        hop, k, c->gen, c->st, b.picks, nullptr, c->vmap, c->lidmap, b.uniq, b.bindptr[hop],
+        b.bindices[hop], nullptr, b.status[hop], mark_args(c, count_mode));
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_remap(glb_ctx* c, uint32_t hop) {
+  k_remap<<<grid_for(c), kThreads, 0, c->stream>>>(hop, c->st, c->lidmap, c->sb.bindices[hop]);
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+}  // namespace glb

@@ -1,0 +1,52 @@
+"""CPU-side checks of the C-ABI boundary: the library builds, loads and exports
+every symbol include/glb.h declares; the product package never touches the
+oracle.  No compute calls (no GPU here)."""
+import ctypes
+import os
+import re
+
+import paper_conf_eurosys_yangtswycyz22_b200 as glb
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def header_symbols():
+    src = open(os.path.join(ROOT, "include", "glb.h")).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(glb_[a-z_]+)\s*\(", src)))
+
+
+def test_library_loads_and_exports_every_declared_symbol():
+    so = glb.build()
+    L = ctypes.CDLL(so)
+    syms = header_symbols()
+    assert len(syms) >= 20
+    for s in syms:
+        assert hasattr(L, s), s
+    assert sorted(glb.EXPORTS) == syms
+
+
+def test_sm100a_code_in_library():
+    import subprocess
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", glb.build()],
+                         capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_product_never_imports_oracle():
+    pkg = os.path.join(ROOT, "paper_conf_eurosys_yangtswycyz22_b200")
+    for dp, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h", ".cpp")):
+                txt = open(os.path.join(dp, f)).read()
+                assert not re.search(r"^\s*(import|from)\s+oracle\b", txt, re.M), f
+                assert "oracle.h" not in txt and "liboracle" not in txt, f
+
+
+def test_context_requires_gpu_and_fails_loudly():
+    import pytest
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(glb.GlbError):
+        glb.Context(0)

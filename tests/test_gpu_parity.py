@@ -1,0 +1,303 @@
+"""GPU parity: the CUDA path (through the C-ABI) against the CPU oracle,
+element by element, bit-exact (integer ids, counts, slots; feature bytes).
+
+Sizes: the tiny config (BASELINE configs[0]) everywhere, small power-law
+graphs for ragged tails / wide fanouts / random walks, and the full PR config
+(configs[1]) in the launch configuration bench.py times, on sampled batches
+(first, second, a random one, the last partial one) plus full PreSC counts.
+"""
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+import oracle  # noqa: E402
+import paper_conf_eurosys_yangtswycyz22_b200 as glb  # noqa: E402
+import synth  # noqa: E402
+
+
+def u32(t):
+    return t.cpu().numpy().view(np.uint32)
+
+
+def assert_same_sample(gs, os_, weighted=False):
+    assert gs.sizes == os_.sizes
+    assert np.array_equal(u32(gs.uniq), os_.uniq)
+    for l in range(len(os_.indices)):
+        assert np.array_equal(u32(gs.indptr[l]), os_.indptr[l]), f"indptr hop {l}"
+        assert np.array_equal(u32(gs.indices[l]), os_.indices[l]), f"indices hop {l}"
+        if weighted:
+            assert np.array_equal(u32(gs.weights[l]), os_.weights[l]), f"weights hop {l}"
+
+
+def make_ctx(g, kind="khop", fanouts=(10, 5), max_batch=None, layers=None):
+    ctx = glb.Context(0)
+    ctx.load_graph(g.indptr, g.indices, g.features)
+    ctx.set_sampler(kind, fanouts=fanouts, layers=layers,
+                    max_batch=max_batch or g.shape.batch)
+    ctx.set_train_set(g.train, g.shape.batch, g.seed)
+    return ctx
+
+
+@pytest.fixture(scope="module")
+def tiny():
+    g = synth.make_graph("tiny")
+    return g, oracle.GraphOracle(g.indptr, g.indices, g.features)
+
+
+def test_worked_example_on_gpu():
+    import json
+    import os
+    gold = json.load(open(os.path.join(os.path.dirname(__file__), "golden",
+                                       "survey_worked_example.json")))
+    indptr = np.array(gold["graph"]["indptr"], np.uint64)
+    indices = np.array(gold["graph"]["indices"], np.uint32)
+    feats = synth.gen_features(8, 32, 42)
+    ctx = glb.Context(0)
+    ctx.load_graph(indptr, indices, feats)
+    ctx.set_sampler("khop", fanouts=(3, 2), max_batch=8)
+    s = ctx.sample(np.array([0, 5], np.uint32), seed=42, epoch=0, batch=0)
+    assert u32(s.uniq).tolist() == gold["khop"]["uniq"]
+    for l, b in enumerate(gold["khop"]["blocks"]):
+        assert u32(s.indptr[l]).tolist() == b["indptr"]
+        assert u32(s.indices[l]).tolist() == b["indices"]
+    s = ctx.sample(np.array([0, 5], np.uint32), seed=42, epoch=0, batch=1)
+    assert u32(s.uniq).tolist() == gold["khop"]["uniq_batch1"]
+    ctx.set_sampler("rwalk", layers=2, max_batch=8)
+    s = ctx.sample(np.array([0, 5], np.uint32), seed=42, epoch=0, batch=0)
+    assert u32(s.uniq).tolist() == gold["rwalk"]["uniq"]
+    for l, b in enumerate(gold["rwalk"]["blocks"]):
+        assert u32(s.indptr[l]).tolist() == b["indptr"]
+        assert u32(s.indices[l]).tolist() == b["indices"]
+        assert u32(s.weights[l]).tolist() == b["weights"]
+    ctx.set_train_set(np.arange(8, dtype=np.uint32), 3, 42)
+    ctx.shuffle(0)
+    assert ctx.permutation(8).tolist() == gold["shuffle"]["epoch0"]
+    ctx.shuffle(1)
+    assert ctx.permutation(8).tolist() == gold["shuffle"]["epoch1"]
+
+
+def test_tiny_every_batch_bit_exact(tiny):
+    g, go = tiny
+    sh = g.shape
+    ctx = make_ctx(g, fanouts=sh.fanouts)
+    for e in [0, 1]:
+        ob = oracle.epoch_batches(g.train, sh.batch, g.seed, e)
+        ctx.shuffle(e)
+        assert np.array_equal(ctx.permutation(g.train.shape[0]), np.concatenate(ob))
+        for b, seeds in enumerate(ob):
+            ctx.sample_batch(e, b)
+            assert_same_sample(ctx.sample_result(), go.sample_khop(seeds, sh.fanouts, g.seed, e, b))
+
+
+def test_host_and_device_seed_paths(tiny):
+    g, go = tiny
+    ctx = make_ctx(g, fanouts=(10, 5))
+    seeds = g.train[100:164]
+    exp = go.sample_khop(seeds, (10, 5), 7, 3, 9)
+    assert_same_sample(ctx.sample(seeds, seed=7, epoch=3, batch=9), exp)
+    dev = torch.from_numpy(seeds.view(np.int32)).cuda()
+    assert_same_sample(ctx.sample(dev, seed=7, epoch=3, batch=9), exp)
+    # fanout override within capacity
+    assert_same_sample(ctx.sample(seeds, fanouts=(4, 2), seed=7, epoch=3, batch=9),
+                       go.sample_khop(seeds, (4, 2), 7, 3, 9))
+
+
+@pytest.mark.parametrize("fanouts", [(25, 10), (15, 10, 5), (3,), (1, 1, 1), (32, 2), (40, 33)])
+def test_fanout_variants_power_law(fanouts):
+    g = synth.small_graph(6000, 90000, 2.1, 8, 700, seed=11)
+    go = oracle.GraphOracle(g.indptr, g.indices)
+    ctx = make_ctx(g, fanouts=fanouts, max_batch=300)
+    for b, n0 in enumerate([1, 37, 300]):
+        seeds = g.train[b * 200:b * 200 + n0]
+        assert_same_sample(ctx.sample(seeds, seed=5, epoch=b, batch=b),
+                           go.sample_khop(seeds, fanouts, 5, b, b))
+
+
+def test_empty_batch_zero_hops_and_degree_zero():
+    # vertex 3 and 4 have no out-edges
+    indptr = np.array([0, 2, 4, 5, 5, 5], np.uint64)
+    indices = np.array([1, 3, 0, 4, 2], np.uint32)
+    go = oracle.GraphOracle(indptr, indices)
+    ctx = glb.Context(0)
+    ctx.load_graph(indptr, indices, None)
+    ctx.set_sampler("khop", fanouts=(2, 2), max_batch=4)
+    s = ctx.sample(np.array([], np.uint32), seed=1)
+    assert s.sizes == [0, 0, 0]
+    for seeds in ([3], [3, 4], [0, 3], [4, 0, 1, 2]):
+        assert_same_sample(ctx.sample(np.array(seeds, np.uint32), seed=1),
+                           go.sample_khop(seeds, (2, 2), 1, 0, 0))
+    s = ctx.sample(np.array([2, 1], np.uint32), fanouts=(), seed=1)
+    assert s.sizes == [2] and u32(s.uniq).tolist() == [2, 1]
+
+
+def test_errors():
+    g = synth.small_graph(500, 3000, 2.2, 4, 50, seed=8)
+    ctx = make_ctx(g, fanouts=(3, 2), max_batch=16)
+    with pytest.raises(glb.GlbError) as e:
+        ctx.sample(np.array([1, 2, 1], np.uint32))
+    assert e.value.code == glb.EINVAL
+    with pytest.raises(glb.GlbError) as e:
+        ctx.sample(np.array([1, 500], np.uint32))
+    assert e.value.code == glb.EINVAL
+    with pytest.raises(glb.GlbError) as e:
+        ctx.sample(np.arange(17, dtype=np.uint32))
+    assert e.value.code == glb.ENOMEM
+    with pytest.raises(glb.GlbError) as e:
+        ctx.sample(np.array([1], np.uint32), epoch=1 << 16)
+    assert e.value.code == glb.ERANGE
+    with pytest.raises(glb.GlbError) as e:
+        ctx.build_cache(1.5)
+    assert e.value.code == glb.EINVAL
+    # the ctx still works after errors
+    go = oracle.GraphOracle(g.indptr, g.indices)
+    assert_same_sample(ctx.sample(np.array([1, 2], np.uint32), seed=3),
+                       go.sample_khop([1, 2], (3, 2), 3, 0, 0))
+    bad = glb.Context(0)
+    with pytest.raises(glb.GlbError) as e:
+        bad.load_graph(np.array([0, 2, 1], np.uint64), np.array([0, 1], np.uint32), None)
+    assert e.value.code == glb.EINVAL
+    with pytest.raises(glb.GlbError) as e:
+        bad.load_graph(np.array([0, 1, 2], np.uint64), np.array([0, 7], np.uint32), None)
+    assert e.value.code == glb.EINVAL
+
+
+@pytest.mark.parametrize("layers,walks,length,topk", [(3, 4, 3, 5), (2, 4, 3, 5), (1, 2, 5, 3),
+                                                      (2, 8, 2, 7)])
+def test_random_walk_parity(layers, walks, length, topk):
+    g = synth.small_graph(8000, 60000, 2.5, 8, 600, seed=21)
+    go = oracle.GraphOracle(g.indptr, g.indices)
+    ctx = glb.Context(0)
+    ctx.load_graph(g.indptr, g.indices, None)
+    ctx.set_sampler("rwalk", layers=layers, walks=walks, walk_len=length, topk=topk, max_batch=200)
+    for b, n0 in enumerate([1, 64, 200]):
+        seeds = g.train[b * 200:b * 200 + n0]
+        gs = ctx.sample(seeds, seed=9, epoch=1, batch=b)
+        os_ = go.sample_rwalk(seeds, layers, 9, 1, b, walks, length, topk)
+        assert_same_sample(gs, os_, weighted=True)
+
+
+def test_presample_cache_and_hit_stats(tiny):
+    g, go = tiny
+    sh = g.shape
+    ctx = make_ctx(g, fanouts=sh.fanouts)
+    for K in [1, 2]:
+        ctx.reset_counts(glb.COUNT_PRESAMPLE)
+        ctx.presample(K)
+        exp = go.presample("khop", g.train, sh.batch, sh.fanouts, g.seed, K)
+        assert np.array_equal(ctx.get_counts(glb.COUNT_PRESAMPLE), exp)
+    counts = go.presample("khop", g.train, sh.batch, sh.fanouts, g.seed, 2)
+    # access recording over the measured epochs 2..3
+    ctx.reset_counts(glb.COUNT_ACCESS)
+    ctx.set_count_mode(glb.COUNT_ACCESS)
+    for e in [2, 3]:
+        for b in range(ctx.num_batches):
+            ctx.sample_batch(e, b)
+    ctx.set_count_mode(glb.COUNT_NONE)
+    ctx.sync()
+    acc = go.visit_counts("khop", g.train, sh.batch, sh.fanouts, g.seed, [2, 3])
+    assert np.array_equal(ctx.get_counts(glb.COUNT_ACCESS), acc)
+    for a in sh.alphas:
+        ctx.build_cache(a)
+        slot = oracle.cache_slots(counts, a)
+        assert np.array_equal(ctx.cache_slots(), slot), a
+        hs = ctx.hit_stats()
+        C = oracle.cache_size(a, g.V)
+        assert hs["cache_rows"] == C
+        tot = int(acc.sum())
+        assert hs["total"] == tot
+        assert hs["hits"] == int(acc[slot >= 0].sum())
+        assert hs["optimal_hits"] / tot == pytest.approx(oracle.optimal_hit_rate(acc, C), abs=0)
+        assert hs["hits"] <= hs["optimal_hits"]
+
+
+@pytest.mark.parametrize("alpha", [0.0, 0.1, 0.5, 1.0])
+def test_extract_sample_bytes(tiny, alpha):
+    g, go = tiny
+    sh = g.shape
+    ctx = make_ctx(g, fanouts=sh.fanouts)
+    ctx.presample(1)
+    ctx.build_cache(alpha)
+    slot = ctx.cache_slots()
+    for e, b in [(1, 0), (1, 15)]:
+        ctx.sample_batch(e, b)
+        s = ctx.sample_result()
+        out = torch.full((s.sizes[-1] + 3, g.D), float("nan"), device="cuda")
+        st = ctx.extract_sample(out, stats=True)
+        seeds = oracle.epoch_batches(g.train, sh.batch, g.seed, e)[b]
+        os_ = go.sample_khop(seeds, sh.fanouts, g.seed, e, b)
+        exp = go.extract(os_.uniq)
+        got = out[:s.sizes[-1]].cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), exp.view(np.uint32))
+        assert torch.isnan(out[s.sizes[-1]:]).all()          # nothing written past n_L
+        assert st["hits"] == int((slot[os_.uniq] >= 0).sum())
+        assert st["hits"] + st["misses"] == s.sizes[-1]
+        assert np.array_equal(s.cache_slot.cpu().numpy(), slot[os_.uniq])
+
+
+@pytest.mark.parametrize("D", [7, 32, 64, 100, 128, 256])
+def test_extract_generic_ids_dims(D):
+    V = 3000
+    g = synth.small_graph(V, 20000, 2.2, D, 300, seed=D)
+    go = oracle.GraphOracle(g.indptr, g.indices, g.features)
+    ctx = make_ctx(g, fanouts=(5,), max_batch=64)
+    ctx.presample(1)
+    ctx.build_cache(0.3)
+    rng = np.random.default_rng(D)
+    for n in [0, 1, 33, 5000]:
+        ids = rng.integers(0, V, n).astype(np.uint32)
+        if n > 3:
+            ids[1] = ids[0]                                   # duplicates allowed
+        out, st = ctx.extract(torch.from_numpy(ids.view(np.int32)).cuda(), stats=True)
+        assert np.array_equal(out.cpu().numpy().view(np.uint32), go.extract(ids).view(np.uint32))
+        assert st["hits"] == int((ctx.cache_slots()[ids] >= 0).sum()) and st["hits"] + st["misses"] == n
+    with pytest.raises(glb.GlbError):
+        ctx.extract(torch.tensor([0, V], dtype=torch.int32, device="cuda"))
+        ctx.sync()
+
+
+def test_degree_hotness_cache():
+    g = synth.small_graph(4000, 40000, 2.2, 16, 200, seed=3)
+    ctx = make_ctx(g, fanouts=(5,), max_batch=64)
+    deg = np.diff(g.indptr).astype(np.uint32)
+    ctx.build_cache(0.1, hotness=torch.from_numpy(deg.view(np.int32)).cuda())
+    assert np.array_equal(ctx.cache_slots(), oracle.cache_slots(deg, 0.1))
+
+
+# ----------------------------------------------------------------------------- full PR size
+@pytest.fixture(scope="module")
+def pr():
+    g = synth.make_graph("PR")
+    return g, oracle.GraphOracle(g.indptr, g.indices, g.features)
+
+
+@pytest.mark.slow
+def test_pr_full_size_parity(pr):
+    """configs[1] at full size, bench launch configuration: PreSC#1 counts in
+    full, cache slots at the sweep's alphas, and every output of four batches."""
+    g, go = pr
+    sh = g.shape
+    ctx = make_ctx(g, fanouts=sh.fanouts)
+    ctx.presample(sh.K)
+    counts = go.presample("khop", g.train, sh.batch, sh.fanouts, g.seed, sh.K)
+    assert np.array_equal(ctx.get_counts(glb.COUNT_PRESAMPLE), counts)
+    for a in (0.05, 0.25):
+        ctx.build_cache(a)
+        assert np.array_equal(ctx.cache_slots(), oracle.cache_slots(counts, a))
+    ctx.build_cache(1.0)
+    e = sh.K
+    ob = oracle.epoch_batches(g.train, sh.batch, g.seed, e)
+    nb = len(ob)
+    rng = np.random.default_rng(0)
+    out = torch.empty((sh.batch * 26 * 11, g.D), device="cuda")
+    for b in [0, 1, int(rng.integers(2, nb - 1)), nb - 1]:
+        ctx.sample_batch(e, b)
+        s = ctx.sample_result()
+        os_ = go.sample_khop(ob[b], sh.fanouts, g.seed, e, b)
+        assert_same_sample(s, os_)
+        ctx.extract_sample(out)
+        torch.cuda.synchronize()
+        idx = rng.integers(0, s.sizes[-1], 4096)
+        got = out[torch.from_numpy(idx).cuda()].cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), g.features[os_.uniq[idx]].view(np.uint32))
