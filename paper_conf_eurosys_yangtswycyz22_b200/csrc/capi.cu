@@ -65,7 +65,7 @@ void free_sample_bufs(glb_ctx* c) {
   for (int l = 0; l < GLB_MAX_HOPS; ++l) {
     dfree(b.bindptr[l]); dfree(b.bindices[l]); dfree(b.bweights[l]); dfree(b.status[l]);
   }
-  dfree(b.hit_dst); dfree(b.hit_src); dfree(b.miss_dst); dfree(b.miss_src);
+  dfree(b.hit_list); dfree(b.miss_list);
   b = SampleBufs();
   c->sampler_set = false;
   c->have_sample = false;
@@ -120,7 +120,6 @@ glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, in
     if (kind == GLB_KHOP_UNIFORM) CK(launch_khop(c, l, k[l], seed, epoch, batch));
     else CK(launch_rwalk(c, l, seed, epoch, batch));
     CK(launch_compact(c, l, k[l], kind == GLB_RANDOM_WALK, mode));
-    CK(launch_remap(c, l));
   }
   c->have_sample = true;
   c->last_L = L;
@@ -181,7 +180,7 @@ glb_status glb_destroy(glb_ctx* c) {
   if (c->stream) cudaStreamSynchronize(c->stream);
   free_sample_bufs(c);
   free_graph(c);
-  dfree(c->xb.hit_dst); dfree(c->xb.hit_src); dfree(c->xb.miss_dst); dfree(c->xb.miss_src);
+  dfree(c->xb.hit_list); dfree(c->xb.miss_list);
   dfree(c->train); dfree(c->perm); dfree(c->shuf_keys); dfree(c->shuf_vals);
   dfree(c->st); dfree(c->st_x); dfree(c->scratch); dfree(c->xcount);
   if (c->sort_tmp) cudaFree(c->sort_tmp);
@@ -316,10 +315,8 @@ glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32
     b.ntiles[l] = (flat + kCompactTile - 1) / kCompactTile;
     CK(dalloc(&b.status[l], b.ntiles[l]));
   }
-  CK(dalloc(&b.hit_dst, un));
-  CK(dalloc(&b.hit_src, un));
-  CK(dalloc(&b.miss_dst, un));
-  CK(dalloc(&b.miss_src, un));
+  CK(dalloc(&b.hit_list, un));
+  CK(dalloc(&b.miss_list, un));
   c->kind = kind;
   c->L = L;
   for (uint32_t l = 0; l < L; ++l) c->fanouts[l] = k[l];
@@ -530,8 +527,8 @@ glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
   if (c->features_mapped && C) {
     CK(dalloc(&c->cache, C * (uint64_t)c->D));
     // cache rows come over PCIe from the mapped host matrix (zero copy)
-    CK(launch_gather(c, c->cache, nullptr, c->features_mapped, nullptr, nullptr, nullptr, order,
-                     nullptr, 0, C));
+    CK(launch_gather(c, c->cache, nullptr, c->features_mapped, nullptr, nullptr, order, nullptr,
+                     0, C));
   }
   CK(cudaStreamSynchronize(c->stream));
   cudaFree(tmp);
@@ -594,18 +591,16 @@ glb_status glb_extract(glb_ctx* c, const uint32_t* vertices, uint64_t n, void* o
   if (n >= 0xFFFFFFFFull) return set_err(c, GLB_EINVAL, "n too large");
   if (n > c->xb.cap) {
     CK(cudaStreamSynchronize(c->stream));
-    dfree(c->xb.hit_dst); dfree(c->xb.hit_src); dfree(c->xb.miss_dst); dfree(c->xb.miss_src);
+    dfree(c->xb.hit_list); dfree(c->xb.miss_list);
     c->xb.cap = 0;
-    CK(dalloc(&c->xb.hit_dst, n));
-    CK(dalloc(&c->xb.hit_src, n));
-    CK(dalloc(&c->xb.miss_dst, n));
-    CK(dalloc(&c->xb.miss_src, n));
+    CK(dalloc(&c->xb.hit_list, n));
+    CK(dalloc(&c->xb.miss_list, n));
     c->xb.cap = n;
   }
   CK(cudaMemsetAsync(&c->st_x->nhit, 0, 2 * sizeof(uint32_t), c->stream));
   if (n) CK(launch_mark(c, vertices, n));
-  CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->xb.hit_dst, c->xb.hit_src,
-                   c->xb.miss_dst, c->xb.miss_src, &c->st_x->nhit, 0, 0));
+  CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->xb.hit_list, c->xb.miss_list,
+                   nullptr, &c->st_x->nhit, 0, 0));
   if (stats) {
     CK(cudaMemcpyAsync(c->h_xcount, c->xcount, 2 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
     c->pending_stats = stats;
@@ -618,8 +613,8 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
   if (!c->have_sample) return set_err(c, GLB_ESTATE, "extract_sample without a current sample");
   if (!c->features_mapped) return set_err(c, GLB_ESTATE, "graph loaded without features");
   if (!out) return set_err(c, GLB_EINVAL, "null out");
-  CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_dst, c->sb.hit_src,
-                   c->sb.miss_dst, c->sb.miss_src, &c->st->nhit, 0, 0));
+  CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_list, c->sb.miss_list,
+                   nullptr, &c->st->nhit, 0, 0));
   if (stats) {
     CK(cudaMemcpyAsync(c->h_xcount, c->xcount, 2 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
     c->pending_stats = stats;

@@ -8,9 +8,14 @@
 // One persistent launch serves both halves: blocks [0, H) gather cache hits
 // from HBM, blocks [H, grid) gather misses straight from the mapped pinned
 // host matrix (zero copy over PCIe), so the HBM gather never waits behind
-// PCIe latency and no CPU thread touches feature bytes.  Rows move as 16-byte
-// vectors (LDG.128/STG.128), each row handled by a group of lanes, four rows
-// in flight per group.
+// PCIe latency and no CPU thread touches feature bytes.
+//
+// A block copies a chunk of R rows per iteration: the chunk's (dst, src)
+// work-list entries are staged in shared memory (double-buffered, the next
+// chunk's entries are loaded while this chunk's rows are in flight), then the
+// R*U 16-byte vectors (U = vectors per row) are spread over all 256 threads,
+// 8 independent LDG.128 per thread issued before any store (MLP ~128 B per
+// thread), stores streamed (st.global.cs).
 #include <cuda_runtime.h>
 
 #include "glb_internal.cuh"
@@ -20,6 +25,8 @@ namespace glb {
 namespace {
 
 constexpr unsigned kFull = 0xFFFFFFFFu;
+constexpr int kVecPerThread = 8;
+constexpr int kChunkUnits = kThreads * kVecPerThread;  // vectors per chunk
 
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t m;
@@ -29,9 +36,8 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 
 __global__ void __launch_bounds__(kThreads)
     k_mark(const uint32_t* __restrict__ vertices, uint64_t n, uint64_t V,
-           const int32_t* __restrict__ slot, DevState* st, uint32_t* __restrict__ hit_dst,
-           uint32_t* __restrict__ hit_src, uint32_t* __restrict__ miss_dst,
-           uint32_t* __restrict__ miss_src) {
+           const int32_t* __restrict__ slot, DevState* st, uint2* __restrict__ hit_list,
+           uint2* __restrict__ miss_list) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i0 = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); i0 < n; i0 += stride) {
     const uint64_t i = i0 + (threadIdx.x & 31);
@@ -56,28 +62,25 @@ __global__ void __launch_bounds__(kThreads)
     }
     bh = __shfl_sync(kFull, bh, 0);
     bm = __shfl_sync(kFull, bm, 0);
-    if (hit) {
-      const uint32_t r = bh + __popc(mh & lanemask_lt());
-      hit_dst[r] = (uint32_t)i;
-      hit_src[r] = (uint32_t)s;
-    }
-    if (miss) {
-      const uint32_t r = bm + __popc(mm & lanemask_lt());
-      miss_dst[r] = (uint32_t)i;
-      miss_src[r] = u;
-    }
+    if (hit) hit_list[bh + __popc(mh & lanemask_lt())] = make_uint2((uint32_t)i, (uint32_t)s);
+    if (miss) miss_list[bm + __popc(mm & lanemask_lt())] = make_uint2((uint32_t)i, u);
   }
 }
 
-// Gather rows src[src_idx[r]] -> out[dst_idx ? dst_idx[r] : r] for both lists.
-// LPR lanes per row; VEC: 16-byte vectors (row bytes % 16 == 0).
-template <int LPR, bool VEC>
-__global__ void __launch_bounds__(kThreads)
-    k_gather(float* __restrict__ out, const float* __restrict__ src_hit,
-             const float* __restrict__ src_miss, const uint32_t* __restrict__ hit_dst,
-             const uint32_t* __restrict__ hit_src, const uint32_t* __restrict__ miss_dst,
-             const uint32_t* __restrict__ miss_src, const uint32_t* __restrict__ dev_counts,
-             uint64_t nh_host, uint64_t nm_host, uint32_t D, unsigned long long* xcount) {
+template <typename T>
+__device__ __forceinline__ T ld_row(const T* p) { return __ldg(p); }
+template <typename T>
+__device__ __forceinline__ void st_row(T* p, T v) { __stcs(p, v); }
+
+// T = float4 (row bytes % 16 == 0) or float.  U = T-units per row.
+template <typename T>
+__global__ void __launch_bounds__(kThreads, 4)
+    k_gather(T* __restrict__ out, const T* __restrict__ src_hit, const T* __restrict__ src_miss,
+             const uint2* __restrict__ hit_list, const uint2* __restrict__ miss_list,
+             const uint32_t* __restrict__ fill_src, const uint32_t* __restrict__ dev_counts,
+             uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t R,
+             unsigned long long* xcount) {
+  __shared__ uint2 ent[2][kThreads];
   const uint64_t nh = dev_counts ? dev_counts[0] : nh_host;
   const uint64_t nm = dev_counts ? dev_counts[1] : nm_host;
   const uint32_t G = gridDim.x;
@@ -87,63 +90,52 @@ __global__ void __launch_bounds__(kThreads)
   const uint32_t rb = is_miss ? blockIdx.x - (G - miss_blocks) : blockIdx.x;
   const uint32_t nrb = is_miss ? miss_blocks : G - miss_blocks;
   const uint64_t n = is_miss ? nm : nh;
-  const uint32_t* dlist = is_miss ? miss_dst : hit_dst;
-  const uint32_t* slist = is_miss ? miss_src : hit_src;
-  const float* src = is_miss ? src_miss : src_hit;
+  const uint2* list = is_miss ? miss_list : hit_list;
+  const uint32_t* fsrc = is_miss ? fill_src : nullptr;
+  const T* src = is_miss ? src_miss : src_hit;
   if (xcount && blockIdx.x == 0 && threadIdx.x == 0) {
     xcount[0] = nh;
     xcount[1] = nm;
   }
   if (n == 0) return;
-  const uint32_t li = threadIdx.x % LPR;
-  const uint64_t grp = ((uint64_t)rb * blockDim.x + threadIdx.x) / LPR;
-  const uint64_t ngrp = (uint64_t)nrb * blockDim.x / LPR;
-  constexpr int U = 4;
-  if (VEC) {
-    const uint32_t vpr = D / 4;
-    const float4* s4 = reinterpret_cast<const float4*>(src);
-    float4* o4 = reinterpret_cast<float4*>(out);
-    for (uint64_t r0 = grp; r0 < n; r0 += U * ngrp) {
-      uint64_t so[U], dof[U];
-      bool ok[U];
+  const uint32_t t = threadIdx.x;
+  const uint64_t nchunks = (n + R - 1) / R;
+  const float inv_u = 1.0f / (float)U;
+  auto load_ent = [&](uint64_t chunk) -> uint2 {
+    const uint64_t r = chunk * R + t;
+    if (t < R && chunk < nchunks && r < n)
+      return fsrc ? make_uint2((uint32_t)r, __ldg(fsrc + r)) : __ldg(list + r);
+    return make_uint2(0u, 0u);
+  };
+  uint2 e = load_ent(rb);
+  int buf = 0;
+  for (uint64_t c = rb; c < nchunks; c += nrb) {
+    if (t < R) ent[buf][t] = e;
+    __syncthreads();
+    e = load_ent(c + nrb);  // prefetch the next chunk's entries
+    const uint64_t rows = min((uint64_t)R, n - c * R);
+    const uint32_t total = (uint32_t)rows * U;
+    for (uint32_t base = 0; base < total; base += kChunkUnits) {
+      T x[kVecPerThread];
+      uint64_t dst[kVecPerThread];
 #pragma unroll
-      for (int q = 0; q < U; ++q) {
-        const uint64_t r = r0 + q * ngrp;
-        ok[q] = r < n;
-        so[q] = ok[q] ? (uint64_t)__ldg(slist + r) * vpr : 0;
-        dof[q] = ok[q] ? (uint64_t)(dlist ? __ldg(dlist + r) : r) * vpr : 0;
+      for (int q = 0; q < kVecPerThread; ++q) {
+        const uint32_t v = base + q * kThreads + t;
+        if (v < total) {
+          uint32_t row = (uint32_t)(((float)v + 0.5f) * inv_u);  // exact for v < 2^20
+          const uint32_t col = v - row * U;
+          const uint2 en = ent[buf][row];
+          x[q] = ld_row(src + (uint64_t)en.y * U + col);
+          dst[q] = (uint64_t)en.x * U + col;
+        }
       }
-      for (uint32_t c = li; c < vpr; c += LPR) {
-        float4 x[U];
 #pragma unroll
-        for (int q = 0; q < U; ++q)
-          if (ok[q]) x[q] = __ldg(s4 + so[q] + c);
-#pragma unroll
-        for (int q = 0; q < U; ++q)
-          if (ok[q]) o4[dof[q] + c] = x[q];
-      }
-    }
-  } else {
-    for (uint64_t r0 = grp; r0 < n; r0 += U * ngrp) {
-      uint64_t so[U], dof[U];
-      bool ok[U];
-#pragma unroll
-      for (int q = 0; q < U; ++q) {
-        const uint64_t r = r0 + q * ngrp;
-        ok[q] = r < n;
-        so[q] = ok[q] ? (uint64_t)__ldg(slist + r) * D : 0;
-        dof[q] = ok[q] ? (uint64_t)(dlist ? __ldg(dlist + r) : r) * D : 0;
-      }
-      for (uint32_t c = li; c < D; c += LPR) {
-        float x[U];
-#pragma unroll
-        for (int q = 0; q < U; ++q)
-          if (ok[q]) x[q] = __ldg(src + so[q] + c);
-#pragma unroll
-        for (int q = 0; q < U; ++q)
-          if (ok[q]) out[dof[q] + c] = x[q];
+      for (int q = 0; q < kVecPerThread; ++q) {
+        const uint32_t v = base + q * kThreads + t;
+        if (v < total) st_row(out + dst[q], x[q]);
       }
     }
+    buf ^= 1;
   }
 }
 
@@ -153,33 +145,30 @@ cudaError_t launch_mark(glb_ctx* c, const uint32_t* vertices, uint64_t n) {
   int grid = (int)((n + kThreads - 1) / kThreads);
   if (grid < 1) grid = 1;
   if (grid > c->num_sms * 8) grid = c->num_sms * 8;
-  k_mark<<<grid, kThreads, 0, c->stream>>>(vertices, n, c->V, c->slot, c->st_x, c->xb.hit_dst,
-                                           c->xb.hit_src, c->xb.miss_dst, c->xb.miss_src);
+  k_mark<<<grid, kThreads, 0, c->stream>>>(vertices, n, c->V, c->slot, c->st_x, c->xb.hit_list,
+                                           c->xb.miss_list);
   count_launch(c);
   return cudaGetLastError();
 }
 
 cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const float* src_miss,
-                          const uint32_t* hit_dst, const uint32_t* hit_src,
-                          const uint32_t* miss_dst, const uint32_t* miss_src,
+                          const uint2* hit_list, const uint2* miss_list, const uint32_t* fill_src,
                           const uint32_t* dev_counts, uint64_t nhit_host, uint64_t nmiss_host) {
   const uint32_t D = c->D;
   const bool vec = (D % 4) == 0;
-  const uint32_t units = vec ? D / 4 : D;  // per-row work units
-  const int grid = c->num_sms * 8;
-#define GLB_GATHER_ARGS                                                                   \
-  out, src_hit, src_miss, hit_dst, hit_src, miss_dst, miss_src, dev_counts, nhit_host, \
-      nmiss_host, D, c->xcount
-  if (vec) {
-    if (units <= 8) k_gather<8, true><<<grid, kThreads, 0, c->stream>>>(GLB_GATHER_ARGS);
-    else if (units <= 16) k_gather<16, true><<<grid, kThreads, 0, c->stream>>>(GLB_GATHER_ARGS);
-    else k_gather<32, true><<<grid, kThreads, 0, c->stream>>>(GLB_GATHER_ARGS);
-  } else {
-    if (units <= 8) k_gather<8, false><<<grid, kThreads, 0, c->stream>>>(GLB_GATHER_ARGS);
-    else if (units <= 16) k_gather<16, false><<<grid, kThreads, 0, c->stream>>>(GLB_GATHER_ARGS);
-    else k_gather<32, false><<<grid, kThreads, 0, c->stream>>>(GLB_GATHER_ARGS);
-  }
-#undef GLB_GATHER_ARGS
+  const uint32_t U = vec ? D / 4 : D;
+  uint32_t R = kChunkUnits / U;
+  if (R > (uint32_t)kThreads) R = kThreads;
+  if (R < 1) R = 1;
+  const int grid = c->num_sms * 4;
+  if (vec)
+    k_gather<float4><<<grid, kThreads, 0, c->stream>>>(
+        (float4*)out, (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list,
+        fill_src, dev_counts, nhit_host, nmiss_host, U, R, c->xcount);
+  else
+    k_gather<float><<<grid, kThreads, 0, c->stream>>>(out, src_hit, src_miss, hit_list, miss_list,
+                                                      fill_src, dev_counts, nhit_host, nmiss_host,
+                                                      U, R, c->xcount);
   count_launch(c);
   return cudaGetLastError();
 }

@@ -84,18 +84,14 @@ struct SampleBufs {
   uint32_t* bweights[GLB_MAX_HOPS] = {};
   unsigned long long* status[GLB_MAX_HOPS] = {};
   uint64_t ntiles[GLB_MAX_HOPS] = {};
-  uint32_t* hit_dst = nullptr;        // extract work lists
-  uint32_t* hit_src = nullptr;
-  uint32_t* miss_dst = nullptr;
-  uint32_t* miss_src = nullptr;
+  uint2* hit_list = nullptr;          // extract work lists: (dst row, cache slot)
+  uint2* miss_list = nullptr;         //                     (dst row, gid)
 };
 
 struct ExtractBufs {
   uint64_t cap = 0;
-  uint32_t* hit_dst = nullptr;
-  uint32_t* hit_src = nullptr;
-  uint32_t* miss_dst = nullptr;
-  uint32_t* miss_src = nullptr;
+  uint2* hit_list = nullptr;
+  uint2* miss_list = nullptr;
 };
 
 }  // namespace glb
@@ -181,11 +177,11 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
                         uint32_t batch);
 cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch, uint32_t batch);
 cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, int count_mode);
-cudaError_t launch_remap(glb_ctx* c, uint32_t hop);
 cudaError_t launch_mark(glb_ctx* c, const uint32_t* vertices, uint64_t n);
+// Gather rows: hits src_hit[list.y] -> out[list.x], misses src_miss[list.y] -> out[list.x];
+// fill_src (non-null) replaces miss_list with (r, fill_src[r]) (identity destination).
 cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const float* src_miss,
-                          const uint32_t* hit_dst, const uint32_t* hit_src,
-                          const uint32_t* miss_dst, const uint32_t* miss_src,
+                          const uint2* hit_list, const uint2* miss_list, const uint32_t* fill_src,
                           const uint32_t* dev_counts /* [nhit, nmiss] on device or null */,
                           uint64_t nhit_host, uint64_t nmiss_host);
 cudaError_t launch_shuffle_keys(glb_ctx* c, uint32_t epoch, unsigned long long* keys, uint32_t* vals);

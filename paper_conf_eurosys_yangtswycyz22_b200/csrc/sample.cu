@@ -9,15 +9,16 @@
 // marked during Sample (L252).
 //
 // Design:
-//  * k_khop: G lanes per frontier vertex (G = next_pow2(fanout) <= 32), one
+//  * k_khop: k lanes per frontier vertex (floor(32/k) vertices per warp), one
 //    lane per slot.  Floyd's draws are independent per slot (counter-based
 //    RNG), so every lane computes its t_s at once; the sequential "t already
 //    chosen?" test is resolved exactly with __match_any_sync + a short
 //    fixed-point over the j-chain (proof in DESIGN.md).
 //  * relabel: direct-address table vmap[gid] = (~gen << 32 | first position),
-//    one atomicMin per pick (filtered by a plain read and a warp match), then a
-//    single-pass decoupled-look-back scan over the padded (vertex, slot) array
-//    assigns new lids in first-occurrence order and builds the block CSR.
+//    one atomicMin per pick (filtered by a plain read), then a single-pass
+//    decoupled-look-back scan over the padded (vertex, slot) array assigns new
+//    lids in first-occurrence order and writes the block CSR with src lids
+//    directly (no separate remap pass).
 #include <cuda_runtime.h>
 
 #include "glb_internal.cuh"
@@ -34,23 +35,6 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
   return m;
 }
 
-// Warp-aggregated append of (dst, src) to a list whose length lives at *ctr.
-__device__ __forceinline__ void warp_append(bool pred, uint32_t* ctr, uint32_t* dst_list,
-                                            uint32_t* src_list, uint32_t dst, uint32_t src) {
-  const uint32_t m = __ballot_sync(kFull, pred);
-  if (!m) return;
-  const int lane = threadIdx.x & 31;
-  const int leader = __ffs(m) - 1;
-  uint32_t base = 0;
-  if (lane == leader) base = atomicAdd(ctr, (uint32_t)__popc(m));
-  base = __shfl_sync(kFull, base, leader);
-  if (pred) {
-    const uint32_t r = base + __popc(m & lanemask_lt());
-    dst_list[r] = dst;
-    src_list[r] = src;
-  }
-}
-
 // Insert one pick into the relabel table: keep the smallest position of this
 // generation.  Values only decrease over time, so a (possibly stale) read that
 // is already <= e proves the atomic would be a no-op.
@@ -63,11 +47,9 @@ __device__ __forceinline__ void vmap_insert(unsigned long long* vmap, uint32_t u
 struct MarkArgs {
   const int32_t* slot;
   int32_t* lidslot;
-  uint32_t* hit_dst;
-  uint32_t* hit_src;
-  uint32_t* miss_dst;
-  uint32_t* miss_src;
-  uint32_t* count;  // nullable visit-count target
+  uint2* hit_list;   // (lid, slot)
+  uint2* miss_list;  // (lid, gid)
+  uint32_t* count;   // nullable visit-count target
 };
 
 struct StatusArgs {  // look-back status arrays to clear for this batch
@@ -88,10 +70,11 @@ __global__ void __launch_bounds__(kThreads)
   const uint32_t stride = gridDim.x * blockDim.x;
   for (uint32_t l = 0; l < za.L; ++l)
     for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < za.n[l]; i += stride) za.p[l][i] = 0ull;
-  // warp-uniform loop bound so that warp_append's ballots see the whole warp
+  const int lane = threadIdx.x & 31;
+  // warp-uniform loop bound so that the ballots below see the whole warp
   for (uint32_t i0 = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); i0 < n0; i0 += stride) {
-    const uint32_t i = i0 + (threadIdx.x & 31);
-    bool act = i < n0;
+    const uint32_t i = i0 + lane;
+    const bool act = i < n0;
     uint32_t u = 0;
     int32_t s = -1;
     if (act) {
@@ -107,13 +90,23 @@ __global__ void __launch_bounds__(kThreads)
       mk.lidslot[i] = s;
       if (mk.count) atomicAdd(mk.count + u, 1u);
     }
-    warp_append(act && s >= 0, &st->nhit, mk.hit_dst, mk.hit_src, i, (uint32_t)s);
-    warp_append(act && s < 0, &st->nmiss, mk.miss_dst, mk.miss_src, i, u);
+    const bool hit = act && s >= 0, miss = act && s < 0;
+    const uint32_t mh = __ballot_sync(kFull, hit), mm = __ballot_sync(kFull, miss);
+    uint32_t bh = 0, bm = 0;
+    if (lane == 0) {
+      if (mh) bh = atomicAdd(&st->nhit, (uint32_t)__popc(mh));
+      if (mm) bm = atomicAdd(&st->nmiss, (uint32_t)__popc(mm));
+    }
+    bh = __shfl_sync(kFull, bh, 0);
+    bm = __shfl_sync(kFull, bm, 0);
+    if (hit) mk.hit_list[bh + __popc(mh & lanemask_lt())] = make_uint2(i, (uint32_t)s);
+    if (miss) mk.miss_list[bm + __popc(mm & lanemask_lt())] = make_uint2(i, u);
   }
 }
 
-// ---------------------------------------------------------------- k-hop (G lanes / vertex)
-template <int G>
+// ---------------------------------------------------------------- k-hop (k lanes / vertex)
+// Fanout k <= 32: floor(32/k) frontier vertices per warp, lane s of a group
+// owns Floyd slot s.
 __global__ void __launch_bounds__(kThreads)
     k_khop(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch, uint32_t gen,
            const DevState* __restrict__ st, DevState* st_w, const uint64_t* __restrict__ indptr,
@@ -123,14 +116,15 @@ __global__ void __launch_bounds__(kThreads)
   const uint32_t base = st->base[hop];
   const uint32_t c3 = ctr3(epoch, hop, kDomKhop);
   const int lane = threadIdx.x & 31;
-  const uint32_t s = lane & (G - 1);
-  const int gbase = lane & ~(G - 1);
-  constexpr uint32_t kGroupsPerWarp = 32 / G;
+  const uint32_t gpw = 32 / k;                 // groups (vertices) per warp
+  const uint32_t gi = (uint32_t)lane / k;      // >= gpw: idle lane
+  const uint32_t s = (uint32_t)lane - gi * k;  // slot
+  const int gbase = (int)(gi * k);
   const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
-  for (uint32_t w0 = warp_global * kGroupsPerWarp; w0 < n_l; w0 += nwarps * kGroupsPerWarp) {
-    const uint32_t d = w0 + lane / G;
-    const bool active = d < n_l;
+  for (uint32_t w0 = warp_global * gpw; w0 < n_l; w0 += nwarps * gpw) {
+    const uint32_t d = w0 + gi;
+    const bool active = gi < gpw && d < n_l;
     uint32_t v = 0, deg = 0;
     uint64_t lo = 0;
     if (active) {
@@ -140,42 +134,38 @@ __global__ void __launch_bounds__(kThreads)
       if (hop == 0 && s == 0 && __ldcg(vmap + v) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
     }
     const bool big = active && deg > k;
-    const bool part = big && s < k;  // lane draws a Floyd candidate
     uint32_t t = 0, j = 0;
-    if (part) {
+    if (big) {
       j = deg - k + s;
       t = bounded(draw64(seed, v, s >> 1, batch, c3, s & 1u), j + 1);
     }
-    // D1: an earlier slot of the same vertex drew the same t
-    const unsigned long long key =
-        part ? (((unsigned long long)(lane / G) << 32) | t) : ((1ull << 63) | (unsigned)lane);
-    const uint32_t eq = __match_any_sync(kFull, key);
-    const bool d1 = (eq & lanemask_lt()) != 0;
-    // j-chain: t equals j_{s'} (s' < s), which is taken iff slot s' was displaced
-    const bool inr = part && t >= deg - k && t < j;
-    const int ref = inr ? gbase + (int)(t - (deg - k)) : lane;
-    bool disp = d1;
-    for (;;) {
-      const bool r = __shfl_sync(kFull, disp, ref);
-      const bool nd = d1 || (inr && r);
-      const bool done = __ballot_sync(kFull, nd) == __ballot_sync(kFull, disp);
-      disp = nd;
-      if (done) break;
-    }
     uint32_t sel = kEmpty;
-    if (big) {
-      if (s < k) sel = disp ? j : t;
-    } else if (active && s < deg) {
-      sel = s;
+    if (__any_sync(kFull, big)) {
+      // D1: an earlier slot of the same vertex drew the same t
+      const unsigned long long key =
+          big ? (((unsigned long long)gi << 32) | t) : ((1ull << 63) | (unsigned)lane);
+      const uint32_t eq = __match_any_sync(kFull, key);
+      const bool d1 = (eq & lanemask_lt()) != 0;
+      // j-chain: t equals j_{s'} (s' < s), which is taken iff slot s' was displaced
+      const bool inr = big && t >= deg - k && t < j;
+      const int ref = inr ? gbase + (int)(t - (deg - k)) : lane;
+      bool disp = d1;
+      for (;;) {
+        const bool r = __shfl_sync(kFull, disp, ref);
+        const bool nd = d1 || (inr && r);
+        const bool done = __ballot_sync(kFull, nd) == __ballot_sync(kFull, disp);
+        disp = nd;
+        if (done) break;
+      }
+      if (big) sel = disp ? j : t;
     }
+    if (!big && active && s < deg) sel = s;
     uint32_t u = kEmpty;
-    if (sel != kEmpty) u = __ldg(indices + lo + sel);
-    if (active && s < k) picks[(size_t)d * k + s] = u;
-    // one atomic per distinct gid per warp (lowest lane = smallest position)
-    const unsigned long long ukey = (u != kEmpty) ? (unsigned long long)u : ((1ull << 32) | (unsigned)lane);
-    const uint32_t peers = __match_any_sync(kFull, ukey);
-    if (u != kEmpty && (peers & lanemask_lt()) == 0)
+    if (sel != kEmpty) {
+      u = __ldg(indices + lo + sel);
       vmap_insert(vmap, u, enc_pos(gen, base + d * k + s));
+    }
+    if (active) picks[(size_t)d * k + s] = u;
   }
 }
 
@@ -322,8 +312,11 @@ __global__ void __launch_bounds__(kThreads)
 
 // ---------------------------------------------------------------- compaction scan
 // Status word of the decoupled look-back: [flag:2][new:31][valid:31].
+// flag 1 = aggregate, 2 = inclusive prefix, 3 = inclusive + this tile's lids
+// are written to lidmap (other tiles may read them).
 constexpr unsigned long long kFlagAgg = 1ull << 62;
 constexpr unsigned long long kFlagInc = 2ull << 62;
+constexpr unsigned long long kFlagDone = 3ull << 62;
 constexpr unsigned long long kValMask = (1ull << 62) - 1;
 
 __device__ __forceinline__ unsigned long long pack_status(unsigned long long flag,
@@ -336,11 +329,12 @@ __device__ __forceinline__ unsigned long long unpack_pair(unsigned long long w) 
   return ((w >> 31) << 32) | (w & 0x7FFFFFFFull);
 }
 
-__device__ __forceinline__ unsigned long long warp_incl_scan64(unsigned long long x) {
+template <typename T>
+__device__ __forceinline__ T warp_incl_scan(T x) {
   const int lane = threadIdx.x & 31;
 #pragma unroll
   for (int o = 1; o < 32; o <<= 1) {
-    const unsigned long long y = __shfl_up_sync(kFull, x, o);
+    const T y = __shfl_up_sync(kFull, x, o);
     if (lane >= o) x += y;
   }
   return x;
@@ -351,17 +345,30 @@ __device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
   return x;
 }
 
+// One tile = kCompactTile consecutive (vertex, slot) positions of hop l.
+//  1. valid = pick present; new = this position is the first occurrence
+//     (vmap holds the minimum position of this generation).
+//  2. block scan of (new, valid) + decoupled look-back -> global prefixes:
+//     new vertices get lid n_l + new-prefix (first-occurrence order); valid
+//     picks get edge slot valid-prefix (block CSR in slot order).
+//  3. new vertices: uniq/lidmap/mark/count; tile publishes "lids written".
+//  4. every edge's src lid: new -> own; repeat of a vertex first seen at an
+//     earlier position p: same tile -> shared memory, earlier tile -> wait for
+//     that tile's flag then lidmap; earlier hop (p < base) -> lidmap.
 template <bool W>
 __global__ void __launch_bounds__(kThreads)
     k_compact(uint32_t hop, uint32_t k, uint32_t gen, DevState* st,
               const uint32_t* __restrict__ picks, const uint32_t* __restrict__ pickw,
-              const unsigned long long* __restrict__ vmap, uint32_t* __restrict__ lidmap,
+              const unsigned long long* __restrict__ vmap, uint32_t* lidmap,
               uint32_t* __restrict__ uniq, uint32_t* __restrict__ bindptr,
               uint32_t* __restrict__ bindices, uint32_t* __restrict__ bweights,
               unsigned long long* status, MarkArgs mk) {
   __shared__ uint32_t s_tile;
   __shared__ unsigned long long s_warp[kThreads / 32];
-  __shared__ unsigned long long s_excl;
+  __shared__ uint32_t s_warp_hm[kThreads / 32];
+  __shared__ unsigned long long s_excl, s_inc;
+  __shared__ uint32_t s_hbase, s_mbase;
+  __shared__ uint32_t s_lid[kCompactTile];
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
   const uint32_t flat = n_l * k;
@@ -382,32 +389,61 @@ __global__ void __launch_bounds__(kThreads)
     __syncthreads();
     const uint32_t tile = s_tile;
     if (tile >= ntiles) break;
-    const uint32_t f0 = tile * kCompactTile + threadIdx.x * kCompactItems;
+    const uint32_t t0 = tile * kCompactTile;
+    const uint32_t l0 = threadIdx.x * kCompactItems;  // first local position of this thread
+    const uint32_t f0 = t0 + l0;
     uint32_t u[kCompactItems];
-    uint32_t flags = 0;  // bit i: valid, bit 16+i: new
+    unsigned long long e[kCompactItems];
+    if (f0 + kCompactItems <= flat) {
+      const uint4 a = *reinterpret_cast<const uint4*>(picks + f0);
+      const uint4 b = *reinterpret_cast<const uint4*>(picks + f0 + 4);
+      u[0] = a.x; u[1] = a.y; u[2] = a.z; u[3] = a.w;
+      u[4] = b.x; u[5] = b.y; u[6] = b.z; u[7] = b.w;
+    } else {
 #pragma unroll
-    for (int i = 0; i < kCompactItems; ++i) {
-      const uint32_t f = f0 + i;
-      u[i] = f < flat ? picks[f] : kEmpty;
+      for (int i = 0; i < kCompactItems; ++i) u[i] = f0 + i < flat ? picks[f0 + i] : kEmpty;
     }
+    uint32_t flags = 0;  // bit i: valid, bit 8+i: new, bit 16+i: new and cached
 #pragma unroll
     for (int i = 0; i < kCompactItems; ++i) {
+      e[i] = 0;
       if (u[i] != kEmpty) {
         flags |= 1u << i;
-        if (__ldg(vmap + u[i]) == enc_pos(gen, base + f0 + i)) flags |= 1u << (16 + i);
+        e[i] = __ldg(vmap + u[i]);
+        if (e[i] == enc_pos(gen, base + f0 + i)) flags |= 1u << (8 + i);
       }
     }
-    const unsigned long long mine =
-        ((unsigned long long)__popc(flags >> 16) << 32) | (unsigned)__popc(flags & 0xFFFFu);
-    // block exclusive scan of (new, valid)
-    const unsigned long long incl = warp_incl_scan64(mine);
-    if (lane == 31) s_warp[wid] = incl;
+    int32_t sl[kCompactItems];
+#pragma unroll
+    for (int i = 0; i < kCompactItems; ++i) {
+      sl[i] = -1;
+      if ((flags >> (8 + i)) & 1u) {
+        sl[i] = __ldg(mk.slot + u[i]);
+        if (sl[i] >= 0) flags |= 1u << (16 + i);
+      }
+    }
+    const uint32_t nnew = __popc((flags >> 8) & 0xFFu), nval = __popc(flags & 0xFFu);
+    const uint32_t nhit = __popc((flags >> 16) & 0xFFu);
+    const unsigned long long mine = ((unsigned long long)nnew << 32) | nval;
+    const uint32_t mine_hm = nhit | ((nnew - nhit) << 16);
+    const unsigned long long incl = warp_incl_scan(mine);
+    const uint32_t incl_hm = warp_incl_scan(mine_hm);
+    if (lane == 31) {
+      s_warp[wid] = incl;
+      s_warp_hm[wid] = incl_hm;
+    }
     __syncthreads();
     if (wid == 0) {
-      unsigned long long x = lane < kThreads / 32 ? s_warp[lane] : 0ull;
-      const unsigned long long xi = warp_incl_scan64(x);
-      if (lane < kThreads / 32) s_warp[lane] = xi - x;  // exclusive warp offsets
+      const unsigned long long x = lane < kThreads / 32 ? s_warp[lane] : 0ull;
+      const unsigned long long xi = warp_incl_scan(x);
+      const uint32_t y = lane < kThreads / 32 ? s_warp_hm[lane] : 0u;
+      const uint32_t yi = warp_incl_scan(y);
+      if (lane < kThreads / 32) {
+        s_warp[lane] = xi - x;  // exclusive warp offsets
+        s_warp_hm[lane] = yi - y;
+      }
       const unsigned long long agg = __shfl_sync(kFull, xi, kThreads / 32 - 1);
+      const uint32_t agg_hm = __shfl_sync(kFull, yi, kThreads / 32 - 1);
       // decoupled look-back
       unsigned long long excl = 0;
       if (tile == 0) {
@@ -423,7 +459,7 @@ __global__ void __launch_bounds__(kThreads)
               wv = *((volatile unsigned long long*)(status + jx));
             } while ((wv >> 62) == 0);
           }
-          const uint32_t incm = __ballot_sync(kFull, (wv >> 62) == 2);
+          const uint32_t incm = __ballot_sync(kFull, (wv >> 62) >= 2);
           if (incm) {
             const int firsti = __ffs(incm) - 1;
             excl += warp_sum64(lane <= firsti ? unpack_pair(wv) : 0ull);
@@ -436,56 +472,79 @@ __global__ void __launch_bounds__(kThreads)
       }
       if (lane == 0) {
         s_excl = excl;
+        s_inc = excl + agg;
+        s_hbase = (agg_hm & 0xFFFFu) ? atomicAdd(&st->nhit, agg_hm & 0xFFFFu) : 0u;
+        s_mbase = (agg_hm >> 16) ? atomicAdd(&st->nmiss, agg_hm >> 16) : 0u;
         if (tile == ntiles - 1) {
           const unsigned long long tot = excl + agg;
-          const uint32_t nnew = (uint32_t)(tot >> 32), nval = (uint32_t)tot;
-          st->n[hop + 1] = n_l + nnew;
-          st->nnz[hop] = nval;
+          st->n[hop + 1] = n_l + (uint32_t)(tot >> 32);
+          st->nnz[hop] = (uint32_t)tot;
           st->base[hop + 1] = base + flat;
-          bindptr[n_l] = nval;
+          bindptr[n_l] = (uint32_t)tot;
         }
       }
     }
     __syncthreads();
-    unsigned long long run = s_excl + s_warp[wid] + (incl - mine);
-    uint32_t d = f0 / k, s = f0 - d * k;
+    const unsigned long long run0 = s_excl + s_warp[wid] + (incl - mine);
+    const uint32_t hm0 = s_warp_hm[wid] + (incl_hm - mine_hm);
+    // 3. new vertices
+    {
+      uint32_t en = (uint32_t)(run0 >> 32);
+      uint32_t h = s_hbase + (hm0 & 0xFFFFu), m = s_mbase + (hm0 >> 16);
 #pragma unroll
-    for (int i = 0; i < kCompactItems; ++i) {
-      const uint32_t f = f0 + i;
-      const uint32_t ev = (uint32_t)run, en = (uint32_t)(run >> 32);
-      const bool valid = (flags >> i) & 1u;
-      const bool isnew = (flags >> (16 + i)) & 1u;
-      if (f < flat) {
-        if (s == 0) bindptr[d] = ev;
-        if (valid) {
-          bindices[ev] = u[i];  // gid; k_remap turns it into a lid
-          if (W) bweights[ev] = pickw[f];
+      for (int i = 0; i < kCompactItems; ++i) {
+        if ((flags >> (8 + i)) & 1u) {
+          const uint32_t lid = n_l + en;
+          uniq[lid] = u[i];
+          lidmap[u[i]] = lid;
+          mk.lidslot[lid] = sl[i];
+          if (sl[i] >= 0) mk.hit_list[h++] = make_uint2(lid, (uint32_t)sl[i]);
+          else mk.miss_list[m++] = make_uint2(lid, u[i]);
+          if (mk.count) atomicAdd(mk.count + u[i], 1u);
+          s_lid[l0 + i] = lid;
+          ++en;
         }
       }
-      int32_t sl = -1;
-      const uint32_t lid = n_l + en;
-      if (isnew) {
-        uniq[lid] = u[i];
-        lidmap[u[i]] = lid;
-        sl = __ldg(mk.slot + u[i]);
-        mk.lidslot[lid] = sl;
-        if (mk.count) atomicAdd(mk.count + u[i], 1u);
+    }
+    __threadfence();
+    __syncthreads();
+    if (threadIdx.x == 0) atomicExch(status + tile, pack_status(kFlagDone, s_inc));
+    // 4. edges (src lids) and block indptr
+    {
+      uint32_t ev = (uint32_t)run0;
+      uint32_t d = f0 / k, s = f0 - d * k;
+#pragma unroll
+      for (int i = 0; i < kCompactItems; ++i) {
+        const uint32_t f = f0 + i;
+        if (f < flat && s == 0) bindptr[d] = ev;
+        if (flags & (1u << i)) {
+          uint32_t lid;
+          if ((flags >> (8 + i)) & 1u) {
+            lid = s_lid[l0 + i];
+          } else {
+            const uint32_t p = (uint32_t)e[i];  // first position of u in this batch
+            const uint32_t fp = p - base;       // ... as a flat index of this hop
+            if (p < base) {
+              lid = __ldcg(lidmap + u[i]);      // discovered by an earlier hop / a seed
+            } else if (fp >= t0) {
+              lid = s_lid[fp - t0];             // first seen earlier in this tile
+            } else {
+              const uint32_t tp = fp / kCompactTile;
+              while ((*((volatile unsigned long long*)(status + tp)) >> 62) != 3) {
+              }
+              __threadfence();
+              lid = __ldcg(lidmap + u[i]);
+            }
+          }
+          bindices[ev] = lid;
+          if (W) bweights[ev] = pickw[f];
+          ++ev;
+        }
+        if (++s == k) { s = 0; ++d; }
       }
-      warp_append(isnew && sl >= 0, &st->nhit, mk.hit_dst, mk.hit_src, lid, (uint32_t)sl);
-      warp_append(isnew && sl < 0, &st->nmiss, mk.miss_dst, mk.miss_src, lid, u[i]);
-      run += ((unsigned long long)isnew << 32) | (unsigned)valid;
-      if (++s == k) { s = 0; ++d; }
     }
     __syncthreads();
   }
-}
-
-__global__ void __launch_bounds__(kThreads)
-    k_remap(uint32_t hop, const DevState* __restrict__ st, const uint32_t* __restrict__ lidmap,
-            uint32_t* __restrict__ bindices) {
-  const uint32_t nnz = st->nnz[hop];
-  for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x)
-    bindices[e] = __ldg(lidmap + bindices[e]);
 }
 
 __global__ void k_validate(const uint64_t* __restrict__ indptr, const uint32_t* __restrict__ indices,
@@ -505,10 +564,8 @@ MarkArgs mark_args(glb_ctx* c, int count_mode) {
   MarkArgs m;
   m.slot = c->slot;
   m.lidslot = c->sb.lidslot;
-  m.hit_dst = c->sb.hit_dst;
-  m.hit_src = c->sb.hit_src;
-  m.miss_dst = c->sb.miss_dst;
-  m.miss_src = c->sb.miss_src;
+  m.hit_list = c->sb.hit_list;
+  m.miss_list = c->sb.miss_list;
   m.count = count_mode == GLB_COUNT_PRESAMPLE ? c->counts
             : count_mode == GLB_COUNT_ACCESS  ? c->access
                                               : nullptr;
@@ -543,15 +600,12 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
                         uint32_t batch) {
   const int grid = grid_for(c);
   const SampleBufs& b = c->sb;
-#define GLB_KHOP_ARGS                                                                  \
-  hop, k, seed, epoch, batch, c->gen, c->st, c->st, c->indptr, c->indices, b.uniq, c->vmap, \
-      b.picks
-  if (k <= 4) k_khop<4><<<grid, kThreads, 0, c->stream>>>(GLB_KHOP_ARGS);
-  else if (k <= 8) k_khop<8><<<grid, kThreads, 0, c->stream>>>(GLB_KHOP_ARGS);
-  else if (k <= 16) k_khop<16><<<grid, kThreads, 0, c->stream>>>(GLB_KHOP_ARGS);
-  else if (k <= 32) k_khop<32><<<grid, kThreads, 0, c->stream>>>(GLB_KHOP_ARGS);
-  else k_khop_wide<<<grid, kThreads, 0, c->stream>>>(GLB_KHOP_ARGS);
-#undef GLB_KHOP_ARGS
+  if (k <= 32)
+    k_khop<<<grid, kThreads, 0, c->stream>>>(hop, k, seed, epoch, batch, c->gen, c->st, c->st,
+                                             c->indptr, c->indices, b.uniq, c->vmap, b.picks);
+  else
+    k_khop_wide<<<grid, kThreads, 0, c->stream>>>(hop, k, seed, epoch, batch, c->gen, c->st, c->st,
+                                                  c->indptr, c->indices, b.uniq, c->vmap, b.picks);
   count_launch(c);
   return cudaGetLastError();
 }
@@ -585,12 +639,6 @@ cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, 
     k_compact<false><<<grid, kThreads, 0, c->stream>>>(
         hop, k, c->gen, c->st, b.picks, nullptr, c->vmap, c->lidmap, b.uniq, b.bindptr[hop],
         b.bindices[hop], nullptr, b.status[hop], mark_args(c, count_mode));
-  count_launch(c);
-  return cudaGetLastError();
-}
-
-cudaError_t launch_remap(glb_ctx* c, uint32_t hop) {
-  k_remap<<<grid_for(c), kThreads, 0, c->stream>>>(hop, c->st, c->lidmap, c->sb.bindices[hop]);
   count_launch(c);
   return cudaGetLastError();
 }
