@@ -22,7 +22,6 @@ import json
 import math
 import os
 import statistics
-import subprocess
 import sys
 import time
 
@@ -39,7 +38,7 @@ METRIC = "sample+extract seeds/sec at 1/2/4/8 B200; cache hit rate vs optimal (%
 def parse():
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
-    p.add_argument("--steps", type=int, default=50)
+    p.add_argument("--steps", type=int, default=400)
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--config", default="PR", choices=list(synth.SHAPES))
@@ -49,6 +48,8 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
     p.add_argument("--measure-epochs", type=int, default=2)
+    p.add_argument("--pipeline", type=int, default=1, choices=[1, 2],
+                   help="2: extract of batch b overlaps sampling of batch b+1 (two streams)")
     return p.parse_args()
 
 
@@ -75,53 +76,60 @@ def read_peaks():
 
 
 class Clocks:
-    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    """SM clock + throttle reasons sampled DURING the timed region (B200_PROFILING.md
+    clocks line), via NVML from a background thread every ~2 ms (ctypes and CUDA
+    syncs release the GIL).  Falls back to None when NVML is unavailable."""
 
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    REASONS = {"hw_slowdown": "nvmlClocksEventReasonHwSlowdown",
+               "hw_thermal_slowdown": "nvmlClocksEventReasonHwThermalSlowdown",
+               "sw_thermal_slowdown": "nvmlClocksEventReasonSwThermalSlowdown",
+               "sw_power_cap": "nvmlClocksEventReasonSwPowerCap",
+               "hw_power_brake": "nvmlClocksEventReasonHwPowerBrakeSlowdown"}
 
     def __init__(self, index):
         self.index = index
-        self.p = None
-        self.path = os.path.join("/tmp", f"glb_clocks_{os.getpid()}.csv")
+        self.ok = False
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+            phys = int(vis.split(",")[index]) if vis and vis.split(",")[0].isdigit() else index
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(phys)
+            self.nv = pynvml
+            self.max = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception:
+            pass
+
+    def _run(self):
+        nv = self.nv
+        while not self.stop_flag:
+            try:
+                self.sm.append(nv.nvmlDeviceGetClockInfo(self.h, nv.NVML_CLOCK_SM))
+                self.rs |= nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+            except Exception:
+                pass
+            time.sleep(0.002)
 
     def start(self):
-        try:
-            self.f = open(self.path, "w")
-            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                                       "-i", str(self.index), "-lms", "100"], stdout=self.f,
-                                      stderr=subprocess.DEVNULL)
-        except (OSError, FileNotFoundError):
-            self.p = None
+        if not self.ok:
+            return
+        import threading
+        self.sm, self.rs, self.stop_flag = [], 0, False
+        self.th = threading.Thread(target=self._run, daemon=True)
+        self.th.start()
 
     def stop(self):
-        if self.p is None:
+        if not self.ok:
             return None
-        self.p.terminate()
-        try:
-            self.p.wait(timeout=5)
-        except subprocess.TimeoutExpired:
-            self.p.kill()
-        self.f.close()
-        sm, mx, reasons = [], None, set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for line in open(self.path):
-            parts = [x.strip() for x in line.split(",")]
-            if len(parts) < 9:
-                continue
-            try:
-                sm.append(float(parts[1]))
-                mx = float(parts[2])
-            except ValueError:
-                continue
-            for nm, v in zip(names, parts[5:9]):
-                if v.lower().startswith("active"):
-                    reasons.add(nm)
-        if not sm:
+        self.stop_flag = True
+        self.th.join()
+        if not self.sm:
             return None
-        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": mx, "reasons": sorted(reasons),
-                "samples": len(sm)}
+        reasons = sorted(k for k, a in self.REASONS.items()
+                         if hasattr(self.nv, a) and self.rs & getattr(self.nv, a))
+        return {"sm_mhz": statistics.median(self.sm), "sm_max_mhz": self.max,
+                "reasons": reasons, "samples": len(self.sm), "source": "nvml"}
 
 
 # ------------------------------------------------------------------------------------------
@@ -258,40 +266,43 @@ def main():
     def n_seeds(b):
         return min(sh.batch, sh.n_train - b * sh.batch)
 
+    ctx.set_pipeline(args.pipeline)
+    xs = ctx.extract_stream()
+
     # ---- warmup
     for i in range(args.warmup):
         e, b = batch_of(i)
         ctx.sample_batch(e, b)
         ctx.extract_sample(out)
+    ctx.sync()
     torch.cuda.synchronize()
 
-    # ---- timed region: device time, CUDA events on the launching stream
+    # ---- timed region: device time, CUDA events on the launching streams (sampling on the
+    # main stream, extract on the extract stream; the last kernel of the region is an extract)
     steps = list(range(args.warmup, args.warmup + args.steps))
-    ev_x = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-            for _ in steps]
     clocks = Clocks(local)
     launches0 = ctx.launches
     barrier()
     torch.cuda.synchronize()
+    ctx.set_timing(True)
     clocks.start()
     t_start = torch.cuda.Event(enable_timing=True)
     t_end = torch.cuda.Event(enable_timing=True)
     t_start.record(stream)
     seeds_done = 0
-    for j, i in enumerate(steps):
+    for i in steps:
         e, b = batch_of(i)
         ctx.sample_batch(e, b)
-        ev_x[j][0].record(stream)
         ctx.extract_sample(out)
-        ev_x[j][1].record(stream)
         seeds_done += n_seeds(b)
-    t_end.record(stream)
+    t_end.record(xs)
     torch.cuda.synchronize()
     barrier()
     clk = clocks.stop()
     launches = ctx.launches - launches0
+    x_ms = ctx.extract_times()
+    ctx.set_timing(False)
     elapsed_ms = t_start.elapsed_time(t_end)
-    x_ms = [a.elapsed_time(bb) for a, bb in ev_x]
     el = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
     tot = torch.tensor([float(seeds_done)], dtype=torch.float64, device=dev)
     if world > 1:
@@ -383,7 +394,7 @@ def main():
                 ctx.sample_batch(e, b)
                 ctx.extract_sample(out)
                 sd += n_seeds(b)
-            s1.record(stream)
+            s1.record(xs)
             torch.cuda.synchronize()
             ms = s0.elapsed_time(s1)
             sweep.append({"alpha": a, "cache_rows": hs["cache_rows"], "hit_rate": H,
@@ -409,6 +420,7 @@ def main():
                        "presample_K": sh.K, "parallelism": f"dp{world}",
                        "l2": "inputs larger than L2 (CSR %.2f GB, feature cache %.2f GB vs 126 MB L2)"
                              % ((8 * (sh.V + 1) + 4 * sh.E) / 1e9, 4 * sh.D * sh.V * args.alpha / 1e9)},
+            "pipeline_depth": args.pipeline,
             "roofline": {"kernel": "k_gather (extract a7)", "bound": "hbm", "achieved": ach_gbs,
                          "peak": peak, "unit": "GB/s", "frac": ach_gbs / peak, "traffic": traffic,
                          "peak_source": peak_src,

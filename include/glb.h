@@ -172,6 +172,22 @@ glb_status glb_extract(glb_ctx* ctx, const uint32_t* vertices, uint64_t n, void*
  * using the marks taken during relabel; no host sync. */
 glb_status glb_extract_sample(glb_ctx* ctx, void* out, glb_extract_stats* stats);
 
+/* Pipelining (Extract || Sample, "pipelining mechanism ... to overlap
+ * the Extract and Train stages", L217 the Sampler/Trainer queue): depth 2 double-buffers
+ * the sample slots; glb_extract_sample then runs on the ctx's extract stream, ordered
+ * after everything enqueued on the main stream before the call (the sample it reads,
+ * the caller's allocation of `out`), while the next glb_sample_batch proceeds on the
+ * main stream (it waits only for the extract that last read its slot).  The caller
+ * must order its reads of `out` after the extract stream (glb_extract_stream).  depth 1 (default): all
+ * work on the main stream.  Synchronous. */
+glb_status glb_set_pipeline(glb_ctx* ctx, int depth);
+glb_status glb_extract_stream(glb_ctx* ctx, void** cuda_stream_out);
+/* Timing of the extract kernel itself (CUDA events around each glb_extract_sample launch,
+ * on the stream it runs on).  glb_extract_times synchronises, returns the durations in
+ * call order (up to max) and resets the record. */
+glb_status glb_set_timing(glb_ctx* ctx, int enable);
+glb_status glb_extract_times(glb_ctx* ctx, float* out_ms, uint64_t max, uint64_t* n);
+
 /* launch counter: number of kernels this ctx launched so far (bench evidence) */
 uint64_t glb_kernel_launches(const glb_ctx* ctx);
 

@@ -34,6 +34,7 @@ EXPORTS = [
     "glb_set_count_mode", "glb_reset_counts", "glb_presample", "glb_counts_device_ptr",
     "glb_get_counts", "glb_build_cache", "glb_get_cache_slots", "glb_cache_size",
     "glb_hit_stats_get", "glb_extract", "glb_extract_sample", "glb_kernel_launches",
+    "glb_set_pipeline", "glb_extract_stream", "glb_set_timing", "glb_extract_times",
 ]
 
 
@@ -108,6 +109,10 @@ def lib(auto_build: bool = True):
         "glb_extract": ([vp, vp, u64, vp, ctypes.POINTER(_XStats)], i32),
         "glb_extract_sample": ([vp, vp, ctypes.POINTER(_XStats)], i32),
         "glb_kernel_launches": ([vp], u64),
+        "glb_set_pipeline": ([vp, i32], i32),
+        "glb_extract_stream": ([vp, ctypes.POINTER(vp)], i32),
+        "glb_set_timing": ([vp, i32], i32),
+        "glb_extract_times": ([vp, vp, u64, ctypes.POINTER(u64)], i32),
     }
     for name, (a, r) in sig.items():
         f = getattr(L, name)
@@ -357,6 +362,28 @@ class Context:
             self.sync()
             return {"hits": st.hits, "misses": st.misses}
         return None
+
+    def set_pipeline(self, depth: int):
+        """depth 2: double-buffered samples, extract on its own stream overlapping the
+        next sample (see include/glb.h glb_set_pipeline)."""
+        self._ck(self._lib.glb_set_pipeline(self._h, depth))
+
+    def extract_stream(self):
+        """torch stream the extracts run on (order consumers of ``out`` after it)."""
+        import torch
+        p = ctypes.c_void_p()
+        self._ck(self._lib.glb_extract_stream(self._h, ctypes.byref(p)))
+        return torch.cuda.ExternalStream(p.value or 0, device=self.device)
+
+    def set_timing(self, enable: bool):
+        self._ck(self._lib.glb_set_timing(self._h, int(enable)))
+
+    def extract_times(self, max_n: int = 1 << 16) -> list:
+        """Durations (ms) of the extract kernels recorded since set_timing(True)."""
+        buf = np.zeros(max_n, np.float32)
+        n = ctypes.c_uint64()
+        self._ck(self._lib.glb_extract_times(self._h, buf.ctypes.data, max_n, ctypes.byref(n)))
+        return buf[:min(n.value, max_n)].tolist()
 
     @property
     def launches(self) -> int:

@@ -15,6 +15,8 @@ ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-I" + INCLUDE,
          "--expt-relaxed-constexpr"]
+if os.environ.get("GLB_TRACE"):  # debug timeline build (tools/trace_compact.py)
+    FLAGS.append("-DGLB_TRACE")
 
 
 def sources():

@@ -6,6 +6,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 
@@ -60,19 +61,34 @@ cudaError_t dalloc(T** p, uint64_t count) {
 }
 
 void free_sample_bufs(glb_ctx* c) {
-  SampleBufs& b = c->sb;
-  dfree(b.seeds); dfree(b.uniq); dfree(b.lidslot); dfree(b.picks); dfree(b.pickw);
-  for (int l = 0; l < GLB_MAX_HOPS; ++l) {
-    dfree(b.bindptr[l]); dfree(b.bindices[l]); dfree(b.bweights[l]); dfree(b.status[l]);
+  for (int s = 0; s < 2; ++s) {
+    SampleBufs& b = c->sbs[s];
+    dfree(b.seeds); dfree(b.uniq); dfree(b.lidslot); dfree(b.picks); dfree(b.pickw);
+    for (int l = 0; l < GLB_MAX_HOPS; ++l) {
+      dfree(b.bindptr[l]); dfree(b.bindices[l]); dfree(b.bweights[l]); dfree(b.status[l]);
+    }
+    dfree(b.hit_list); dfree(b.miss_list);
+    b = SampleBufs();
   }
-  dfree(b.hit_list); dfree(b.miss_list);
-  b = SampleBufs();
+  c->sb = SampleBufs();
   c->sampler_set = false;
   c->have_sample = false;
 }
 
+void use_slot(glb_ctx* c, int s) {
+  c->cur = s;
+  c->sb = c->sbs[s];
+  c->st = c->sts[s];
+}
+
+cudaError_t sync_all(glb_ctx* c) {
+  cudaError_t e = cudaStreamSynchronize(c->stream);
+  if (e == cudaSuccess && c->xstream) e = cudaStreamSynchronize(c->xstream);
+  return e;
+}
+
 void free_graph(glb_ctx* c) {
-  dfree(c->indptr); dfree(c->indices); dfree(c->vmap); dfree(c->lidmap);
+  dfree(c->indptr); dfree(c->indices); dfree(c->vmap);
   dfree(c->slot); dfree(c->cache); dfree(c->counts); dfree(c->access);
   if (c->registered && c->h_features) cudaHostUnregister((void*)c->h_features);
   c->registered = false;
@@ -113,6 +129,10 @@ glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, in
     c->gen = 0;
   }
   c->gen += 1;
+  const int slot = c->nslots == 2 ? c->cur ^ 1 : 0;
+  // the extract that last read this slot must finish before it is overwritten
+  if (c->nslots == 2) CK(cudaStreamWaitEvent(c->stream, c->ev_extracted[slot], 0));
+  use_slot(c, slot);
   CK(cudaMemsetAsync(c->st, 0, sizeof(DevState), c->stream));
   const int mode = c->count_mode;
   CK(launch_seed_init(c, seeds_dev, n0, mode));
@@ -121,6 +141,7 @@ glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, in
     else CK(launch_rwalk(c, l, seed, epoch, batch));
     CK(launch_compact(c, l, k[l], kind == GLB_RANDOM_WALK, mode));
   }
+  if (L) CK(launch_fixup(c, L - 1));  // blocks 0..L-2 were fixed inside the next hop's kernel
   c->have_sample = true;
   c->last_L = L;
   c->last_kind = kind;
@@ -157,19 +178,28 @@ glb_status glb_create(int device, glb_ctx** out) {
   if ((e = cudaSetDevice(device)) != cudaSuccess ||
       (e = cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device)) != cudaSuccess ||
       (e = cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking)) != cudaSuccess ||
-      (e = cudaMalloc(&c->st, sizeof(DevState))) != cudaSuccess ||
+      (e = cudaStreamCreateWithFlags(&c->xstream, cudaStreamNonBlocking)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_sampled[0], cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_sampled[1], cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_extracted[0], cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_extracted[1], cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaMalloc(&c->sts[0], sizeof(DevState))) != cudaSuccess ||
+      (e = cudaMalloc(&c->sts[1], sizeof(DevState))) != cudaSuccess ||
       (e = cudaMalloc(&c->st_x, sizeof(DevState))) != cudaSuccess ||
       (e = cudaMalloc(&c->scratch, 4 * sizeof(unsigned long long))) != cudaSuccess ||
       (e = cudaMalloc(&c->xcount, 2 * sizeof(unsigned long long))) != cudaSuccess ||
       (e = cudaMallocHost(&c->h_st, sizeof(DevState))) != cudaSuccess ||
       (e = cudaMallocHost(&c->h_xcount, 2 * sizeof(unsigned long long))) != cudaSuccess ||
-      (e = cudaMemset(c->st, 0, sizeof(DevState))) != cudaSuccess ||
+      (e = cudaMemset(c->sts[0], 0, sizeof(DevState))) != cudaSuccess ||
+      (e = cudaMemset(c->sts[1], 0, sizeof(DevState))) != cudaSuccess ||
       (e = cudaMemset(c->st_x, 0, sizeof(DevState))) != cudaSuccess) {
     glb_status s = set_err(nullptr, GLB_ECUDA, "glb_create: %s", cudaGetErrorString(e));
     glb_destroy(c);
     return s;
   }
   c->stream = c->own_stream;
+  c->st = c->sts[0];
+  if (const char* g = getenv("GLB_GATHER_BPS")) c->gather_bps = atoi(g) > 0 ? atoi(g) : 4;
   *out = c;
   return GLB_OK;
 }
@@ -178,11 +208,18 @@ glb_status glb_destroy(glb_ctx* c) {
   if (!c) return GLB_OK;
   cudaSetDevice(c->device);
   if (c->stream) cudaStreamSynchronize(c->stream);
+  if (c->xstream) cudaStreamSynchronize(c->xstream);
   free_sample_bufs(c);
   free_graph(c);
   dfree(c->xb.hit_list); dfree(c->xb.miss_list);
   dfree(c->train); dfree(c->perm); dfree(c->shuf_keys); dfree(c->shuf_vals);
-  dfree(c->st); dfree(c->st_x); dfree(c->scratch); dfree(c->xcount);
+  dfree(c->sts[0]); dfree(c->sts[1]); dfree(c->st_x); dfree(c->scratch); dfree(c->xcount);
+  for (int i = 0; i < 2; ++i) {
+    if (c->ev_sampled[i]) cudaEventDestroy(c->ev_sampled[i]);
+    if (c->ev_extracted[i]) cudaEventDestroy(c->ev_extracted[i]);
+  }
+  for (cudaEvent_t ev : c->tev) cudaEventDestroy(ev);
+  if (c->xstream) cudaStreamDestroy(c->xstream);
   if (c->sort_tmp) cudaFree(c->sort_tmp);
   if (c->h_st) cudaFreeHost(c->h_st);
   if (c->h_xcount) cudaFreeHost(c->h_xcount);
@@ -199,7 +236,7 @@ glb_status glb_set_stream(glb_ctx* c, void* s) {
 
 glb_status glb_sync(glb_ctx* c) {
   ENTER(c);
-  CK(cudaStreamSynchronize(c->stream));
+  CK(sync_all(c));
   if (c->pending_stats) {
     c->pending_stats->hits = c->h_xcount[0];
     c->pending_stats->misses = c->h_xcount[1];
@@ -213,11 +250,11 @@ glb_status glb_sync(glb_ctx* c) {
 glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* indptr,
                           const uint32_t* indices, const void* features, uint32_t D) {
   ENTER(c);
-  if (V == 0 || V >= 0xFFFFFFFFull) return set_err(c, GLB_EINVAL, "V=%llu out of range", (unsigned long long)V);
+  if (V == 0 || V >= 0x80000000ull) return set_err(c, GLB_EINVAL, "V=%llu out of range [1, 2^31)", (unsigned long long)V);
   if (!indptr || (E && !indices)) return set_err(c, GLB_EINVAL, "null CSR");
   if (indptr[0] != 0 || indptr[V] != E) return set_err(c, GLB_EINVAL, "indptr[0]!=0 or indptr[V]!=E");
   if (features && D == 0) return set_err(c, GLB_EINVAL, "feat_dim 0");
-  CK(cudaStreamSynchronize(c->stream));
+  CK(sync_all(c));
   free_graph(c);
   free_sample_bufs(c);
   c->V = V;
@@ -225,7 +262,6 @@ glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* in
   CK(dalloc(&c->indptr, V + 1));
   CK(dalloc(&c->indices, E));
   CK(dalloc(&c->vmap, V));
-  CK(dalloc(&c->lidmap, V));
   CK(dalloc(&c->slot, V));
   CK(dalloc(&c->counts, V));
   CK(dalloc(&c->access, V));
@@ -284,9 +320,9 @@ glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32
   } else {
     return set_err(c, GLB_EINVAL, "unknown sampler kind %d", kind);
   }
-  CK(cudaStreamSynchronize(c->stream));
+  CK(sync_all(c));
   free_sample_bufs(c);
-  SampleBufs& b = c->sb;
+  SampleBufs b;
   b.cap_batch = max_batch;
   b.L = L;
   b.ub[0] = max_batch < c->V ? max_batch : c->V;
@@ -302,21 +338,26 @@ glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32
   }
   if (pos >= 0xFFFFFFFFull) return set_err(c, GLB_ENOMEM, "relabel positions overflow 2^32");
   const uint64_t un = b.ub[L] > max_batch ? b.ub[L] : max_batch;
-  CK(dalloc(&b.seeds, max_batch));
-  CK(dalloc(&b.uniq, un));
-  CK(dalloc(&b.lidslot, un));
-  CK(dalloc(&b.picks, maxflat));
-  if (kind == GLB_RANDOM_WALK) CK(dalloc(&b.pickw, maxflat));
-  for (uint32_t l = 0; l < L; ++l) {
-    const uint64_t flat = b.ub[l] * k[l];
-    CK(dalloc(&b.bindptr[l], b.ub[l] + 1));
-    CK(dalloc(&b.bindices[l], flat));
-    if (kind == GLB_RANDOM_WALK) CK(dalloc(&b.bweights[l], flat));
-    b.ntiles[l] = (flat + kCompactTile - 1) / kCompactTile;
-    CK(dalloc(&b.status[l], b.ntiles[l]));
+  for (int s = 1; s >= 0; --s) {  // two slots: pipeline depth 2 double-buffers samples
+    SampleBufs& bs = c->sbs[s];
+    bs = b;
+    CK(dalloc(&bs.seeds, max_batch));
+    CK(dalloc(&bs.uniq, un));
+    CK(dalloc(&bs.lidslot, un));
+    CK(dalloc(&bs.picks, maxflat));
+    if (kind == GLB_RANDOM_WALK) CK(dalloc(&bs.pickw, maxflat));
+    for (uint32_t l = 0; l < L; ++l) {
+      const uint64_t flat = bs.ub[l] * k[l];
+      CK(dalloc(&bs.bindptr[l], bs.ub[l] + 1));
+      CK(dalloc(&bs.bindices[l], flat));
+      if (kind == GLB_RANDOM_WALK) CK(dalloc(&bs.bweights[l], flat));
+      bs.ntiles[l] = (flat + kCompactTile - 1) / kCompactTile;
+      CK(dalloc(&bs.status[l], bs.ntiles[l]));
+    }
+    CK(dalloc(&bs.hit_list, un));
+    CK(dalloc(&bs.miss_list, un));
   }
-  CK(dalloc(&b.hit_list, un));
-  CK(dalloc(&b.miss_list, un));
+  use_slot(c, 0);
   c->kind = kind;
   c->L = L;
   for (uint32_t l = 0; l < L; ++l) c->fanouts[l] = k[l];
@@ -506,6 +547,7 @@ glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
   uint64_t C = (uint64_t)std::floor(alpha * (double)V);
   if (C > V) C = V;
   const uint32_t* hot = hotness ? hotness : c->counts;
+  CK(sync_all(c));  // an in-flight extract may still read the old cache
   uint32_t* tmp = nullptr;
   CK(dalloc(&tmp, 4 * V));
   uint32_t *k0 = tmp, *v0 = tmp + V, *k1 = tmp + 2 * V, *v1 = tmp + 3 * V;
@@ -613,12 +655,75 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
   if (!c->have_sample) return set_err(c, GLB_ESTATE, "extract_sample without a current sample");
   if (!c->features_mapped) return set_err(c, GLB_ESTATE, "graph loaded without features");
   if (!out) return set_err(c, GLB_EINVAL, "null out");
-  CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_list, c->sb.miss_list,
-                   nullptr, &c->st->nhit, 0, 0));
-  if (stats) {
-    CK(cudaMemcpyAsync(c->h_xcount, c->xcount, 2 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
+  cudaStream_t main = c->stream;
+  const int slot = c->cur;
+  if (c->nslots == 2) {  // extract on its own stream, overlapping the next sample;
+    // it is ordered after everything enqueued on the main stream so far (the sample it
+    // reads and any caller work, e.g. allocating `out`)
+    CK(cudaEventRecord(c->ev_sampled[slot], main));
+    CK(cudaStreamWaitEvent(c->xstream, c->ev_sampled[slot], 0));
+    c->stream = c->xstream;
+  }
+  cudaEvent_t t0 = nullptr, t1 = nullptr;
+  if (c->timing) {
+    if (c->tev_used + 2 > c->tev.size()) {
+      for (int i = 0; i < 2; ++i) {
+        cudaEvent_t ev;
+        cudaError_t e = cudaEventCreate(&ev);
+        if (e != cudaSuccess) { c->stream = main; return cuda_fail(c, e, "cudaEventCreate"); }
+        c->tev.push_back(ev);
+      }
+    }
+    t0 = c->tev[c->tev_used];
+    t1 = c->tev[c->tev_used + 1];
+    c->tev_used += 2;
+    cudaEventRecord(t0, c->stream);
+  }
+  cudaError_t e = launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_list,
+                                c->sb.miss_list, nullptr, &c->st->nhit, 0, 0);
+  if (e == cudaSuccess && t1) e = cudaEventRecord(t1, c->stream);
+  if (e == cudaSuccess && stats) {
+    e = cudaMemcpyAsync(c->h_xcount, c->xcount, 2 * sizeof(unsigned long long),
+                        cudaMemcpyDeviceToHost, c->stream);
     c->pending_stats = stats;
   }
+  if (e == cudaSuccess && c->nslots == 2) e = cudaEventRecord(c->ev_extracted[slot], c->stream);
+  c->stream = main;
+  if (e != cudaSuccess) return cuda_fail(c, e, "extract_sample");
+  return GLB_OK;
+}
+
+glb_status glb_set_pipeline(glb_ctx* c, int depth) {
+  ENTER(c);
+  if (depth != 1 && depth != 2) return set_err(c, GLB_EINVAL, "pipeline depth must be 1 or 2");
+  CK(sync_all(c));
+  c->nslots = depth;
+  return GLB_OK;
+}
+
+glb_status glb_extract_stream(glb_ctx* c, void** out) {
+  ENTER(c);
+  if (!out) return set_err(c, GLB_EINVAL, "null out");
+  *out = c->nslots == 2 ? (void*)c->xstream : (void*)c->stream;
+  return GLB_OK;
+}
+
+glb_status glb_set_timing(glb_ctx* c, int enable) {
+  ENTER(c);
+  CK(sync_all(c));
+  c->timing = enable != 0;
+  c->tev_used = 0;
+  return GLB_OK;
+}
+
+glb_status glb_extract_times(glb_ctx* c, float* out_ms, uint64_t max, uint64_t* n) {
+  ENTER(c);
+  CK(sync_all(c));
+  const uint64_t have = c->tev_used / 2;
+  if (n) *n = have;
+  for (uint64_t i = 0; i < have && i < max; ++i)
+    CK(cudaEventElapsedTime(out_ms + i, c->tev[2 * i], c->tev[2 * i + 1]));
+  c->tev_used = 0;
   return GLB_OK;
 }
 

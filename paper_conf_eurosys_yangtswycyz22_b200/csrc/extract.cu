@@ -160,7 +160,7 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   uint32_t R = kChunkUnits / U;
   if (R > (uint32_t)kThreads) R = kThreads;
   if (R < 1) R = 1;
-  const int grid = c->num_sms * 4;
+  const int grid = c->num_sms * c->gather_bps;
   if (vec)
     k_gather<float4><<<grid, kThreads, 0, c->stream>>>(
         (float4*)out, (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list,

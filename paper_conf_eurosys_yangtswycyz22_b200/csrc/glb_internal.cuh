@@ -13,7 +13,7 @@ namespace glb {
 
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr int kThreads = 256;          // block size of every grid-stride kernel
-constexpr int kCompactItems = 8;       // flat positions per thread in a compaction tile
+constexpr int kCompactItems = 16;      // flat positions per thread in a compaction tile
 constexpr int kCompactTile = kThreads * kCompactItems;
 constexpr int kMaxFanout = 1024;
 constexpr int kMaxWalkLen = 8;
@@ -115,8 +115,7 @@ struct glb_ctx {
   uint32_t D = 0;
 
   // relabel tables (D6): direct-address over gids
-  unsigned long long* vmap = nullptr;  // u64[V]
-  uint32_t* lidmap = nullptr;          // u32[V]
+  unsigned long long* vmap = nullptr;  // u64[V]: (gen, first position) then (gen, lid)
   uint32_t gen = 0;
 
   // cache (D3, D4, D5)
@@ -133,8 +132,18 @@ struct glb_ctx {
   uint32_t L = 0;
   uint32_t fanouts[GLB_MAX_HOPS] = {};
   uint32_t rw_walks = 4, rw_len = 3, rw_topk = 5;
-  glb::SampleBufs sb;
+  glb::SampleBufs sb;            // view of the current sample slot (sbs[cur])
+  glb::SampleBufs sbs[2];        // double-buffered sample slots (pipeline depth 2)
   glb::ExtractBufs xb;
+  int nslots = 1;                // pipeline depth (glb_set_pipeline)
+  int cur = 0;                   // slot of the last sample
+  cudaStream_t xstream = nullptr;  // extract stream (pipeline depth 2)
+  cudaEvent_t ev_sampled[2] = {nullptr, nullptr};
+  cudaEvent_t ev_extracted[2] = {nullptr, nullptr};
+  int gather_bps = 4;            // gather blocks per SM
+  bool timing = false;           // record per-extract kernel events
+  std::vector<cudaEvent_t> tev;  // pairs (start, end) of recorded extracts
+  size_t tev_used = 0;
 
   // training set (D9)
   uint32_t* train = nullptr;
@@ -152,7 +161,8 @@ struct glb_ctx {
   int last_kind = 0;
   uint32_t last_n0 = 0;
 
-  glb::DevState* st = nullptr;    // device: current sample
+  glb::DevState* st = nullptr;    // device: current sample (sts[cur])
+  glb::DevState* sts[2] = {nullptr, nullptr};
   glb::DevState* h_st = nullptr;  // pinned mirror
   glb::DevState* st_x = nullptr;  // device: generic glb_extract (mark lists, errors)
   unsigned long long* scratch = nullptr;  // device [4] u64 reductions
@@ -177,6 +187,7 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
                         uint32_t batch);
 cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch, uint32_t batch);
 cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, int count_mode);
+cudaError_t launch_fixup(glb_ctx* c, uint32_t hop);
 cudaError_t launch_mark(glb_ctx* c, const uint32_t* vertices, uint64_t n);
 // Gather rows: hits src_hit[list.y] -> out[list.x], misses src_miss[list.y] -> out[list.x];
 // fill_src (non-null) replaces miss_list with (r, fill_src[r]) (identity destination).

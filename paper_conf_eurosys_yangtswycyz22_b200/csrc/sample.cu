@@ -23,6 +23,23 @@
 
 #include "glb_internal.cuh"
 
+#ifdef GLB_TRACE
+// debug timeline of the compaction tiles: [hop][tile][event] = %globaltimer (ns)
+__device__ unsigned long long g_trace[GLB_MAX_HOPS][4096][8];
+extern "C" glb_status glb_trace_dump(void* host, size_t bytes) {
+  return cudaMemcpyFromSymbol(host, g_trace, bytes) == cudaSuccess ? GLB_OK : GLB_ECUDA;
+}
+__device__ __forceinline__ unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define TRACE(h, t, ev) \
+  do { if (threadIdx.x == 0 && (t) < 4096) ::g_trace[h][t][ev] = gtime(); } while (0)
+#else
+#define TRACE(h, t, ev) do {} while (0)
+#endif
+
 namespace glb {
 
 namespace {
@@ -44,6 +61,17 @@ __device__ __forceinline__ void vmap_insert(unsigned long long* vmap, uint32_t u
   if (old > e) atomicMin(vmap + u, e);
 }
 
+constexpr uint32_t kDefer = 0x80000000u;  // deferred src lid marker (gids < 2^31, glb_load_graph)
+
+// Resolve deferred src lids of block `hop` (entries gid | kDefer).
+__device__ __forceinline__ void fixup_block(uint32_t nnz, const unsigned long long* vmap,
+                                            uint32_t* __restrict__ bindices) {
+  for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x) {
+    const uint32_t x = bindices[e];
+    if (x & kDefer) bindices[e] = (uint32_t)__ldcg(vmap + (x & ~kDefer));  // (gen, lid)
+  }
+}
+
 struct MarkArgs {
   const int32_t* slot;
   int32_t* lidslot;
@@ -61,8 +89,8 @@ struct StatusArgs {  // look-back status arrays to clear for this batch
 // ---------------------------------------------------------------- seeds
 __global__ void __launch_bounds__(kThreads)
     k_seed_init(const uint32_t* __restrict__ seeds, uint32_t n0, uint64_t V, DevState* st,
-                uint32_t* __restrict__ uniq, unsigned long long* vmap, uint32_t* lidmap,
-                uint32_t gen, MarkArgs mk, StatusArgs za) {
+                uint32_t* __restrict__ uniq, unsigned long long* vmap, uint32_t gen, MarkArgs mk,
+                StatusArgs za) {
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     st->n[0] = n0;
     st->base[0] = n0;
@@ -84,8 +112,7 @@ __global__ void __launch_bounds__(kThreads)
         u = 0;  // keep later kernels in bounds; the batch is reported invalid
       }
       uniq[i] = u;
-      atomicMin(vmap + u, enc_pos(gen, i));
-      lidmap[u] = i;
+      atomicMin(vmap + u, enc_pos(gen, i));  // a seed's position is its lid
       s = __ldg(mk.slot + u);
       mk.lidslot[i] = s;
       if (mk.count) atomicAdd(mk.count + u, 1u);
@@ -111,7 +138,8 @@ __global__ void __launch_bounds__(kThreads)
     k_khop(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch, uint32_t gen,
            const DevState* __restrict__ st, DevState* st_w, const uint64_t* __restrict__ indptr,
            const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
-           unsigned long long* vmap, uint32_t* __restrict__ picks) {
+           unsigned long long* vmap, uint32_t* __restrict__ picks, uint32_t* fix_ind) {
+  if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);  // deferred lids of block hop-1
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
   const uint32_t c3 = ctr3(epoch, hop, kDomKhop);
@@ -175,8 +203,9 @@ __global__ void __launch_bounds__(kThreads)
                 uint32_t gen, const DevState* __restrict__ st, DevState* st_w,
                 const uint64_t* __restrict__ indptr, const uint32_t* __restrict__ indices,
                 const uint32_t* __restrict__ uniq, unsigned long long* vmap,
-                uint32_t* __restrict__ picks) {
+                uint32_t* __restrict__ picks, uint32_t* fix_ind) {
   __shared__ uint32_t chosen[kThreads / 32][kMaxFanout];
+  if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
   const uint32_t c3 = ctr3(epoch, hop, kDomKhop);
@@ -221,7 +250,9 @@ __global__ void __launch_bounds__(kThreads)
             uint32_t epoch, uint32_t batch, uint32_t gen, const DevState* __restrict__ st,
             DevState* st_w, const uint64_t* __restrict__ indptr,
             const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
-            unsigned long long* vmap, uint32_t* __restrict__ picks, uint32_t* __restrict__ pickw) {
+            unsigned long long* vmap, uint32_t* __restrict__ picks, uint32_t* __restrict__ pickw,
+            uint32_t* fix_ind) {
+  if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
   const uint32_t c3 = ctr3(epoch, hop, kDomRwalk);
@@ -312,11 +343,9 @@ __global__ void __launch_bounds__(kThreads)
 
 // ---------------------------------------------------------------- compaction scan
 // Status word of the decoupled look-back: [flag:2][new:31][valid:31].
-// flag 1 = aggregate, 2 = inclusive prefix, 3 = inclusive + this tile's lids
-// are written to lidmap (other tiles may read them).
+// flag 1 = aggregate, 2 = inclusive prefix.
 constexpr unsigned long long kFlagAgg = 1ull << 62;
 constexpr unsigned long long kFlagInc = 2ull << 62;
-constexpr unsigned long long kFlagDone = 3ull << 62;
 constexpr unsigned long long kValMask = (1ull << 62) - 1;
 
 __device__ __forceinline__ unsigned long long pack_status(unsigned long long flag,
@@ -345,35 +374,48 @@ __device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
   return x;
 }
 
-// One tile = kCompactTile consecutive (vertex, slot) positions of hop l.
+// One tile = kCompactTile consecutive (vertex, slot) positions of hop l; warp
+// w owns positions [w*512, w*512+512) of the tile and walks them 32 at a time
+// (lane = position), so every load and every compacted store is coalesced.
 //  1. valid = pick present; new = this position is the first occurrence
 //     (vmap holds the minimum position of this generation).
-//  2. block scan of (new, valid) + decoupled look-back -> global prefixes:
+//  2. warp ballots + block scan + decoupled look-back -> global prefixes:
 //     new vertices get lid n_l + new-prefix (first-occurrence order); valid
 //     picks get edge slot valid-prefix (block CSR in slot order).
-//  3. new vertices: uniq/lidmap/mark/count; tile publishes "lids written".
+//  3. new vertices: uniq / lidmap / mark lists / visit count.
 //  4. every edge's src lid: new -> own; repeat of a vertex first seen at an
-//     earlier position p: same tile -> shared memory, earlier tile -> wait for
-//     that tile's flag then lidmap; earlier hop (p < base) -> lidmap.
+//     earlier position p: same tile -> shared memory; relabelled already
+//     (vmap holds (gen, lid) with lid < base) -> that lid; earlier tile of
+//     this hop -> deferred: the entry holds gid | kDefer and fixup_block (in
+//     the next kernel) reads the lid from vmap once every tile has written.
+//  vmap doubles as the gid -> lid map: the first-occurrence tile overwrites
+//  (gen, position) with (gen, lid); lid <= position, so the table stays
+//  monotone (later atomicMins never replace it) and a concurrent reader sees
+//  either value, both of which it resolves correctly.
+constexpr int kWarpSpan = kCompactTile / (kThreads / 32);  // positions per warp
+
 template <bool W>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads, 4)
     k_compact(uint32_t hop, uint32_t k, uint32_t gen, DevState* st,
               const uint32_t* __restrict__ picks, const uint32_t* __restrict__ pickw,
-              const unsigned long long* __restrict__ vmap, uint32_t* lidmap,
+              unsigned long long* vmap,
               uint32_t* __restrict__ uniq, uint32_t* __restrict__ bindptr,
               uint32_t* __restrict__ bindices, uint32_t* __restrict__ bweights,
               unsigned long long* status, MarkArgs mk) {
+  constexpr int NW = kThreads / 32;
   __shared__ uint32_t s_tile;
-  __shared__ unsigned long long s_warp[kThreads / 32];
-  __shared__ uint32_t s_warp_hm[kThreads / 32];
-  __shared__ unsigned long long s_excl, s_inc;
+  __shared__ unsigned long long s_wnv[NW];  // per warp (new << 32 | valid), then exclusive
+  __shared__ uint32_t s_whm[NW];            // per warp (hit | miss << 16), then exclusive
+  __shared__ unsigned long long s_excl;
   __shared__ uint32_t s_hbase, s_mbase;
   __shared__ uint32_t s_lid[kCompactTile];
+  __shared__ int32_t s_slot[kCompactTile];
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
   const uint32_t flat = n_l * k;
   const uint32_t ntiles = (flat + kCompactTile - 1) / kCompactTile;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const uint32_t lt = lanemask_lt();
   if (flat == 0) {
     if (blockIdx.x == 0 && threadIdx.x == 0) {
       st->n[hop + 1] = n_l;
@@ -389,61 +431,66 @@ __global__ void __launch_bounds__(kThreads)
     __syncthreads();
     const uint32_t tile = s_tile;
     if (tile >= ntiles) break;
+    TRACE(hop, tile, 0);
     const uint32_t t0 = tile * kCompactTile;
-    const uint32_t l0 = threadIdx.x * kCompactItems;  // first local position of this thread
-    const uint32_t f0 = t0 + l0;
+    const uint32_t loc0 = wid * kWarpSpan + lane;  // local position of item 0
     uint32_t u[kCompactItems];
-    unsigned long long e[kCompactItems];
-    if (f0 + kCompactItems <= flat) {
-      const uint4 a = *reinterpret_cast<const uint4*>(picks + f0);
-      const uint4 b = *reinterpret_cast<const uint4*>(picks + f0 + 4);
-      u[0] = a.x; u[1] = a.y; u[2] = a.z; u[3] = a.w;
-      u[4] = b.x; u[5] = b.y; u[6] = b.z; u[7] = b.w;
-    } else {
-#pragma unroll
-      for (int i = 0; i < kCompactItems; ++i) u[i] = f0 + i < flat ? picks[f0 + i] : kEmpty;
-    }
-    uint32_t flags = 0;  // bit i: valid, bit 8+i: new, bit 16+i: new and cached
+    uint32_t p[kCompactItems];  // first position (this generation) of u[i]
 #pragma unroll
     for (int i = 0; i < kCompactItems; ++i) {
-      e[i] = 0;
+      const uint32_t f = t0 + loc0 + i * 32;
+      u[i] = f < flat ? picks[f] : kEmpty;
+    }
+    uint32_t vmask = 0, nmask = 0, hmask = 0;
+#pragma unroll
+    for (int i = 0; i < kCompactItems; ++i) {
+      p[i] = 0;
       if (u[i] != kEmpty) {
-        flags |= 1u << i;
-        e[i] = __ldg(vmap + u[i]);
-        if (e[i] == enc_pos(gen, base + f0 + i)) flags |= 1u << (8 + i);
+        vmask |= 1u << i;
+        const unsigned long long e = __ldcg(vmap + u[i]);  // position, or lid (< base) once relabelled
+        p[i] = (uint32_t)e;
+        if (e == enc_pos(gen, base + t0 + loc0 + i * 32)) nmask |= 1u << i;
       }
     }
-    int32_t sl[kCompactItems];
 #pragma unroll
     for (int i = 0; i < kCompactItems; ++i) {
-      sl[i] = -1;
-      if ((flags >> (8 + i)) & 1u) {
-        sl[i] = __ldg(mk.slot + u[i]);
-        if (sl[i] >= 0) flags |= 1u << (16 + i);
+      if ((nmask >> i) & 1u) {
+        const int32_t sl = __ldg(mk.slot + u[i]);
+        s_slot[loc0 + i * 32] = sl;
+        if (sl >= 0) hmask |= 1u << i;
       }
     }
-    const uint32_t nnew = __popc((flags >> 8) & 0xFFu), nval = __popc(flags & 0xFFu);
-    const uint32_t nhit = __popc((flags >> 16) & 0xFFu);
-    const unsigned long long mine = ((unsigned long long)nnew << 32) | nval;
-    const uint32_t mine_hm = nhit | ((nnew - nhit) << 16);
-    const unsigned long long incl = warp_incl_scan(mine);
-    const uint32_t incl_hm = warp_incl_scan(mine_hm);
-    if (lane == 31) {
-      s_warp[wid] = incl;
-      s_warp_hm[wid] = incl_hm;
+    TRACE(hop, tile, 1);
+    {  // warp totals
+      const uint32_t nn = __popc(nmask), nh = __popc(hmask);
+      unsigned long long nv = ((unsigned long long)nn << 32) | __popc(vmask);
+      uint32_t hm = nh | ((nn - nh) << 16);
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        nv += __shfl_xor_sync(kFull, nv, o);
+        hm += __shfl_xor_sync(kFull, hm, o);
+      }
+      if (lane == 0) {
+        s_wnv[wid] = nv;
+        s_whm[wid] = hm;
+      }
     }
     __syncthreads();
     if (wid == 0) {
-      const unsigned long long x = lane < kThreads / 32 ? s_warp[lane] : 0ull;
+      const unsigned long long x = lane < NW ? s_wnv[lane] : 0ull;
       const unsigned long long xi = warp_incl_scan(x);
-      const uint32_t y = lane < kThreads / 32 ? s_warp_hm[lane] : 0u;
+      const uint32_t y = lane < NW ? s_whm[lane] : 0u;
       const uint32_t yi = warp_incl_scan(y);
-      if (lane < kThreads / 32) {
-        s_warp[lane] = xi - x;  // exclusive warp offsets
-        s_warp_hm[lane] = yi - y;
+      if (lane < NW) {
+        s_wnv[lane] = xi - x;  // exclusive warp offsets
+        s_whm[lane] = yi - y;
       }
-      const unsigned long long agg = __shfl_sync(kFull, xi, kThreads / 32 - 1);
-      const uint32_t agg_hm = __shfl_sync(kFull, yi, kThreads / 32 - 1);
+      const unsigned long long agg = __shfl_sync(kFull, xi, NW - 1);
+      const uint32_t agg_hm = __shfl_sync(kFull, yi, NW - 1);
+      if (lane == 0) {  // list space for this tile's marks (independent of the look-back)
+        s_hbase = (agg_hm & 0xFFFFu) ? atomicAdd(&st->nhit, agg_hm & 0xFFFFu) : 0u;
+        s_mbase = (agg_hm >> 16) ? atomicAdd(&st->nmiss, agg_hm >> 16) : 0u;
+      }
       // decoupled look-back
       unsigned long long excl = 0;
       if (tile == 0) {
@@ -470,11 +517,9 @@ __global__ void __launch_bounds__(kThreads)
         }
         if (lane == 0) atomicExch(status + tile, pack_status(kFlagInc, excl + agg));
       }
+      TRACE(hop, tile, 2);
       if (lane == 0) {
         s_excl = excl;
-        s_inc = excl + agg;
-        s_hbase = (agg_hm & 0xFFFFu) ? atomicAdd(&st->nhit, agg_hm & 0xFFFFu) : 0u;
-        s_mbase = (agg_hm >> 16) ? atomicAdd(&st->nmiss, agg_hm >> 16) : 0u;
         if (tile == ntiles - 1) {
           const unsigned long long tot = excl + agg;
           st->n[hop + 1] = n_l + (uint32_t)(tot >> 32);
@@ -485,66 +530,75 @@ __global__ void __launch_bounds__(kThreads)
       }
     }
     __syncthreads();
-    const unsigned long long run0 = s_excl + s_warp[wid] + (incl - mine);
-    const uint32_t hm0 = s_warp_hm[wid] + (incl_hm - mine_hm);
-    // 3. new vertices
+    TRACE(hop, tile, 3);
+    const unsigned long long ex = s_excl + s_wnv[wid];
+    // 3. new vertices (compacted, coalesced)
     {
-      uint32_t en = (uint32_t)(run0 >> 32);
-      uint32_t h = s_hbase + (hm0 & 0xFFFFu), m = s_mbase + (hm0 >> 16);
+      uint32_t rn = (uint32_t)(ex >> 32);
+      uint32_t rh = s_hbase + (s_whm[wid] & 0xFFFFu), rm = s_mbase + (s_whm[wid] >> 16);
 #pragma unroll
       for (int i = 0; i < kCompactItems; ++i) {
-        if ((flags >> (8 + i)) & 1u) {
-          const uint32_t lid = n_l + en;
+        const bool isn = (nmask >> i) & 1u, ish = (hmask >> i) & 1u;
+        const uint32_t nb = __ballot_sync(kFull, isn);
+        const uint32_t hb = __ballot_sync(kFull, ish);
+        const uint32_t mb = nb & ~hb;
+        if (isn) {
+          const uint32_t loc = loc0 + i * 32;
+          const uint32_t lid = n_l + rn + __popc(nb & lt);
+          const int32_t sl = s_slot[loc];
           uniq[lid] = u[i];
-          lidmap[u[i]] = lid;
-          mk.lidslot[lid] = sl[i];
-          if (sl[i] >= 0) mk.hit_list[h++] = make_uint2(lid, (uint32_t)sl[i]);
-          else mk.miss_list[m++] = make_uint2(lid, u[i]);
+          __stcg(vmap + u[i], enc_pos(gen, lid));  // relabelled: later readers get the lid
+          mk.lidslot[lid] = sl;
+          if (ish) mk.hit_list[rh + __popc(hb & lt)] = make_uint2(lid, (uint32_t)sl);
+          else mk.miss_list[rm + __popc(mb & lt)] = make_uint2(lid, u[i]);
           if (mk.count) atomicAdd(mk.count + u[i], 1u);
-          s_lid[l0 + i] = lid;
-          ++en;
+          s_lid[loc] = lid;
         }
+        rn += __popc(nb);
+        rh += __popc(hb);
+        rm += __popc(mb);
       }
     }
-    __threadfence();
     __syncthreads();
-    if (threadIdx.x == 0) atomicExch(status + tile, pack_status(kFlagDone, s_inc));
-    // 4. edges (src lids) and block indptr
+    TRACE(hop, tile, 4);
+    // 4. edges (src lids, compacted, coalesced) and block indptr
     {
-      uint32_t ev = (uint32_t)run0;
-      uint32_t d = f0 / k, s = f0 - d * k;
+      uint32_t lid[kCompactItems];
+#pragma unroll
+      for (int i = 0; i < kCompactItems; ++i) {  // independent loads first
+        lid[i] = 0;
+        if ((vmask >> i) & 1u) {
+          const uint32_t fp = p[i] - base;  // first position as a flat index of this hop
+          if ((nmask >> i) & 1u) lid[i] = s_lid[loc0 + i * 32];
+          else if (p[i] < base) lid[i] = p[i];                   // relabelled earlier (lid)
+          else if (fp >= t0) lid[i] = s_lid[fp - t0];           // earlier in this tile
+          else lid[i] = u[i] | kDefer;                          // earlier tile: fixup
+        }
+      }
+      uint32_t rv = (uint32_t)ex;
 #pragma unroll
       for (int i = 0; i < kCompactItems; ++i) {
-        const uint32_t f = f0 + i;
-        if (f < flat && s == 0) bindptr[d] = ev;
-        if (flags & (1u << i)) {
-          uint32_t lid;
-          if ((flags >> (8 + i)) & 1u) {
-            lid = s_lid[l0 + i];
-          } else {
-            const uint32_t p = (uint32_t)e[i];  // first position of u in this batch
-            const uint32_t fp = p - base;       // ... as a flat index of this hop
-            if (p < base) {
-              lid = __ldcg(lidmap + u[i]);      // discovered by an earlier hop / a seed
-            } else if (fp >= t0) {
-              lid = s_lid[fp - t0];             // first seen earlier in this tile
-            } else {
-              const uint32_t tp = fp / kCompactTile;
-              while ((*((volatile unsigned long long*)(status + tp)) >> 62) != 3) {
-              }
-              __threadfence();
-              lid = __ldcg(lidmap + u[i]);
-            }
-          }
-          bindices[ev] = lid;
+        const uint32_t f = t0 + loc0 + i * 32;
+        const bool isv = (vmask >> i) & 1u;
+        const uint32_t vb = __ballot_sync(kFull, isv);
+        const uint32_t ev = rv + __popc(vb & lt);
+        if (f < flat && f % k == 0) bindptr[f / k] = ev;
+        if (isv) {
+          bindices[ev] = lid[i];
           if (W) bweights[ev] = pickw[f];
-          ++ev;
         }
-        if (++s == k) { s = 0; ++d; }
+        rv += __popc(vb);
       }
     }
     __syncthreads();
+    TRACE(hop, tile, 5);
   }
+}
+
+__global__ void __launch_bounds__(kThreads)
+    k_fixup(uint32_t hop, const DevState* __restrict__ st, const unsigned long long* vmap,
+            uint32_t* __restrict__ bindices) {
+  fixup_block(st->nnz[hop], vmap, bindices);
 }
 
 __global__ void k_validate(const uint64_t* __restrict__ indptr, const uint32_t* __restrict__ indices,
@@ -591,7 +645,7 @@ cudaError_t launch_seed_init(glb_ctx* c, const uint32_t* seeds, uint32_t n0, int
     za.n[l] = (uint32_t)c->sb.ntiles[l];
   }
   k_seed_init<<<blocks, kThreads, 0, c->stream>>>(seeds, n0, c->V, c->st, c->sb.uniq, c->vmap,
-                                                  c->lidmap, c->gen, mark_args(c, count_mode), za);
+                                                  c->gen, mark_args(c, count_mode), za);
   count_launch(c);
   return cudaGetLastError();
 }
@@ -600,12 +654,15 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
                         uint32_t batch) {
   const int grid = grid_for(c);
   const SampleBufs& b = c->sb;
+  uint32_t* fix = hop ? b.bindices[hop - 1] : nullptr;
   if (k <= 32)
     k_khop<<<grid, kThreads, 0, c->stream>>>(hop, k, seed, epoch, batch, c->gen, c->st, c->st,
-                                             c->indptr, c->indices, b.uniq, c->vmap, b.picks);
+                                             c->indptr, c->indices, b.uniq, c->vmap, b.picks,
+                                             fix);
   else
     k_khop_wide<<<grid, kThreads, 0, c->stream>>>(hop, k, seed, epoch, batch, c->gen, c->st, c->st,
-                                                  c->indptr, c->indices, b.uniq, c->vmap, b.picks);
+                                                  c->indptr, c->indices, b.uniq, c->vmap, b.picks,
+                                                  fix);
   count_launch(c);
   return cudaGetLastError();
 }
@@ -615,7 +672,8 @@ cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch
   const SampleBufs& b = c->sb;
 #define GLB_RW_ARGS                                                                          \
   hop, c->rw_walks, c->rw_len, c->rw_topk, seed, epoch, batch, c->gen, c->st, c->st, c->indptr, \
-      c->indices, b.uniq, c->vmap, b.picks, b.pickw
+      c->indices, b.uniq, c->vmap, b.picks, b.pickw, fix
+  uint32_t* fix = hop ? b.bindices[hop - 1] : nullptr;
   const uint32_t w = c->rw_walks;
   if (w <= 1) k_rwalk<1><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
   else if (w <= 2) k_rwalk<2><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
@@ -628,16 +686,22 @@ cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch
   return cudaGetLastError();
 }
 
+cudaError_t launch_fixup(glb_ctx* c, uint32_t hop) {
+  k_fixup<<<grid_for(c), kThreads, 0, c->stream>>>(hop, c->st, c->vmap, c->sb.bindices[hop]);
+  count_launch(c);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, int count_mode) {
   const SampleBufs& b = c->sb;
   const int grid = grid_for(c, 4);
   if (weighted)
     k_compact<true><<<grid, kThreads, 0, c->stream>>>(
-        hop, k, c->gen, c->st, b.picks, b.pickw, c->vmap, c->lidmap, b.uniq, b.bindptr[hop],
+        hop, k, c->gen, c->st, b.picks, b.pickw, c->vmap, b.uniq, b.bindptr[hop],
         b.bindices[hop], b.bweights[hop], b.status[hop], mark_args(c, count_mode));
   else
     k_compact<false><<<grid, kThreads, 0, c->stream>>>(
-        hop, k, c->gen, c->st, b.picks, nullptr, c->vmap, c->lidmap, b.uniq, b.bindptr[hop],
+        hop, k, c->gen, c->st, b.picks, nullptr, c->vmap, b.uniq, b.bindptr[hop],
         b.bindices[hop], nullptr, b.status[hop], mark_args(c, count_mode));
   count_launch(c);
   return cudaGetLastError();

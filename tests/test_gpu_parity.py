@@ -301,3 +301,32 @@ def test_pr_full_size_parity(pr):
         idx = rng.integers(0, s.sizes[-1], 4096)
         got = out[torch.from_numpy(idx).cuda()].cpu().numpy()
         assert np.array_equal(got.view(np.uint32), g.features[os_.uniq[idx]].view(np.uint32))
+
+
+@pytest.mark.parametrize("alpha", [1.0, 0.3])
+def test_pipeline_depth2_bit_exact(tiny, alpha):
+    """Pipelined Extract || Sample (two streams, double-buffered slots) gives the
+    same bytes as the oracle for every batch of an epoch."""
+    g, go = tiny
+    sh = g.shape
+    ctx = make_ctx(g, fanouts=sh.fanouts)
+    ctx.presample(1)
+    ctx.build_cache(alpha)
+    ctx.set_pipeline(2)
+    e = 1
+    ob = oracle.epoch_batches(g.train, sh.batch, g.seed, e)
+    outs, sizes = [], []
+    for b in range(len(ob)):
+        ctx.sample_batch(e, b)
+        outs.append(torch.full((64 * 11 * 6, g.D), float("nan"), device="cuda"))
+        ctx.extract_sample(outs[-1])
+    ctx.sync()
+    for b, seeds in enumerate(ob):
+        exp = go.sample_khop(seeds, sh.fanouts, g.seed, e, b)
+        n = exp.sizes[-1]
+        got = outs[b][:n].cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), go.extract(exp.uniq).view(np.uint32)), b
+        assert torch.isnan(outs[b][n:]).all()
+    # the current sample is still readable after the pipeline drained
+    assert_same_sample(ctx.sample_result(),
+                       go.sample_khop(ob[-1], sh.fanouts, g.seed, e, len(ob) - 1))
