@@ -48,6 +48,10 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
     p.add_argument("--measure-epochs", type=int, default=2)
+    p.add_argument("--mode", default="dp", choices=["dp", "factored"],
+                   help="factored: Ns sampler + Nt trainer ranks (PAPER.md §5.2-5.3)")
+    p.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
+                   help="gloo: CPU-staged send/recv (lets N ranks share one GPU for testing)")
     p.add_argument("--pipeline", type=int, default=1, choices=[1, 2],
                    help="2: extract of batch b overlaps sampling of batch b+1 (two streams)")
     return p.parse_args()
@@ -200,6 +204,102 @@ def cpu_baseline(g, sh, budget_s):
 
 
 # ------------------------------------------------------------------------------------------
+def run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_cache, par, glb):
+    """Factored mode (§5.2-5.3): profile Ts/Tt, split ranks into Ns samplers
+    and Nt trainers (Ns = ceil(N/(K+1)), K = Tt/Ts, L262), then samplers pull batches
+    from the global scheduler and hand samples to trainers, which extract."""
+    import torch
+    import torch.distributed as dist
+    cpu_comm = args.backend == "gloo"
+    comm_dev = "cpu" if cpu_comm else dev
+    # profile one sampler step and one trainer step (L260: "training an epoch in advance")
+    ts_l, tt_l = [], []
+    for i in range(max(args.warmup, 3)):
+        e, b = par.dp_step_batch(i, rank, world, nb, sh.K)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        ctx.sample_batch(e, b)
+        s = ctx.sample_result()
+        t1 = time.perf_counter()
+        ctx.extract(s.uniq, out=out[:s.sizes[-1]])
+        torch.cuda.synchronize()
+        ts_l.append(t1 - t0)
+        tt_l.append(time.perf_counter() - t1)
+    prof = torch.tensor([statistics.median(ts_l), statistics.median(tt_l)], dtype=torch.float64)
+    if world > 1:
+        prof = prof.to(comm_dev)
+        dist.all_reduce(prof)
+        prof = prof.cpu() / world
+    ns = par.num_samplers(world, float(prof[0]), float(prof[1]))
+    roles = par.Roles(ns, world)
+    total = args.steps * world
+    store = dist.distributed_c10d._get_default_store() if world > 1 else None
+    tag = "bench"
+    seeds = {"n": 0}
+
+    def sample_fn(gidx):
+        e, b = sh.K + gidx // nb, gidx % nb
+        ctx.sample_batch(e, b)
+        blk = ctx.sample_result()
+        return e, blk
+
+    def extract_fn(gidx, epoch, sizes, nnz, payload):
+        uniq = payload[0]
+        if uniq.device.type != "cuda":
+            uniq = uniq.to(dev, non_blocking=True)
+        ctx.extract(uniq.contiguous(), out=out[:sizes[-1]])
+        seeds["n"] += sizes[0]
+
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    if world == 1:
+        for gidx in range(total):
+            e, blk = sample_fn(gidx)
+            extract_fn(gidx, e, blk.sizes, blk.nnz, (blk.uniq,))
+    elif roles.is_sampler(rank):
+        if cpu_comm:
+            orig = sample_fn
+
+            def sample_fn(gidx):  # noqa: F811
+                e, blk = orig(gidx)
+                import types
+                return e, types.SimpleNamespace(
+                    sizes=blk.sizes, nnz=blk.nnz, uniq=blk.uniq.cpu(),
+                    indptr=[x.cpu() for x in blk.indptr], indices=[x.cpu() for x in blk.indices],
+                    weights=None if blk.weights is None else [x.cpu() for x in blk.weights])
+        par.run_sampler(sample_fn, roles, rank, total, store, tag, comm_dev)
+    else:
+        par.run_trainer(extract_fn, roles, rank, total, store, tag, comm_dev)
+    torch.cuda.synchronize()
+    el = time.perf_counter() - t0
+    red = torch.tensor([el, float(seeds["n"])], dtype=torch.float64)
+    if world > 1:
+        r2 = red.to(comm_dev)
+        t_max = r2[:1].clone()
+        dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
+        n_sum = r2[1:].clone()
+        dist.all_reduce(n_sum)
+        el, n_all = float(t_max.cpu()), float(n_sum.cpu())
+    else:
+        n_all = float(seeds["n"])
+    if rank == 0:
+        line = {"metric": METRIC, "value": n_all / el, "unit": "seeds/s", "n_gpus": world,
+                "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * el / args.steps,
+                "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+                "data": "synthetic",
+                "config": {"workload": workload_name(sh, args.alpha), "mode": "factored",
+                           "samplers": ns, "trainers": world - ns,
+                           "Ts_ms": 1e3 * float(prof[0]), "Tt_ms": 1e3 * float(prof[1]),
+                           "backend": args.backend, "parallelism": f"factored{ns}s{world - ns}t"},
+                "timing": "host wall clock around the sampler/trainer loops (max over ranks)",
+                "preprocess_s": {"presample": t_pre, "build_cache": t_cache}}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
 def main():
     args = parse()
     if args.impl == "reference":
@@ -208,11 +308,16 @@ def main():
     import torch.distributed as dist
 
     import paper_conf_eurosys_yangtswycyz22_b200 as glb
+    from paper_conf_eurosys_yangtswycyz22_b200 import parallel as par
 
     world, rank, local = dist_env()
+    local = local % torch.cuda.device_count()
     if world > 1:
         torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
     dev = torch.device("cuda", local)
     torch.cuda.set_device(dev)
     sh = synth.SHAPES[args.config]
@@ -246,7 +351,13 @@ def main():
     t0 = time.perf_counter()
     ctx.presample(sh.K, rank, world)
     if world > 1:
-        dist.all_reduce(ctx.counts_tensor(glb.COUNT_PRESAMPLE))  # u32 sums (< 2^31)
+        t_counts = ctx.counts_tensor(glb.COUNT_PRESAMPLE)
+        if args.backend == "nccl":
+            par.allreduce_counts(t_counts)  # u32 sums (< 2^31), NCCL over NVLink
+        else:
+            c = t_counts.cpu()
+            par.allreduce_counts(c)
+            t_counts.copy_(c)
     torch.cuda.synchronize()
     t_pre = time.perf_counter() - t0
     t0 = time.perf_counter()
@@ -260,14 +371,17 @@ def main():
     out = torch.empty((ub, sh.D), dtype=torch.float32, device=dev)
 
     def batch_of(i):
-        gidx = i * world + rank
-        return sh.K + gidx // nb, gidx % nb
+        return par.dp_step_batch(i, rank, world, nb, sh.K)
 
     def n_seeds(b):
         return min(sh.batch, sh.n_train - b * sh.batch)
 
+    if args.mode == "factored":
+        return run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_cache,
+                            par, glb)
+
     ctx.set_pipeline(args.pipeline)
-    xs = ctx.extract_stream()
+    xs = ctx.extract_stream() if args.pipeline == 2 else stream
 
     # ---- warmup
     for i in range(args.warmup):
@@ -289,6 +403,7 @@ def main():
     t_start = torch.cuda.Event(enable_timing=True)
     t_end = torch.cuda.Event(enable_timing=True)
     t_start.record(stream)
+    wall0 = time.perf_counter()
     seeds_done = 0
     for i in steps:
         e, b = batch_of(i)
@@ -296,7 +411,9 @@ def main():
         ctx.extract_sample(out)
         seeds_done += n_seeds(b)
     t_end.record(xs)
+    enqueue_ms = 1e3 * (time.perf_counter() - wall0)
     torch.cuda.synchronize()
+    wall_ms = 1e3 * (time.perf_counter() - wall0)
     barrier()
     clk = clocks.stop()
     launches = ctx.launches - launches0
@@ -306,6 +423,8 @@ def main():
     el = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
     tot = torch.tensor([float(seeds_done)], dtype=torch.float64, device=dev)
     if world > 1:
+        if args.backend == "gloo":
+            el, tot = el.cpu(), tot.cpu()
         dist.all_reduce(el, op=dist.ReduceOp.MAX)
         dist.all_reduce(tot)
     elapsed_max = float(el.item())
@@ -359,6 +478,8 @@ def main():
     e2e_t = torch.tensor([time.perf_counter() - t0], dtype=torch.float64, device=dev)
     e2e_n = torch.tensor([float(e2e_seeds)], dtype=torch.float64, device=dev)
     if world > 1:
+        if args.backend == "gloo":
+            e2e_t, e2e_n = e2e_t.cpu(), e2e_n.cpu()
         dist.all_reduce(e2e_t, op=dist.ReduceOp.MAX)
         dist.all_reduce(e2e_n)
     e2e_val = float(e2e_n.item()) / float(e2e_t.item())
@@ -377,7 +498,11 @@ def main():
         ctx.set_count_mode(glb.COUNT_NONE)
         ctx.sync()
         if world > 1:
-            dist.all_reduce(ctx.counts_tensor(glb.COUNT_ACCESS))
+            t_acc = ctx.counts_tensor(glb.COUNT_ACCESS)
+            c = t_acc if args.backend == "nccl" else t_acc.cpu()
+            par.allreduce_counts(c)
+            if c is not t_acc:
+                t_acc.copy_(c)
         for a in sorted(set(sh.alphas) | {args.alpha}):
             ctx.build_cache(a)
             hs = ctx.hit_stats()
@@ -421,6 +546,8 @@ def main():
                        "l2": "inputs larger than L2 (CSR %.2f GB, feature cache %.2f GB vs 126 MB L2)"
                              % ((8 * (sh.V + 1) + 4 * sh.E) / 1e9, 4 * sh.D * sh.V * args.alpha / 1e9)},
             "pipeline_depth": args.pipeline,
+            "host_wall_ms_timed_region": wall_ms,
+            "host_enqueue_ms_timed_region": enqueue_ms,
             "roofline": {"kernel": "k_gather (extract a7)", "bound": "hbm", "achieved": ach_gbs,
                          "peak": peak, "unit": "GB/s", "frac": ach_gbs / peak, "traffic": traffic,
                          "peak_source": peak_src,

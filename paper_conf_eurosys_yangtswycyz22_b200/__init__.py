@@ -373,7 +373,9 @@ class Context:
         import torch
         p = ctypes.c_void_p()
         self._ck(self._lib.glb_extract_stream(self._h, ctypes.byref(p)))
-        return torch.cuda.ExternalStream(p.value or 0, device=self.device)
+        if not p.value:  # the legacy default stream
+            return torch.cuda.default_stream(self.device)
+        return torch.cuda.ExternalStream(p.value, device=self.device)
 
     def set_timing(self, enable: bool):
         self._ck(self._lib.glb_set_timing(self._h, int(enable)))

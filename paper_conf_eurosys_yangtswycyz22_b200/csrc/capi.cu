@@ -125,7 +125,7 @@ glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, in
   for (uint32_t l = 0; l < L; ++l)
     if (k[l] > c->sb.k[l]) return set_err(c, GLB_ENOMEM, "fanout %u > configured %u at hop %u", k[l], c->sb.k[l], l);
   if (c->gen >= 0xFFFFFFF0u) {  // generation wrap: clear the relabel table once
-    CK(cudaMemsetAsync(c->vmap, 0xFF, sizeof(unsigned long long) * c->V, c->stream));
+    CK(launch_vmap_reset(c));
     c->gen = 0;
   }
   c->gen += 1;
@@ -267,8 +267,8 @@ glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* in
   CK(dalloc(&c->access, V));
   CK(cudaMemcpy(c->indptr, indptr, sizeof(uint64_t) * (V + 1), cudaMemcpyHostToDevice));
   if (E) CK(cudaMemcpy(c->indices, indices, sizeof(uint32_t) * E, cudaMemcpyHostToDevice));
-  CK(cudaMemsetAsync(c->vmap, 0xFF, sizeof(unsigned long long) * V, c->stream));
   CK(cudaMemsetAsync(c->slot, 0xFF, sizeof(int32_t) * V, c->stream));
+  CK(launch_vmap_reset(c));
   CK(cudaMemsetAsync(c->counts, 0, sizeof(uint32_t) * V, c->stream));
   CK(cudaMemsetAsync(c->access, 0, sizeof(uint32_t) * V, c->stream));
   CK(cudaMemsetAsync(c->st, 0, sizeof(DevState), c->stream));
@@ -564,6 +564,8 @@ glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
   CK(radix_sort_pairs_u32(c, k0, v0, k1, v1, V, bits, &ko, &order));
   CK(cudaMemsetAsync(c->slot, 0xFF, sizeof(int32_t) * V, c->stream));
   CK(launch_assign_slots(c, order, C));
+  CK(launch_vmap_reset(c));  // copy the slots into the relabel entries (and clear them)
+  c->gen = 0;
   dfree(c->cache);
   c->C = C;
   if (c->features_mapped && C) {

@@ -69,6 +69,15 @@ __device__ __forceinline__ uint64_t enc_pos(uint32_t gen, uint32_t pos) {
   return ((uint64_t)(0xFFFFFFFFu - gen) << 32) | pos;
 }
 
+// Relabel-table entry (one per vertex): gp = ((0xFFFFFFFF - gen) << 32) | first
+// position, then | lid once relabelled; slot = the vertex's cache slot (-1 = not
+// cached), co-located so one 16-byte load gives both (a4 mark needs no extra access).
+struct __align__(16) VEntry {
+  unsigned long long gp;
+  int32_t slot;
+  uint32_t pad;
+};
+
 struct SampleBufs {
   uint32_t cap_batch = 0;
   uint32_t L = 0;
@@ -115,7 +124,7 @@ struct glb_ctx {
   uint32_t D = 0;
 
   // relabel tables (D6): direct-address over gids
-  unsigned long long* vmap = nullptr;  // u64[V]: (gen, first position) then (gen, lid)
+  glb::VEntry* vmap = nullptr;  // [V]: (gen, first position) then (gen, lid); cache slot
   uint32_t gen = 0;
 
   // cache (D3, D4, D5)
@@ -208,6 +217,7 @@ cudaError_t launch_max_u32(glb_ctx* c, const uint32_t* a, uint64_t n, uint32_t* 
 cudaError_t launch_rank_keys(glb_ctx* c, const uint32_t* hot, uint32_t maxc, uint32_t* keys,
                              uint32_t* vals);
 cudaError_t launch_assign_slots(glb_ctx* c, const uint32_t* order, uint64_t C);
+cudaError_t launch_vmap_reset(glb_ctx* c);   // gp = ~0, slot = c->slot[v]
 cudaError_t launch_hit_stats(glb_ctx* c, unsigned long long* out3 /* total,hits,max */);
 cudaError_t launch_value_hist(glb_ctx* c, const uint32_t* a, uint64_t n, unsigned long long* bins,
                               uint32_t nbins);

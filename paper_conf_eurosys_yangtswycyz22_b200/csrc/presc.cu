@@ -238,6 +238,18 @@ __global__ void k_assign_slots(const uint32_t* __restrict__ order, uint64_t C, i
     slot[order[i]] = (int32_t)i;
 }
 
+__global__ void k_vmap_reset(VEntry* __restrict__ vmap, const int32_t* __restrict__ slot,
+                             uint64_t n) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    VEntry e;
+    e.gp = ~0ull;
+    e.slot = slot[i];
+    e.pad = 0;
+    vmap[i] = e;
+  }
+}
+
 __global__ void k_hit_stats(const uint32_t* __restrict__ acc, const int32_t* __restrict__ slot,
                             uint64_t n, unsigned long long* out3) {
   unsigned long long tot = 0, hit = 0;
@@ -372,6 +384,12 @@ cudaError_t launch_rank_keys(glb_ctx* c, const uint32_t* hot, uint32_t maxc, uin
 cudaError_t launch_assign_slots(glb_ctx* c, const uint32_t* order, uint64_t C) {
   if (C == 0) return cudaSuccess;
   k_assign_slots<<<grid_for(c), kThreads, 0, c->stream>>>(order, C, c->slot);
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_vmap_reset(glb_ctx* c) {
+  k_vmap_reset<<<grid_for(c), kThreads, 0, c->stream>>>(c->vmap, c->slot, c->V);
   count_launch(c);
   return cudaGetLastError();
 }

@@ -30,9 +30,7 @@ extern "C" glb_status glb_trace_dump(void* host, size_t bytes) {
   return cudaMemcpyFromSymbol(host, g_trace, bytes) == cudaSuccess ? GLB_OK : GLB_ECUDA;
 }
 __device__ __forceinline__ unsigned long long gtime() {
-  unsigned long long t;
-  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-  return t;
+  return (unsigned long long)clock64();  // SM cycles (relative deltas within a tile)
 }
 #define TRACE(h, t, ev) \
   do { if (threadIdx.x == 0 && (t) < 4096) ::g_trace[h][t][ev] = gtime(); } while (0)
@@ -55,20 +53,31 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 // Insert one pick into the relabel table: keep the smallest position of this
 // generation.  Values only decrease over time, so a (possibly stale) read that
 // is already <= e proves the atomic would be a no-op.
-__device__ __forceinline__ void vmap_insert(unsigned long long* vmap, uint32_t u,
-                                            unsigned long long e) {
-  const unsigned long long old = __ldcg(vmap + u);
-  if (old > e) atomicMin(vmap + u, e);
+__device__ __forceinline__ unsigned long long vmap_insert(VEntry* vmap, uint32_t u,
+                                                          unsigned long long e) {
+  unsigned long long old = __ldcg(&vmap[u].gp);
+  if (old > e) old = atomicMin(&vmap[u].gp, e);
+  return old;  // <= e: an earlier position (or a lid) of this generation holds u
+}
+
+// Encoded pick: the gid, or -- when the sampler already found u relabelled by an
+// earlier hop / as a seed (table value (gen, lid) with lid < base) -- lid | kOld,
+// so the compaction needs no table access for it.  gids and lids are < 2^31.
+constexpr uint32_t kOld = 0x80000000u;
+__device__ __forceinline__ uint32_t encode_pick(uint32_t u, unsigned long long old,
+                                                unsigned long long e, uint32_t base) {
+  if (old <= e && (uint32_t)old < base) return (uint32_t)old | kOld;
+  return u;
 }
 
 constexpr uint32_t kDefer = 0x80000000u;  // deferred src lid marker (gids < 2^31, glb_load_graph)
 
 // Resolve deferred src lids of block `hop` (entries gid | kDefer).
-__device__ __forceinline__ void fixup_block(uint32_t nnz, const unsigned long long* vmap,
+__device__ __forceinline__ void fixup_block(uint32_t nnz, const VEntry* vmap,
                                             uint32_t* __restrict__ bindices) {
   for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x) {
     const uint32_t x = bindices[e];
-    if (x & kDefer) bindices[e] = (uint32_t)__ldcg(vmap + (x & ~kDefer));  // (gen, lid)
+    if (x & kDefer) bindices[e] = (uint32_t)__ldcg(&vmap[x & ~kDefer].gp);  // (gen, lid)
   }
 }
 
@@ -89,7 +98,7 @@ struct StatusArgs {  // look-back status arrays to clear for this batch
 // ---------------------------------------------------------------- seeds
 __global__ void __launch_bounds__(kThreads)
     k_seed_init(const uint32_t* __restrict__ seeds, uint32_t n0, uint64_t V, DevState* st,
-                uint32_t* __restrict__ uniq, unsigned long long* vmap, uint32_t gen, MarkArgs mk,
+                uint32_t* __restrict__ uniq, VEntry* vmap, uint32_t gen, MarkArgs mk,
                 StatusArgs za) {
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     st->n[0] = n0;
@@ -112,7 +121,7 @@ __global__ void __launch_bounds__(kThreads)
         u = 0;  // keep later kernels in bounds; the batch is reported invalid
       }
       uniq[i] = u;
-      atomicMin(vmap + u, enc_pos(gen, i));  // a seed's position is its lid
+      atomicMin(&vmap[u].gp, enc_pos(gen, i));  // a seed's position is its lid
       s = __ldg(mk.slot + u);
       mk.lidslot[i] = s;
       if (mk.count) atomicAdd(mk.count + u, 1u);
@@ -138,7 +147,7 @@ __global__ void __launch_bounds__(kThreads)
     k_khop(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch, uint32_t gen,
            const DevState* __restrict__ st, DevState* st_w, const uint64_t* __restrict__ indptr,
            const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
-           unsigned long long* vmap, uint32_t* __restrict__ picks, uint32_t* fix_ind) {
+           VEntry* vmap, uint32_t* __restrict__ picks, uint32_t* fix_ind) {
   if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);  // deferred lids of block hop-1
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
@@ -159,7 +168,7 @@ __global__ void __launch_bounds__(kThreads)
       v = uniq[d];
       lo = indptr[v];
       deg = (uint32_t)(indptr[v + 1] - lo);
-      if (hop == 0 && s == 0 && __ldcg(vmap + v) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
+      if (hop == 0 && s == 0 && __ldcg(&vmap[v].gp) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
     }
     const bool big = active && deg > k;
     uint32_t t = 0, j = 0;
@@ -191,7 +200,8 @@ __global__ void __launch_bounds__(kThreads)
     uint32_t u = kEmpty;
     if (sel != kEmpty) {
       u = __ldg(indices + lo + sel);
-      vmap_insert(vmap, u, enc_pos(gen, base + d * k + s));
+      const unsigned long long e = enc_pos(gen, base + d * k + s);
+      u = encode_pick(u, vmap_insert(vmap, u, e), e, base);
     }
     if (active) picks[(size_t)d * k + s] = u;
   }
@@ -202,7 +212,7 @@ __global__ void __launch_bounds__(kThreads)
     k_khop_wide(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch,
                 uint32_t gen, const DevState* __restrict__ st, DevState* st_w,
                 const uint64_t* __restrict__ indptr, const uint32_t* __restrict__ indices,
-                const uint32_t* __restrict__ uniq, unsigned long long* vmap,
+                const uint32_t* __restrict__ uniq, VEntry* vmap,
                 uint32_t* __restrict__ picks, uint32_t* fix_ind) {
   __shared__ uint32_t chosen[kThreads / 32][kMaxFanout];
   if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);
@@ -217,7 +227,7 @@ __global__ void __launch_bounds__(kThreads)
     const uint32_t v = uniq[d];
     const uint64_t lo = indptr[v];
     const uint32_t deg = (uint32_t)(indptr[v + 1] - lo);
-    if (hop == 0 && lane == 0 && __ldcg(vmap + v) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
+    if (hop == 0 && lane == 0 && __ldcg(&vmap[v].gp) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
     if (deg > k) {
       if (lane == 0) {
         for (uint32_t s = 0; s < k; ++s) {
@@ -234,9 +244,12 @@ __global__ void __launch_bounds__(kThreads)
       uint32_t sel = kEmpty;
       if (deg > k) sel = ch[s];
       else if (s < deg) sel = s;
-      const uint32_t u = sel != kEmpty ? __ldg(indices + lo + sel) : kEmpty;
+      uint32_t u = sel != kEmpty ? __ldg(indices + lo + sel) : kEmpty;
+      if (u != kEmpty) {
+        const unsigned long long e = enc_pos(gen, base + d * k + s);
+        u = encode_pick(u, vmap_insert(vmap, u, e), e, base);
+      }
       picks[(size_t)d * k + s] = u;
-      if (u != kEmpty) vmap_insert(vmap, u, enc_pos(gen, base + d * k + s));
     }
     __syncwarp();
   }
@@ -250,7 +263,7 @@ __global__ void __launch_bounds__(kThreads)
             uint32_t epoch, uint32_t batch, uint32_t gen, const DevState* __restrict__ st,
             DevState* st_w, const uint64_t* __restrict__ indptr,
             const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
-            unsigned long long* vmap, uint32_t* __restrict__ picks, uint32_t* __restrict__ pickw,
+            VEntry* vmap, uint32_t* __restrict__ picks, uint32_t* __restrict__ pickw,
             uint32_t* fix_ind) {
   if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);
   const uint32_t n_l = st->n[hop];
@@ -271,7 +284,7 @@ __global__ void __launch_bounds__(kThreads)
     for (int t = 0; t < kMaxWalkLen; ++t) vis[t] = kEmpty;
     if (active) {
       v = uniq[d];
-      if (hop == 0 && w == 0 && __ldcg(vmap + v) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
+      if (hop == 0 && w == 0 && __ldcg(&vmap[v].gp) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
       if (w < walks) {
         uint32_t cur = v;
 #pragma unroll
@@ -332,9 +345,9 @@ __global__ void __launch_bounds__(kThreads)
       for (int t = 0; t < kMaxWalkLen; ++t) {
         if (vis[t] != kEmpty && first[t] && rank[t] < topk) {
           const uint32_t f = d * topk + rank[t];
-          picks[f] = vis[t];
+          const unsigned long long e = enc_pos(gen, base + f);
+          picks[f] = encode_pick(vis[t], vmap_insert(vmap, vis[t], e), e, base);
           pickw[f] = cnt[t];
-          vmap_insert(vmap, vis[t], enc_pos(gen, base + f));
         }
       }
     }
@@ -395,10 +408,10 @@ __device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
 constexpr int kWarpSpan = kCompactTile / (kThreads / 32);  // positions per warp
 
 template <bool W>
-__global__ void __launch_bounds__(kThreads, 4)
+__global__ void __launch_bounds__(kThreads, 3)
     k_compact(uint32_t hop, uint32_t k, uint32_t gen, DevState* st,
               const uint32_t* __restrict__ picks, const uint32_t* __restrict__ pickw,
-              unsigned long long* vmap,
+              VEntry* vmap,
               uint32_t* __restrict__ uniq, uint32_t* __restrict__ bindptr,
               uint32_t* __restrict__ bindices, uint32_t* __restrict__ bweights,
               unsigned long long* status, MarkArgs mk) {
@@ -447,17 +460,19 @@ __global__ void __launch_bounds__(kThreads, 4)
       p[i] = 0;
       if (u[i] != kEmpty) {
         vmask |= 1u << i;
-        const unsigned long long e = __ldcg(vmap + u[i]);  // position, or lid (< base) once relabelled
-        p[i] = (uint32_t)e;
-        if (e == enc_pos(gen, base + t0 + loc0 + i * 32)) nmask |= 1u << i;
-      }
-    }
-#pragma unroll
-    for (int i = 0; i < kCompactItems; ++i) {
-      if ((nmask >> i) & 1u) {
-        const int32_t sl = __ldg(mk.slot + u[i]);
-        s_slot[loc0 + i * 32] = sl;
-        if (sl >= 0) hmask |= 1u << i;
+        if (u[i] & kOld) {
+          p[i] = u[i] & ~kOld;  // the sampler resolved it: a lid < base
+        } else {
+          // one 16-byte load: (gen, position-or-lid) and the cache slot
+          const ulonglong2 ent = __ldcg(reinterpret_cast<const ulonglong2*>(vmap + u[i]));
+          p[i] = (uint32_t)ent.x;
+          if (ent.x == enc_pos(gen, base + t0 + loc0 + i * 32)) {
+            nmask |= 1u << i;
+            const int32_t sl = (int32_t)(uint32_t)ent.y;
+            s_slot[loc0 + i * 32] = sl;
+            if (sl >= 0) hmask |= 1u << i;
+          }
+        }
       }
     }
     TRACE(hop, tile, 1);
@@ -547,7 +562,7 @@ __global__ void __launch_bounds__(kThreads, 4)
           const uint32_t lid = n_l + rn + __popc(nb & lt);
           const int32_t sl = s_slot[loc];
           uniq[lid] = u[i];
-          __stcg(vmap + u[i], enc_pos(gen, lid));  // relabelled: later readers get the lid
+          __stcg(&vmap[u[i]].gp, enc_pos(gen, lid));  // relabelled: later readers get the lid
           mk.lidslot[lid] = sl;
           if (ish) mk.hit_list[rh + __popc(hb & lt)] = make_uint2(lid, (uint32_t)sl);
           else mk.miss_list[rm + __popc(mb & lt)] = make_uint2(lid, u[i]);
@@ -596,7 +611,7 @@ __global__ void __launch_bounds__(kThreads, 4)
 }
 
 __global__ void __launch_bounds__(kThreads)
-    k_fixup(uint32_t hop, const DevState* __restrict__ st, const unsigned long long* vmap,
+    k_fixup(uint32_t hop, const DevState* __restrict__ st, const VEntry* vmap,
             uint32_t* __restrict__ bindices) {
   fixup_block(st->nnz[hop], vmap, bindices);
 }
@@ -694,7 +709,7 @@ cudaError_t launch_fixup(glb_ctx* c, uint32_t hop) {
 
 cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, int count_mode) {
   const SampleBufs& b = c->sb;
-  const int grid = grid_for(c, 4);
+  const int grid = grid_for(c, 3);
   if (weighted)
     k_compact<true><<<grid, kThreads, 0, c->stream>>>(
         hop, k, c->gen, c->st, b.picks, b.pickw, c->vmap, b.uniq, b.bindptr[hop],

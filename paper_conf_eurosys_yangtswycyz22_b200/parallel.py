@@ -1,0 +1,191 @@
+"""Multi-GPU orchestration of the sample+extract path (one process per GPU).
+
+Two modes, both over ``torch.distributed`` (NCCL on GPUs, gloo in CPU tests):
+
+* **DP** (default): mini-batch g of an epoch goes to rank
+  g mod N (static) -- every draw is keyed by (epoch, batch), so per-batch
+  outputs are identical on any rank.  The only collective is the sum
+  all-reduce of the u32 PreSC counts (and of measured-epoch access counts for
+  the hit-rate metric): integer sums, bit-identical at every N.
+
+* **Factored** (§5.2-5.3): Ns sampler ranks and
+  Nt = N - Ns trainer ranks.  Ns = ceil(N / (K + 1)) with K = Tt / Ts from a
+  profiled warm-up (L262-L263; Tt is the trainer's per-batch time, which on
+  this path is Extract, L438).  A global scheduler hands batches to samplers
+  dynamically without synchronisation (L250): a host-side atomic counter in
+  the process group's store.  Batch g is extracted by trainer g mod Nt; the
+  sampler that produced it publishes (g -> sampler rank) in the store (the
+  "global queue" descriptor, L217) and sends a fixed-size header and one
+  flat payload (uniq gids, block CSRs) with point-to-point send/recv.
+
+The sampler/trainer roles talk to a ``ctx`` through a narrow interface so
+CPU tests can drive the protocol with a stand-in sampler (tests/test_parallel.py).
+"""
+from __future__ import annotations
+
+import dataclasses
+import math
+
+import torch
+import torch.distributed as dist
+
+HEADER_WORDS = 32  # int64: [batch, epoch, L, n_0..n_L, nnz_0..nnz_{L-1}, weighted, ...]
+
+
+# ----------------------------------------------------------------------------- DP
+def dp_batches(num_batches: int, rank: int, world: int):
+    """Batches of one epoch owned by ``rank`` (round-robin, L252 data parallelism)."""
+    return list(range(rank, num_batches, world))
+
+
+def dp_step_batch(i: int, rank: int, world: int, num_batches: int, first_epoch: int):
+    """(epoch, batch) of this rank's i-th step when epochs are consumed in order."""
+    g = i * world + rank
+    return first_epoch + g // num_batches, g % num_batches
+
+
+def allreduce_counts(t: torch.Tensor, group=None):
+    """Sum u32 visit counts across ranks (int32 view; sums stay < 2^31)."""
+    if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+    return t
+
+
+def presample_dp(ctx, K: int, rank: int, world: int, group=None):
+    """PreSC#K sharded by batch, then the count all-reduce."""
+    ctx.presample(K, rank, world)
+    allreduce_counts(ctx.counts_tensor(1), group)
+
+
+# ----------------------------------------------------------------------------- factored
+def num_samplers(n_gpus: int, t_sample: float, t_train: float) -> int:
+    """Ns = ceil(Ng / (K + 1)), K = Tt / Ts; at least one of each
+    role when n_gpus >= 2."""
+    if n_gpus <= 1:
+        return n_gpus
+    K = t_train / max(t_sample, 1e-12)
+    ns = math.ceil(n_gpus / (K + 1.0))
+    return min(max(ns, 1), n_gpus - 1)
+
+
+@dataclasses.dataclass
+class Roles:
+    n_samplers: int
+    world: int
+
+    @property
+    def n_trainers(self):
+        return self.world - self.n_samplers
+
+    def is_sampler(self, rank):
+        return rank < self.n_samplers
+
+    def trainer_rank(self, g: int) -> int:
+        """Trainer (global rank) that extracts batch g."""
+        return self.n_samplers + g % self.n_trainers
+
+    def trainer_batches(self, rank: int, total: int):
+        t = rank - self.n_samplers
+        return list(range(t, total, self.n_trainers))
+
+
+def pack_header(g: int, epoch: int, sizes, nnz, weighted: bool, device) -> torch.Tensor:
+    h = torch.zeros(HEADER_WORDS, dtype=torch.int64)
+    L = len(nnz)
+    assert 4 + 2 * L + 1 <= HEADER_WORDS
+    h[0], h[1], h[2], h[3] = g, epoch, L, int(weighted)
+    h[4:5 + L] = torch.tensor(sizes, dtype=torch.int64)
+    h[5 + L:5 + 2 * L] = torch.tensor(nnz, dtype=torch.int64)
+    return h.to(device)
+
+
+def unpack_header(h: torch.Tensor):
+    h = h.cpu().tolist()
+    g, epoch, L, weighted = h[0], h[1], h[2], bool(h[3])
+    sizes = h[4:5 + L]
+    nnz = h[5 + L:5 + 2 * L]
+    return g, epoch, sizes, nnz, weighted
+
+
+def payload_len(sizes, nnz, weighted) -> int:
+    L = len(nnz)
+    n = sizes[-1] + sum(sizes[l] + 1 for l in range(L)) + sum(nnz)
+    return n + (sum(nnz) if weighted else 0)
+
+
+def pack_payload(blocks) -> torch.Tensor:
+    """uniq | indptr_0..L-1 | indices_0..L-1 | (weights_0..L-1), int32, contiguous."""
+    parts = [blocks.uniq] + list(blocks.indptr) + list(blocks.indices)
+    if blocks.weights is not None:
+        parts += list(blocks.weights)
+    return torch.cat([p.reshape(-1).to(torch.int32) for p in parts])
+
+
+def unpack_payload(buf: torch.Tensor, sizes, nnz, weighted):
+    L = len(nnz)
+    o = 0
+    uniq = buf[o:o + sizes[-1]]
+    o += sizes[-1]
+    indptr = []
+    for l in range(L):
+        indptr.append(buf[o:o + sizes[l] + 1])
+        o += sizes[l] + 1
+    indices = []
+    for l in range(L):
+        indices.append(buf[o:o + nnz[l]])
+        o += nnz[l]
+    weights = None
+    if weighted:
+        weights = []
+        for l in range(L):
+            weights.append(buf[o:o + nnz[l]])
+            o += nnz[l]
+    return uniq, indptr, indices, weights
+
+
+class GlobalScheduler:
+    """Dynamic batch assignment to samplers without synchronisation (L250): an atomic
+    counter in the process group's key-value store."""
+
+    def __init__(self, store, key: str):
+        self.store = store
+        self.key = key
+
+    def next(self) -> int:
+        return int(self.store.add(self.key, 1)) - 1
+
+
+def run_sampler(sample_fn, roles: Roles, rank: int, total: int, store, tag: str, device):
+    """Sampler executor (Fig 9): pull batch ids, sample, publish the
+    descriptor, send header + payload to the batch's trainer.  Returns #batches."""
+    sched = GlobalScheduler(store, f"{tag}/next")
+    done = 0
+    while True:
+        g = sched.next()
+        if g >= total:
+            break
+        epoch, blocks = sample_fn(g)
+        weighted = blocks.weights is not None
+        store.set(f"{tag}/src/{g}", str(rank))
+        dst = roles.trainer_rank(g)
+        dist.send(pack_header(g, epoch, blocks.sizes, blocks.nnz, weighted, device), dst)
+        dist.send(pack_payload(blocks).to(device), dst)
+        done += 1
+    return done
+
+
+def run_trainer(extract_fn, roles: Roles, rank: int, total: int, store, tag: str, device):
+    """Trainer executor (Fig 9): for each batch it owns, find the sampler
+    through the global queue, receive the samples, extract.  Returns #batches."""
+    n = 0
+    for g in roles.trainer_batches(rank, total):
+        src = int(store.get(f"{tag}/src/{g}"))  # blocks until the descriptor exists
+        h = torch.empty(HEADER_WORDS, dtype=torch.int64, device=device)
+        dist.recv(h, src)
+        g2, epoch, sizes, nnz, weighted = unpack_header(h)
+        assert g2 == g, (g2, g)
+        buf = torch.empty(payload_len(sizes, nnz, weighted), dtype=torch.int32, device=device)
+        dist.recv(buf, src)
+        extract_fn(g, epoch, sizes, nnz, unpack_payload(buf, sizes, nnz, weighted))
+        n += 1
+    return n

@@ -1,0 +1,78 @@
+"""N>1 paths on the real GPU: two ranks sharing cuda:0 over gloo (NCCL needs one
+GPU per rank; gpurun gives one).  DP: sharded PreSC + count all-reduce equals
+the oracle's full counts bit for bit.  bench.py runs end to end under torchrun
+in DP and factored modes."""
+import json
+import os
+import socket
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _dp_worker(rank, world, port, out):
+    import torch.distributed as dist
+
+    import paper_conf_eurosys_yangtswycyz22_b200 as glb
+    import synth
+    from paper_conf_eurosys_yangtswycyz22_b200 import parallel as par
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    g = synth.make_graph("tiny")
+    sh = g.shape
+    ctx = glb.Context(0)
+    ctx.load_graph(g.indptr, g.indices, g.features)
+    ctx.set_sampler("khop", fanouts=sh.fanouts, max_batch=sh.batch)
+    ctx.set_train_set(g.train, sh.batch, g.seed)
+    ctx.presample(2, rank, world)
+    c = ctx.counts_tensor(glb.COUNT_PRESAMPLE).cpu()
+    par.allreduce_counts(c)
+    if rank == 0:
+        np.save(out, c.numpy())
+    dist.destroy_process_group()
+
+
+def test_dp_presample_two_ranks_equals_oracle(tmp_path):
+    import torch.multiprocessing as mp
+
+    import oracle
+    import synth
+    out = str(tmp_path / "c.npy")
+    mp.spawn(_dp_worker, args=(2, free_port(), out), nprocs=2, join=True)
+    g = synth.make_graph("tiny")
+    sh = g.shape
+    full = oracle.GraphOracle(g.indptr, g.indices).presample("khop", g.train, sh.batch,
+                                                            sh.fanouts, g.seed, 2)
+    assert np.array_equal(np.load(out).view(np.uint32), full)
+
+
+@pytest.mark.parametrize("mode", ["dp", "factored"])
+def test_bench_two_ranks(mode):
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()), "bench.py",
+           "--gpus", "2", "--steps", "16", "--warmup", "3", "--config", "tiny",
+           "--backend", "gloo", "--mode", mode, "--no-sweep", "--no-cpu-baseline"]
+    r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0
+    if mode == "factored":
+        assert d["config"]["samplers"] + d["config"]["trainers"] == 2

@@ -1,0 +1,154 @@
+"""Multi-process (gloo, CPU) tests of the N>1 orchestration in
+paper_conf_eurosys_yangtswycyz22_b200.parallel: DP sharding + count
+all-reduce, the factored sampler->trainer protocol (global scheduler,
+global-queue descriptors, header/payload send/recv), and the Ns formula.
+The GPU sampler is replaced by the CPU oracle as a stand-in (tests only)."""
+import os
+import socket
+import types
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_eurosys_yangtswycyz22_b200 import parallel as par
+
+
+def free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _init(rank, world, port):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+
+
+def test_num_samplers_formula():
+    # Ns = ceil(Ng / (K+1)), K = Tt/Ts
+    assert par.num_samplers(8, 1.0, 3.0) == 2
+    assert par.num_samplers(8, 1.0, 1.0) == 4
+    assert par.num_samplers(8, 2.0, 1.0) == 6
+    assert par.num_samplers(8, 1.0, 0.0) == 7      # at least one trainer
+    assert par.num_samplers(8, 1.0, 100.0) == 1    # at least one sampler
+    assert par.num_samplers(1, 1.0, 1.0) == 1
+
+
+def test_dp_sharding_covers_every_batch_once():
+    for world in [1, 2, 3, 8]:
+        nb = 25
+        seen = sorted(b for r in range(world) for b in par.dp_batches(nb, r, world))
+        assert seen == list(range(nb))
+        steps = sorted(par.dp_step_batch(i, r, world, nb, 1) for r in range(world)
+                       for i in range(10))
+        assert len(set(steps)) == 10 * world
+        assert steps[0] == (1, 0)
+
+
+def _dp_worker(rank, world, port, out):
+    import oracle
+    import synth
+    _init(rank, world, port)
+    g = synth.make_graph("tiny")
+    sh = g.shape
+    go = oracle.GraphOracle(g.indptr, g.indices)
+    nb = -(-sh.n_train // sh.batch)
+    mine = set(par.dp_batches(nb, rank, world))
+    c = go.visit_counts("khop", g.train, sh.batch, sh.fanouts, g.seed, range(2),
+                        batch_filter=lambda e, b: b in mine)
+    t = torch.from_numpy(c.view(np.int32).copy())
+    par.allreduce_counts(t)
+    if rank == 0:
+        np.save(out, t.numpy())
+    dist.destroy_process_group()
+
+
+def test_dp_presample_allreduce_equals_single_process(tmp_path):
+    import oracle
+    import synth
+    out = str(tmp_path / "c.npy")
+    world = 2
+    mp.spawn(_dp_worker, args=(world, free_port(), out), nprocs=world, join=True)
+    g = synth.make_graph("tiny")
+    sh = g.shape
+    go = oracle.GraphOracle(g.indptr, g.indices)
+    full = go.presample("khop", g.train, sh.batch, sh.fanouts, g.seed, 2)
+    assert np.array_equal(np.load(out).view(np.uint32), full)
+
+
+def _factored_worker(rank, world, port, ns, outdir):
+    import oracle
+    import synth
+    _init(rank, world, port)
+    g = synth.make_graph("tiny")
+    sh = g.shape
+    go = oracle.GraphOracle(g.indptr, g.indices, g.features)
+    roles = par.Roles(ns, world)
+    batches = oracle.epoch_batches(g.train, sh.batch, g.seed, 1)
+    total = len(batches)
+    store = dist.distributed_c10d._get_default_store()
+    if roles.is_sampler(rank):
+        def sample_fn(gidx):
+            s = go.sample_khop(batches[gidx], sh.fanouts, g.seed, 1, gidx)
+            t = lambda a: torch.from_numpy(np.ascontiguousarray(a).view(np.int32))  # noqa: E731
+            return 1, types.SimpleNamespace(
+                sizes=s.sizes, nnz=[len(x) for x in s.indices], uniq=t(s.uniq),
+                indptr=[t(x) for x in s.indptr], indices=[t(x) for x in s.indices], weights=None)
+        n = par.run_sampler(sample_fn, roles, rank, total, store, "t", "cpu")
+        np.save(os.path.join(outdir, f"s{rank}.npy"), np.array([n]))
+    else:
+        got = {}
+
+        def extract_fn(gidx, epoch, sizes, nnz, payload):
+            uniq, indptr, indices, _ = payload
+            exp = go.sample_khop(batches[gidx], sh.fanouts, g.seed, 1, gidx)
+            assert epoch == 1 and sizes == exp.sizes
+            assert np.array_equal(uniq.numpy().view(np.uint32), exp.uniq)
+            for l in range(len(sh.fanouts)):
+                assert np.array_equal(indptr[l].numpy().view(np.uint32), exp.indptr[l])
+                assert np.array_equal(indices[l].numpy().view(np.uint32), exp.indices[l])
+            feats = go.extract(uniq.numpy().view(np.uint32))
+            got[gidx] = float(feats.sum(dtype=np.float64))
+
+        n = par.run_trainer(extract_fn, roles, rank, total, store, "t", "cpu")
+        np.save(os.path.join(outdir, f"t{rank}.npy"), np.array(sorted(got)))
+        assert n == len(roles.trainer_batches(rank, total))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,ns", [(2, 1), (3, 2), (3, 1)])
+def test_factored_handoff_protocol(tmp_path, world, ns):
+    mp.spawn(_factored_worker, args=(world, free_port(), ns, str(tmp_path)), nprocs=world,
+             join=True)
+    total = 16
+    trained = sorted(int(x) for r in range(ns, world)
+                     for x in np.load(tmp_path / f"t{r}.npy"))
+    assert trained == list(range(total))                        # every batch extracted once
+    sampled = sum(int(np.load(tmp_path / f"s{r}.npy")[0]) for r in range(ns))
+    assert sampled == total                                     # every batch sampled once
+
+
+def test_header_payload_roundtrip():
+    b = types.SimpleNamespace(sizes=[3, 7, 12], nnz=[5, 9], uniq=torch.arange(12, dtype=torch.int32),
+                              indptr=[torch.tensor([0, 2, 4, 5], dtype=torch.int32),
+                                      torch.arange(8, dtype=torch.int32)],
+                              indices=[torch.arange(5, dtype=torch.int32),
+                                       torch.arange(9, dtype=torch.int32)],
+                              weights=[torch.ones(5, dtype=torch.int32),
+                                       torch.full((9,), 2, dtype=torch.int32)])
+    h = par.pack_header(41, 3, b.sizes, b.nnz, True, "cpu")
+    g, e, sizes, nnz, w = par.unpack_header(h)
+    assert (g, e, sizes, nnz, w) == (41, 3, b.sizes, b.nnz, True)
+    buf = par.pack_payload(b)
+    assert buf.numel() == par.payload_len(sizes, nnz, w)
+    uniq, ip, ix, ws = par.unpack_payload(buf, sizes, nnz, w)
+    assert torch.equal(uniq, b.uniq) and all(torch.equal(a, c) for a, c in zip(ip, b.indptr))
+    assert all(torch.equal(a, c) for a, c in zip(ix, b.indices))
+    assert all(torch.equal(a, c) for a, c in zip(ws, b.weights))

@@ -25,8 +25,7 @@ for hop in range(2):
     t = buf[hop].astype(np.int64)
     n = int((t[:, 0] > 0).sum())
     t = t[:n]
-    t0 = t[:, 0].min()
-    rel = (t - t0) / 1e3
+    rel = (t - t[:, :1]) / 1.965e3  # cycles -> us at 1965 MHz, relative to the tile claim
     print(f"hop {hop}: {n} tiles; span {rel[:, 5].max():.1f} us")
     names = ["claim", "loaded", "lookback", "scanned", "done", "end"]
     for ev in range(6):
