@@ -351,7 +351,8 @@ glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32
       CK(dalloc(&bs.bindptr[l], bs.ub[l] + 1));
       CK(dalloc(&bs.bindices[l], flat));
       if (kind == GLB_RANDOM_WALK) CK(dalloc(&bs.bweights[l], flat));
-      bs.ntiles[l] = (flat + kCompactTile - 1) / kCompactTile;
+      const uint64_t min_tile = (uint64_t)kThreads * kCompactMinItems;
+      bs.ntiles[l] = (flat + min_tile - 1) / min_tile;
       CK(dalloc(&bs.status[l], bs.ntiles[l]));
     }
     CK(dalloc(&bs.hit_list, un));

@@ -80,6 +80,7 @@ __global__ void __launch_bounds__(kThreads, 4)
              const uint32_t* __restrict__ fill_src, const uint32_t* __restrict__ dev_counts,
              uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t R,
              unsigned long long* xcount) {
+  pdl_enter();
   __shared__ uint2 ent[2][kThreads];
   const uint64_t nh = dev_counts ? dev_counts[0] : nh_host;
   const uint64_t nm = dev_counts ? dev_counts[1] : nm_host;
@@ -161,16 +162,16 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   if (R > (uint32_t)kThreads) R = kThreads;
   if (R < 1) R = 1;
   const int grid = c->num_sms * c->gather_bps;
+  cudaError_t e;
   if (vec)
-    k_gather<float4><<<grid, kThreads, 0, c->stream>>>(
-        (float4*)out, (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list,
-        fill_src, dev_counts, nhit_host, nmiss_host, U, R, c->xcount);
+    e = launch_pdl(k_gather<float4>, grid, kThreads, c->stream, (float4*)out,
+                   (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
+                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount);
   else
-    k_gather<float><<<grid, kThreads, 0, c->stream>>>(out, src_hit, src_miss, hit_list, miss_list,
-                                                      fill_src, dev_counts, nhit_host, nmiss_host,
-                                                      U, R, c->xcount);
+    e = launch_pdl(k_gather<float>, grid, kThreads, c->stream, out, src_hit, src_miss, hit_list,
+                   miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R, c->xcount);
   count_launch(c);
-  return cudaGetLastError();
+  return e;
 }
 
 }  // namespace glb

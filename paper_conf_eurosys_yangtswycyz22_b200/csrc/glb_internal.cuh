@@ -13,8 +13,16 @@ namespace glb {
 
 constexpr uint32_t kEmpty = 0xFFFFFFFFu;
 constexpr int kThreads = 256;          // block size of every grid-stride kernel
-constexpr int kCompactItems = 16;      // flat positions per thread in a compaction tile
-constexpr int kCompactTile = kThreads * kCompactItems;
+constexpr int kCompactItems = 16;      // max flat positions per thread in a compaction tile
+constexpr int kCompactTile = kThreads * kCompactItems;  // max tile
+constexpr int kCompactMinItems = 2;    // tiles shrink to >= 2 per SM for small hops
+// positions per thread for a hop of `flat` positions: aim at ~2 tiles per SM
+__host__ __device__ inline uint32_t compact_items(uint32_t flat, uint32_t num_sms) {
+  const uint32_t per = 2u * num_sms * (uint32_t)kThreads;
+  uint32_t it = (flat + per - 1) / per;
+  return it < (uint32_t)kCompactMinItems ? (uint32_t)kCompactMinItems
+         : it > (uint32_t)kCompactItems ? (uint32_t)kCompactItems : it;
+}
 constexpr int kMaxFanout = 1024;
 constexpr int kMaxWalkLen = 8;
 
@@ -188,6 +196,32 @@ struct glb_ctx {
 };
 
 namespace glb {
+
+// ---- programmatic dependent launch (sm_90+): a kernel of the hot path is
+// launched with programmaticStreamSerialization, so it is staged while its
+// predecessor drains; every such kernel starts with pdl_enter(): it allows its
+// own successor to be staged, then waits for its predecessor's completion and
+// memory before touching any data (no RAW/WAR hazard is possible).
+__device__ __forceinline__ void pdl_enter() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+  asm volatile("griddepcontrol.wait;" ::: "memory");
+}
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), unsigned grid, unsigned block,
+                              cudaStream_t s, Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(block);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
 
 // ---- launchers (defined in the .cu files) ----
 cudaError_t launch_validate_graph(glb_ctx* c);

@@ -55,9 +55,9 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 // is already <= e proves the atomic would be a no-op.
 __device__ __forceinline__ unsigned long long vmap_insert(VEntry* vmap, uint32_t u,
                                                           unsigned long long e) {
-  unsigned long long old = __ldcg(&vmap[u].gp);
-  if (old > e) old = atomicMin(&vmap[u].gp, e);
-  return old;  // <= e: an earlier position (or a lid) of this generation holds u
+  const unsigned long long old = __ldcg(&vmap[u].gp);
+  if (old > e) atomicMin(&vmap[u].gp, e);  // no return value needed: RED, no round trip
+  return old;  // <= e: an earlier position (or a lid) of this generation already held u
 }
 
 // Encoded pick: the gid, or -- when the sampler already found u relabelled by an
@@ -100,6 +100,7 @@ __global__ void __launch_bounds__(kThreads)
     k_seed_init(const uint32_t* __restrict__ seeds, uint32_t n0, uint64_t V, DevState* st,
                 uint32_t* __restrict__ uniq, VEntry* vmap, uint32_t gen, MarkArgs mk,
                 StatusArgs za) {
+  pdl_enter();
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     st->n[0] = n0;
     st->base[0] = n0;
@@ -148,6 +149,7 @@ __global__ void __launch_bounds__(kThreads)
            const DevState* __restrict__ st, DevState* st_w, const uint64_t* __restrict__ indptr,
            const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
            VEntry* vmap, uint32_t* __restrict__ picks, uint32_t* fix_ind) {
+  pdl_enter();
   if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);  // deferred lids of block hop-1
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
@@ -214,6 +216,7 @@ __global__ void __launch_bounds__(kThreads)
                 const uint64_t* __restrict__ indptr, const uint32_t* __restrict__ indices,
                 const uint32_t* __restrict__ uniq, VEntry* vmap,
                 uint32_t* __restrict__ picks, uint32_t* fix_ind) {
+  pdl_enter();
   __shared__ uint32_t chosen[kThreads / 32][kMaxFanout];
   if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);
   const uint32_t n_l = st->n[hop];
@@ -265,6 +268,7 @@ __global__ void __launch_bounds__(kThreads)
             const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
             VEntry* vmap, uint32_t* __restrict__ picks, uint32_t* __restrict__ pickw,
             uint32_t* fix_ind) {
+  pdl_enter();
   if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
@@ -405,7 +409,6 @@ __device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
 //  (gen, position) with (gen, lid); lid <= position, so the table stays
 //  monotone (later atomicMins never replace it) and a concurrent reader sees
 //  either value, both of which it resolves correctly.
-constexpr int kWarpSpan = kCompactTile / (kThreads / 32);  // positions per warp
 
 template <bool W>
 __global__ void __launch_bounds__(kThreads, 3)
@@ -414,7 +417,8 @@ __global__ void __launch_bounds__(kThreads, 3)
               VEntry* vmap,
               uint32_t* __restrict__ uniq, uint32_t* __restrict__ bindptr,
               uint32_t* __restrict__ bindices, uint32_t* __restrict__ bweights,
-              unsigned long long* status, MarkArgs mk) {
+              unsigned long long* status, MarkArgs mk, uint32_t num_sms) {
+  pdl_enter();
   constexpr int NW = kThreads / 32;
   __shared__ uint32_t s_tile;
   __shared__ unsigned long long s_wnv[NW];  // per warp (new << 32 | valid), then exclusive
@@ -426,7 +430,9 @@ __global__ void __launch_bounds__(kThreads, 3)
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
   const uint32_t flat = n_l * k;
-  const uint32_t ntiles = (flat + kCompactTile - 1) / kCompactTile;
+  const uint32_t items = compact_items(flat, num_sms);  // positions per thread
+  const uint32_t tile_n = items * kThreads;
+  const uint32_t ntiles = (flat + tile_n - 1) / tile_n;
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
   const uint32_t lt = lanemask_lt();
   if (flat == 0) {
@@ -445,14 +451,14 @@ __global__ void __launch_bounds__(kThreads, 3)
     const uint32_t tile = s_tile;
     if (tile >= ntiles) break;
     TRACE(hop, tile, 0);
-    const uint32_t t0 = tile * kCompactTile;
-    const uint32_t loc0 = wid * kWarpSpan + lane;  // local position of item 0
+    const uint32_t t0 = tile * tile_n;
+    const uint32_t loc0 = wid * items * 32 + lane;  // local position of item 0
     uint32_t u[kCompactItems];
     uint32_t p[kCompactItems];  // first position (this generation) of u[i]
 #pragma unroll
     for (int i = 0; i < kCompactItems; ++i) {
       const uint32_t f = t0 + loc0 + i * 32;
-      u[i] = f < flat ? picks[f] : kEmpty;
+      u[i] = ((uint32_t)i < items && f < flat) ? picks[f] : kEmpty;
     }
     uint32_t vmask = 0, nmask = 0, hmask = 0;
 #pragma unroll
@@ -597,7 +603,7 @@ __global__ void __launch_bounds__(kThreads, 3)
         const bool isv = (vmask >> i) & 1u;
         const uint32_t vb = __ballot_sync(kFull, isv);
         const uint32_t ev = rv + __popc(vb & lt);
-        if (f < flat && f % k == 0) bindptr[f / k] = ev;
+        if ((uint32_t)i < items && f < flat && f % k == 0) bindptr[f / k] = ev;
         if (isv) {
           bindices[ev] = lid[i];
           if (W) bweights[ev] = pickw[f];
@@ -613,6 +619,7 @@ __global__ void __launch_bounds__(kThreads, 3)
 __global__ void __launch_bounds__(kThreads)
     k_fixup(uint32_t hop, const DevState* __restrict__ st, const VEntry* vmap,
             uint32_t* __restrict__ bindices) {
+  pdl_enter();
   fixup_block(st->nnz[hop], vmap, bindices);
 }
 
@@ -659,10 +666,10 @@ cudaError_t launch_seed_init(glb_ctx* c, const uint32_t* seeds, uint32_t n0, int
     za.p[l] = c->sb.status[l];
     za.n[l] = (uint32_t)c->sb.ntiles[l];
   }
-  k_seed_init<<<blocks, kThreads, 0, c->stream>>>(seeds, n0, c->V, c->st, c->sb.uniq, c->vmap,
-                                                  c->gen, mark_args(c, count_mode), za);
+  const cudaError_t e = launch_pdl(k_seed_init, blocks, kThreads, c->stream, seeds, n0, c->V, c->st,
+                                   c->sb.uniq, c->vmap, c->gen, mark_args(c, count_mode), za);
   count_launch(c);
-  return cudaGetLastError();
+  return e;
 }
 
 cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch,
@@ -670,56 +677,71 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
   const int grid = grid_for(c);
   const SampleBufs& b = c->sb;
   uint32_t* fix = hop ? b.bindices[hop - 1] : nullptr;
+  const DevState* stc = c->st;
+  const uint64_t* ip = c->indptr;
+  const uint32_t* ix = c->indices;
+  const uint32_t* uq = b.uniq;
+  cudaError_t e;
   if (k <= 32)
-    k_khop<<<grid, kThreads, 0, c->stream>>>(hop, k, seed, epoch, batch, c->gen, c->st, c->st,
-                                             c->indptr, c->indices, b.uniq, c->vmap, b.picks,
-                                             fix);
+    e = launch_pdl(k_khop, grid, kThreads, c->stream, hop, k, seed, epoch, batch, c->gen, stc,
+                   c->st, ip, ix, uq, c->vmap, b.picks, fix);
   else
-    k_khop_wide<<<grid, kThreads, 0, c->stream>>>(hop, k, seed, epoch, batch, c->gen, c->st, c->st,
-                                                  c->indptr, c->indices, b.uniq, c->vmap, b.picks,
-                                                  fix);
+    e = launch_pdl(k_khop_wide, grid, kThreads, c->stream, hop, k, seed, epoch, batch, c->gen, stc,
+                   c->st, ip, ix, uq, c->vmap, b.picks, fix);
   count_launch(c);
-  return cudaGetLastError();
+  return e;
 }
 
 cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch, uint32_t batch) {
   const int grid = grid_for(c);
   const SampleBufs& b = c->sb;
-#define GLB_RW_ARGS                                                                          \
-  hop, c->rw_walks, c->rw_len, c->rw_topk, seed, epoch, batch, c->gen, c->st, c->st, c->indptr, \
-      c->indices, b.uniq, c->vmap, b.picks, b.pickw, fix
+#define GLB_RW_ARGS                                                                     \
+  hop, c->rw_walks, c->rw_len, c->rw_topk, seed, epoch, batch, c->gen, stc, c->st, ip, ix, uq, \
+      c->vmap, b.picks, b.pickw, fix
   uint32_t* fix = hop ? b.bindices[hop - 1] : nullptr;
   const uint32_t w = c->rw_walks;
-  if (w <= 1) k_rwalk<1><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
-  else if (w <= 2) k_rwalk<2><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
-  else if (w <= 4) k_rwalk<4><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
-  else if (w <= 8) k_rwalk<8><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
-  else if (w <= 16) k_rwalk<16><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
-  else k_rwalk<32><<<grid, kThreads, 0, c->stream>>>(GLB_RW_ARGS);
+  const DevState* stc = c->st;
+  const uint64_t* ip = c->indptr;
+  const uint32_t* ix = c->indices;
+  const uint32_t* uq = b.uniq;
+  cudaError_t e;
+  if (w <= 1) e = launch_pdl(k_rwalk<1>, grid, kThreads, c->stream, GLB_RW_ARGS);
+  else if (w <= 2) e = launch_pdl(k_rwalk<2>, grid, kThreads, c->stream, GLB_RW_ARGS);
+  else if (w <= 4) e = launch_pdl(k_rwalk<4>, grid, kThreads, c->stream, GLB_RW_ARGS);
+  else if (w <= 8) e = launch_pdl(k_rwalk<8>, grid, kThreads, c->stream, GLB_RW_ARGS);
+  else if (w <= 16) e = launch_pdl(k_rwalk<16>, grid, kThreads, c->stream, GLB_RW_ARGS);
+  else e = launch_pdl(k_rwalk<32>, grid, kThreads, c->stream, GLB_RW_ARGS);
 #undef GLB_RW_ARGS
   count_launch(c);
-  return cudaGetLastError();
+  return e;
 }
 
 cudaError_t launch_fixup(glb_ctx* c, uint32_t hop) {
-  k_fixup<<<grid_for(c), kThreads, 0, c->stream>>>(hop, c->st, c->vmap, c->sb.bindices[hop]);
+  const DevState* stc = c->st;
+  const VEntry* vm = c->vmap;
+  const cudaError_t e = launch_pdl(k_fixup, grid_for(c), kThreads, c->stream, hop, stc, vm,
+                                   c->sb.bindices[hop]);
   count_launch(c);
-  return cudaGetLastError();
+  return e;
 }
 
 cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, int count_mode) {
   const SampleBufs& b = c->sb;
   const int grid = grid_for(c, 3);
+  const uint32_t* pk = b.picks;
+  const uint32_t* pw = b.pickw;
+  const uint32_t nsm = (uint32_t)c->num_sms;
+  cudaError_t e;
   if (weighted)
-    k_compact<true><<<grid, kThreads, 0, c->stream>>>(
-        hop, k, c->gen, c->st, b.picks, b.pickw, c->vmap, b.uniq, b.bindptr[hop],
-        b.bindices[hop], b.bweights[hop], b.status[hop], mark_args(c, count_mode));
+    e = launch_pdl(k_compact<true>, grid, kThreads, c->stream, hop, k, c->gen, c->st, pk, pw,
+                   c->vmap, b.uniq, b.bindptr[hop], b.bindices[hop], b.bweights[hop],
+                   b.status[hop], mark_args(c, count_mode), nsm);
   else
-    k_compact<false><<<grid, kThreads, 0, c->stream>>>(
-        hop, k, c->gen, c->st, b.picks, nullptr, c->vmap, b.uniq, b.bindptr[hop],
-        b.bindices[hop], nullptr, b.status[hop], mark_args(c, count_mode));
+    e = launch_pdl(k_compact<false>, grid, kThreads, c->stream, hop, k, c->gen, c->st, pk,
+                   (const uint32_t*)nullptr, c->vmap, b.uniq, b.bindptr[hop], b.bindices[hop],
+                   (uint32_t*)nullptr, b.status[hop], mark_args(c, count_mode), nsm);
   count_launch(c);
-  return cudaGetLastError();
+  return e;
 }
 
 }  // namespace glb
