@@ -260,7 +260,9 @@ __global__ void __launch_bounds__(kThreads)
 
 // ---------------------------------------------------------------- random walk
 // PinSAGE (L209, L353): G >= walks lanes per frontier vertex, one walk per lane.
-template <int G>
+// PinSAGE (L209, L353): G >= walks lanes per frontier vertex, one walk per lane;
+// LEN >= walk length (register arrays; 3 for PinSAGE).
+template <int G, int LEN>
 __global__ void __launch_bounds__(kThreads)
     k_rwalk(uint32_t hop, uint32_t walks, uint32_t len, uint32_t topk, uint64_t seed,
             uint32_t epoch, uint32_t batch, uint32_t gen, const DevState* __restrict__ st,
@@ -283,16 +285,16 @@ __global__ void __launch_bounds__(kThreads)
     const uint32_t d = w0 + lane / G;
     const bool active = d < n_l;
     uint32_t v = 0;
-    uint32_t vis[kMaxWalkLen];
+    uint32_t vis[LEN];
 #pragma unroll
-    for (int t = 0; t < kMaxWalkLen; ++t) vis[t] = kEmpty;
+    for (int t = 0; t < LEN; ++t) vis[t] = kEmpty;
     if (active) {
       v = uniq[d];
       if (hop == 0 && w == 0 && __ldcg(&vmap[v].gp) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
       if (w < walks) {
         uint32_t cur = v;
 #pragma unroll
-        for (int t = 0; t < kMaxWalkLen; ++t) {
+        for (int t = 0; t < LEN; ++t) {
           if ((uint32_t)t < len) {
             const uint64_t b = indptr[cur];
             const uint32_t deg = (uint32_t)(indptr[cur + 1] - b);
@@ -305,38 +307,38 @@ __global__ void __launch_bounds__(kThreads)
       }
     }
     // visit counts and first occurrences over the group's walks*len entries
-    uint32_t cnt[kMaxWalkLen];
-    bool first[kMaxWalkLen];
+    uint32_t cnt[LEN];
+    bool first[LEN];
 #pragma unroll
-    for (int t = 0; t < kMaxWalkLen; ++t) { cnt[t] = 0; first[t] = true; }
+    for (int t = 0; t < LEN; ++t) { cnt[t] = 0; first[t] = true; }
     for (uint32_t src = 0; src < G; ++src) {
 #pragma unroll
-      for (int tt = 0; tt < kMaxWalkLen; ++tt) {
+      for (int tt = 0; tt < LEN; ++tt) {
         const uint32_t x = __shfl_sync(kFull, vis[tt], gbase + src);
 #pragma unroll
-        for (int t = 0; t < kMaxWalkLen; ++t) {
+        for (int t = 0; t < LEN; ++t) {
           if (vis[t] != kEmpty && x == vis[t]) {
             ++cnt[t];
-            if (src * kMaxWalkLen + tt < w * kMaxWalkLen + t) first[t] = false;
+            if (src * LEN + tt < w * LEN + t) first[t] = false;
           }
         }
       }
     }
     // rank of each distinct visited vertex by (count desc, gid asc)
-    uint32_t rank[kMaxWalkLen];
+    uint32_t rank[LEN];
     uint32_t ndist = 0;
 #pragma unroll
-    for (int t = 0; t < kMaxWalkLen; ++t) rank[t] = 0;
+    for (int t = 0; t < LEN; ++t) rank[t] = 0;
     for (uint32_t src = 0; src < G; ++src) {
 #pragma unroll
-      for (int tt = 0; tt < kMaxWalkLen; ++tt) {
+      for (int tt = 0; tt < LEN; ++tt) {
         const uint32_t x = __shfl_sync(kFull, vis[tt], gbase + src);
         const uint32_t xc = __shfl_sync(kFull, cnt[tt], gbase + src);
         const bool xf = __shfl_sync(kFull, first[tt], gbase + src);
         if (x != kEmpty && xf) {
           ++ndist;
 #pragma unroll
-          for (int t = 0; t < kMaxWalkLen; ++t)
+          for (int t = 0; t < LEN; ++t)
             if (vis[t] != kEmpty && first[t] && (xc > cnt[t] || (xc == cnt[t] && x < vis[t])))
               ++rank[t];
         }
@@ -346,7 +348,7 @@ __global__ void __launch_bounds__(kThreads)
       for (uint32_t r = w; r < topk; r += G)
         if (r >= ndist) picks[(size_t)d * topk + r] = kEmpty;
 #pragma unroll
-      for (int t = 0; t < kMaxWalkLen; ++t) {
+      for (int t = 0; t < LEN; ++t) {
         if (vis[t] != kEmpty && first[t] && rank[t] < topk) {
           const uint32_t f = d * topk + rank[t];
           const unsigned long long e = enc_pos(gen, base + f);
@@ -705,12 +707,16 @@ cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch
   const uint32_t* ix = c->indices;
   const uint32_t* uq = b.uniq;
   cudaError_t e;
-  if (w <= 1) e = launch_pdl(k_rwalk<1>, grid, kThreads, c->stream, GLB_RW_ARGS);
-  else if (w <= 2) e = launch_pdl(k_rwalk<2>, grid, kThreads, c->stream, GLB_RW_ARGS);
-  else if (w <= 4) e = launch_pdl(k_rwalk<4>, grid, kThreads, c->stream, GLB_RW_ARGS);
-  else if (w <= 8) e = launch_pdl(k_rwalk<8>, grid, kThreads, c->stream, GLB_RW_ARGS);
-  else if (w <= 16) e = launch_pdl(k_rwalk<16>, grid, kThreads, c->stream, GLB_RW_ARGS);
-  else e = launch_pdl(k_rwalk<32>, grid, kThreads, c->stream, GLB_RW_ARGS);
+#define GLB_RW_G(GG)                                                                    \
+  (c->rw_len <= 3 ? launch_pdl(k_rwalk<GG, 3>, grid, kThreads, c->stream, GLB_RW_ARGS) \
+                  : launch_pdl(k_rwalk<GG, kMaxWalkLen>, grid, kThreads, c->stream, GLB_RW_ARGS))
+  if (w <= 1) e = GLB_RW_G(1);
+  else if (w <= 2) e = GLB_RW_G(2);
+  else if (w <= 4) e = GLB_RW_G(4);
+  else if (w <= 8) e = GLB_RW_G(8);
+  else if (w <= 16) e = GLB_RW_G(16);
+  else e = GLB_RW_G(32);
+#undef GLB_RW_G
 #undef GLB_RW_ARGS
   count_launch(c);
   return e;
