@@ -52,6 +52,8 @@ def parse():
                    help="factored: Ns sampler + Nt trainer ranks (PAPER.md §5.2-5.3)")
     p.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                    help="gloo: CPU-staged send/recv (lets N ranks share one GPU for testing)")
+    p.add_argument("--relabel", default="auto", choices=["auto", "dense", "hash"],
+                   help="relabel table (glb_set_relabel_mode)")
     p.add_argument("--pipeline", type=int, default=1, choices=[1, 2],
                    help="2: extract of batch b overlaps sampling of batch b+1 (two streams)")
     return p.parse_args()
@@ -333,6 +335,7 @@ def main():
     ctx.load_graph(g.indptr, g.indices, g.features)
     t_load = time.perf_counter() - t0
     kind = sh.sampler
+    ctx.set_relabel_mode(args.relabel)
     if kind == "khop":
         ctx.set_sampler("khop", fanouts=sh.fanouts, max_batch=sh.batch)
     else:
@@ -546,6 +549,7 @@ def main():
                        "l2": "inputs larger than L2 (CSR %.2f GB, feature cache %.2f GB vs 126 MB L2)"
                              % ((8 * (sh.V + 1) + 4 * sh.E) / 1e9, 4 * sh.D * sh.V * args.alpha / 1e9)},
             "pipeline_depth": args.pipeline,
+            "relabel_table": ctx.relabel_mode,
             "host_wall_ms_timed_region": wall_ms,
             "host_enqueue_ms_timed_region": enqueue_ms,
             "roofline": {"kernel": "k_gather (extract a7)", "bound": "hbm", "achieved": ach_gbs,

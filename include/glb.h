@@ -84,6 +84,14 @@ glb_status glb_set_sampler(glb_ctx* ctx, int kind, const uint32_t* fanouts, uint
                            uint32_t rw_walks, uint32_t rw_len, uint32_t rw_topk,
                            uint32_t max_batch);
 
+/* Relabel table used by the next glb_set_sampler (dedup/relabel, L230 "remap(dedup(samples))"):
+ * 1 = dense direct-address table (16 B per vertex), 2 = open-addressing hash table sized
+ * from the batch's unique-vertex bound (L2-resident for large graphs), 0 = auto (dense unless
+ * V > 2x the hash capacity).  Results are identical in both modes.  glb_relabel_mode reports
+ * the mode in use (1 or 2). */
+glb_status glb_set_relabel_mode(glb_ctx* ctx, int mode);
+glb_status glb_relabel_mode(const glb_ctx* ctx, int* out);
+
 /* Training set T (host u32[n], distinct, each < V) and mini-batch size B
  * (L305 §6.2: shuffle T each epoch and divide it; last batch partial).
  * seed keys every draw of the ctx (shuffle and sampling).  Synchronous. */

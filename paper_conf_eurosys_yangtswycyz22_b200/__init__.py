@@ -35,6 +35,7 @@ EXPORTS = [
     "glb_get_counts", "glb_build_cache", "glb_get_cache_slots", "glb_cache_size",
     "glb_hit_stats_get", "glb_extract", "glb_extract_sample", "glb_kernel_launches",
     "glb_set_pipeline", "glb_extract_stream", "glb_set_timing", "glb_extract_times",
+    "glb_set_relabel_mode", "glb_relabel_mode",
 ]
 
 
@@ -113,6 +114,8 @@ def lib(auto_build: bool = True):
         "glb_extract_stream": ([vp, ctypes.POINTER(vp)], i32),
         "glb_set_timing": ([vp, i32], i32),
         "glb_extract_times": ([vp, vp, u64, ctypes.POINTER(u64)], i32),
+        "glb_set_relabel_mode": ([vp, i32], i32),
+        "glb_relabel_mode": ([vp, ctypes.POINTER(i32)], i32),
     }
     for name, (a, r) in sig.items():
         f = getattr(L, name)
@@ -228,6 +231,16 @@ class Context:
         self._ck(self._lib.glb_set_sampler(self._h, k, _np_ptr(fan), L, walks, walk_len, topk,
                                            max_batch))
         self.kind, self.L = kind, L
+
+    def set_relabel_mode(self, mode: str):
+        """'auto' | 'dense' | 'hash' -- relabel table for the next set_sampler."""
+        self._ck(self._lib.glb_set_relabel_mode(self._h, {"auto": 0, "dense": 1, "hash": 2}[mode]))
+
+    @property
+    def relabel_mode(self) -> str:
+        m = ctypes.c_int()
+        self._ck(self._lib.glb_relabel_mode(self._h, ctypes.byref(m)))
+        return {1: "dense", 2: "hash"}[m.value]
 
     def set_train_set(self, train: np.ndarray, batch_size: int, seed: int):
         t = np.ascontiguousarray(train, dtype=np.uint32)

@@ -64,6 +64,7 @@ void free_sample_bufs(glb_ctx* c) {
   for (int s = 0; s < 2; ++s) {
     SampleBufs& b = c->sbs[s];
     dfree(b.seeds); dfree(b.uniq); dfree(b.lidslot); dfree(b.picks); dfree(b.pickw);
+    dfree(b.pidx);
     for (int l = 0; l < GLB_MAX_HOPS; ++l) {
       dfree(b.bindptr[l]); dfree(b.bindices[l]); dfree(b.bweights[l]); dfree(b.status[l]);
     }
@@ -88,7 +89,11 @@ cudaError_t sync_all(glb_ctx* c) {
 }
 
 void free_graph(glb_ctx* c) {
-  dfree(c->indptr); dfree(c->indices); dfree(c->vmap);
+  dfree(c->indptr); dfree(c->indices); dfree(c->vmap); dfree(c->htab);
+  c->hslot = nullptr;
+  c->hmask = 0;
+  c->hash_mode = false;
+  c->pin = L2Window();
   dfree(c->slot); dfree(c->cache); dfree(c->counts); dfree(c->access);
   if (c->registered && c->h_features) cudaHostUnregister((void*)c->h_features);
   c->registered = false;
@@ -110,6 +115,7 @@ glb_status check_dev_err(glb_ctx* c, DevState* st) {
     if (err & kErrDupSeed) return set_err(c, GLB_EINVAL, "duplicate seed in batch");
     if (err & kErrRange) return set_err(c, GLB_EINVAL, "vertex id >= V");
     if (err & kErrBadGraph) return set_err(c, GLB_EINVAL, "invalid CSR");
+    if (err & kErrCapacity) return set_err(c, GLB_ENOMEM, "relabel hash table full");
     return set_err(c, GLB_EINVAL, "device error 0x%x", err);
   }
   return GLB_OK;
@@ -126,6 +132,7 @@ glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, in
     if (k[l] > c->sb.k[l]) return set_err(c, GLB_ENOMEM, "fanout %u > configured %u at hop %u", k[l], c->sb.k[l], l);
   if (c->gen >= 0xFFFFFFF0u) {  // generation wrap: clear the relabel table once
     CK(launch_vmap_reset(c));
+    CK(launch_table_reset(c));
     c->gen = 0;
   }
   c->gen += 1;
@@ -148,6 +155,25 @@ glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, in
   c->last_n0 = n0;
   for (uint32_t l = 0; l < L; ++l) c->last_k[l] = k[l];
   return GLB_OK;
+}
+
+// Persisting-L2 set-aside + window over the relabel table (skipped if unsupported).
+void set_l2_window(glb_ctx* c, void* base, size_t bytes) {
+  c->pin = L2Window();
+  if (!c->l2_pin || !base || !bytes) return;
+  int max_persist = 0, max_window = 0;
+  cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, c->device);
+  cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, c->device);
+  if (max_persist <= 0 || max_window <= 0) return;
+  const size_t setaside = bytes < (size_t)max_persist ? bytes : (size_t)max_persist;
+  if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setaside) != cudaSuccess) {
+    (void)cudaGetLastError();
+    return;
+  }
+  c->pin.base = base;
+  c->pin.bytes = bytes < (size_t)max_window ? bytes : (size_t)max_window;
+  const double r = (double)setaside / (double)c->pin.bytes;
+  c->pin.hit_ratio = r > 1.0 ? 1.0f : (float)r;
 }
 
 glb_status ensure_perm(glb_ctx* c, uint32_t epoch) {
@@ -200,6 +226,7 @@ glb_status glb_create(int device, glb_ctx** out) {
   c->stream = c->own_stream;
   c->st = c->sts[0];
   if (const char* g = getenv("GLB_GATHER_BPS")) c->gather_bps = atoi(g) > 0 ? atoi(g) : 4;
+  if (const char* g = getenv("GLB_L2_PIN")) c->l2_pin = atoi(g) != 0;
   *out = c;
   return GLB_OK;
 }
@@ -261,14 +288,12 @@ glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* in
   c->E = E;
   CK(dalloc(&c->indptr, V + 1));
   CK(dalloc(&c->indices, E));
-  CK(dalloc(&c->vmap, V));
   CK(dalloc(&c->slot, V));
   CK(dalloc(&c->counts, V));
   CK(dalloc(&c->access, V));
   CK(cudaMemcpy(c->indptr, indptr, sizeof(uint64_t) * (V + 1), cudaMemcpyHostToDevice));
   if (E) CK(cudaMemcpy(c->indices, indices, sizeof(uint32_t) * E, cudaMemcpyHostToDevice));
   CK(cudaMemsetAsync(c->slot, 0xFF, sizeof(int32_t) * V, c->stream));
-  CK(launch_vmap_reset(c));
   CK(cudaMemsetAsync(c->counts, 0, sizeof(uint32_t) * V, c->stream));
   CK(cudaMemsetAsync(c->access, 0, sizeof(uint32_t) * V, c->stream));
   CK(cudaMemsetAsync(c->st, 0, sizeof(DevState), c->stream));
@@ -338,6 +363,36 @@ glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32
   }
   if (pos >= 0xFFFFFFFFull) return set_err(c, GLB_ENOMEM, "relabel positions overflow 2^32");
   const uint64_t un = b.ub[L] > max_batch ? b.ub[L] : max_batch;
+  // relabel table: dense (one entry per vertex) unless the vertex count dwarfs the
+  // batch's unique-vertex bound -- then an L2-sized open-addressing hash table
+  uint64_t H = 1024;
+  while (H < un + un / 4 && H < kMaxHashEntries) H <<= 1;
+  if (const char* hc = getenv("GLB_HASH_LOG2")) {  // experiment: explicit capacity
+    const int lg = atoi(hc);
+    if (lg >= 10 && lg <= 30) H = 1ull << lg;
+  }
+  // auto = dense: measured equal or faster than the hash table on every config
+  // (DESIGN.md §7); hash only when the dense table would not fit comfortably.
+  size_t free_b = 0, total_b = 0;
+  cudaMemGetInfo(&free_b, &total_b);
+  const bool hash = c->relabel_mode == 2 ||
+                    (c->relabel_mode == 0 && c->V * sizeof(VEntry) > free_b / 4);
+  dfree(c->vmap); dfree(c->htab);
+  c->hslot = nullptr;
+  c->hmask = 0;
+  c->hash_mode = hash;
+  if (hash) {
+    // one allocation: entries then their cache slots, so one L2 window covers both
+    CK(dalloc(&c->htab, H + (H * sizeof(int32_t) + sizeof(VEntry) - 1) / sizeof(VEntry)));
+    c->hslot = reinterpret_cast<int32_t*>(c->htab + H);
+    c->hmask = (uint32_t)(H - 1);
+    CK(launch_table_reset(c));
+  } else {
+    CK(dalloc(&c->vmap, c->V));
+    CK(launch_vmap_reset(c));
+  }
+  set_l2_window(c, hash ? (void*)c->htab : (void*)c->vmap,
+                hash ? H * (sizeof(VEntry) + sizeof(int32_t)) : c->V * sizeof(VEntry));
   for (int s = 1; s >= 0; --s) {  // two slots: pipeline depth 2 double-buffers samples
     SampleBufs& bs = c->sbs[s];
     bs = b;
@@ -345,6 +400,7 @@ glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32
     CK(dalloc(&bs.uniq, un));
     CK(dalloc(&bs.lidslot, un));
     CK(dalloc(&bs.picks, maxflat));
+    if (hash) CK(dalloc(&bs.pidx, maxflat));
     if (kind == GLB_RANDOM_WALK) CK(dalloc(&bs.pickw, maxflat));
     for (uint32_t l = 0; l < L; ++l) {
       const uint64_t flat = bs.ub[l] * k[l];
@@ -431,6 +487,7 @@ glb_status glb_sample_result(glb_ctx* c, glb_blocks* out) {
     CK(cudaMemsetAsync(&c->st->err, 0, sizeof(uint32_t), c->stream));
     if (h.err & kErrDupSeed) return set_err(c, GLB_EINVAL, "duplicate seed in batch");
     if (h.err & kErrRange) return set_err(c, GLB_EINVAL, "seed id >= V");
+    if (h.err & kErrCapacity) return set_err(c, GLB_ENOMEM, "relabel hash table full");
     return set_err(c, GLB_EINVAL, "device error 0x%x", h.err);
   }
   if (!out) return GLB_OK;
@@ -565,8 +622,7 @@ glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
   CK(radix_sort_pairs_u32(c, k0, v0, k1, v1, V, bits, &ko, &order));
   CK(cudaMemsetAsync(c->slot, 0xFF, sizeof(int32_t) * V, c->stream));
   CK(launch_assign_slots(c, order, C));
-  CK(launch_vmap_reset(c));  // copy the slots into the relabel entries (and clear them)
-  c->gen = 0;
+  CK(launch_vmap_reset(c));  // dense mode: copy the slots into the relabel entries
   dfree(c->cache);
   c->C = C;
   if (c->features_mapped && C) {
@@ -693,6 +749,19 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
   if (e == cudaSuccess && c->nslots == 2) e = cudaEventRecord(c->ev_extracted[slot], c->stream);
   c->stream = main;
   if (e != cudaSuccess) return cuda_fail(c, e, "extract_sample");
+  return GLB_OK;
+}
+
+glb_status glb_set_relabel_mode(glb_ctx* c, int mode) {
+  ENTER(c);
+  if (mode < 0 || mode > 2) return set_err(c, GLB_EINVAL, "relabel mode must be 0 (auto), 1 (dense) or 2 (hash)");
+  c->relabel_mode = mode;
+  return GLB_OK;
+}
+
+glb_status glb_relabel_mode(const glb_ctx* c, int* out) {
+  if (!c || !out) return GLB_EINVAL;
+  *out = c->hash_mode ? 2 : 1;
   return GLB_OK;
 }
 

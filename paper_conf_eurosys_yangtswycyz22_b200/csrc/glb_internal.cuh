@@ -31,6 +31,7 @@ enum : uint32_t { kDomShuffle = 1, kDomKhop = 2, kDomRwalk = 3 };
 
 // device error bits (DevState::err)
 enum : uint32_t { kErrDupSeed = 1u, kErrRange = 2u, kErrCapacity = 4u, kErrBadGraph = 8u };
+constexpr uint32_t kMaxHashEntries = 1u << 23;  // 128 MB table cap
 
 // Per-batch device state.  Sizes live here so no kernel needs a host sync.
 struct DevState {
@@ -77,13 +78,21 @@ __device__ __forceinline__ uint64_t enc_pos(uint32_t gen, uint32_t pos) {
   return ((uint64_t)(0xFFFFFFFFu - gen) << 32) | pos;
 }
 
-// Relabel-table entry (one per vertex): gp = ((0xFFFFFFFF - gen) << 32) | first
-// position, then | lid once relabelled; slot = the vertex's cache slot (-1 = not
-// cached), co-located so one 16-byte load gives both (a4 mark needs no extra access).
+// Relabel-table entry: gp = ((0xFFFFFFFF - gen) << 32) | first position, then
+// | lid once relabelled.  Dense mode (one entry per vertex): aux = the vertex's
+// cache slot (-1 = not cached), co-located so one 16-byte load gives both (a4
+// mark needs no extra access).  Hash mode: aux = (gen << 32 | gid) key.
 struct __align__(16) VEntry {
   unsigned long long gp;
-  int32_t slot;
-  uint32_t pad;
+  unsigned long long aux;  // dense: cache slot (low 32 bits); hash: gen << 32 | gid
+};
+
+// Optional L2 access-policy window: the relabel table is marked persisting so the
+// random CSR / feature traffic between its accesses does not evict it.
+struct L2Window {
+  void* base = nullptr;
+  size_t bytes = 0;
+  float hit_ratio = 0.f;
 };
 
 struct SampleBufs {
@@ -95,6 +104,7 @@ struct SampleBufs {
   uint32_t* uniq = nullptr;           // u32[ub[L]]
   int32_t* lidslot = nullptr;         // i32[ub[L]]  (a4 marks)
   uint32_t* picks = nullptr;          // u32[max ub[l]*k[l]]
+  uint32_t* pidx = nullptr;           // u32[...] hash mode: table index of each pick
   uint32_t* pickw = nullptr;          // u32[...] random-walk counts
   uint32_t* bindptr[GLB_MAX_HOPS] = {};
   uint32_t* bindices[GLB_MAX_HOPS] = {};
@@ -132,7 +142,14 @@ struct glb_ctx {
   uint32_t D = 0;
 
   // relabel tables (D6): direct-address over gids
-  glb::VEntry* vmap = nullptr;  // [V]: (gen, first position) then (gen, lid); cache slot
+  glb::VEntry* vmap = nullptr;  // dense relabel table [V]: (gen, position|lid), cache slot
+  glb::VEntry* htab = nullptr;  // hash relabel table [hmask+1]: (gen, position|lid), key
+  int32_t* hslot = nullptr;     // [hmask+1] cache slot of each hash entry
+  uint32_t hmask = 0;
+  bool hash_mode = false;
+  int relabel_mode = 0;         // 0 auto, 1 dense, 2 hash (glb_set_relabel_mode)
+  glb::L2Window pin;            // persisting-L2 window over the relabel table
+  bool l2_pin = false;          // GLB_L2_PIN=1 enables (measured slower: DESIGN.md)
   uint32_t gen = 0;
 
   // cache (D3, D4, D5)
@@ -208,19 +225,35 @@ __device__ __forceinline__ void pdl_enter() {
 }
 
 template <typename... KArgs, typename... Args>
-inline cudaError_t launch_pdl(void (*kern)(KArgs...), unsigned grid, unsigned block,
-                              cudaStream_t s, Args... args) {
+inline cudaError_t launch_pdl_w(const L2Window& w, void (*kern)(KArgs...), unsigned grid,
+                                unsigned block, cudaStream_t s, Args... args) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(grid);
   cfg.blockDim = dim3(block);
   cfg.dynamicSmemBytes = 0;
   cfg.stream = s;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = 1;
+  int n = 1;
+  if (w.bytes) {
+    attr[1].id = cudaLaunchAttributeAccessPolicyWindow;
+    attr[1].val.accessPolicyWindow.base_ptr = w.base;
+    attr[1].val.accessPolicyWindow.num_bytes = w.bytes;
+    attr[1].val.accessPolicyWindow.hitRatio = w.hit_ratio;
+    attr[1].val.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    attr[1].val.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    n = 2;
+  }
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = n;
   return cudaLaunchKernelEx(&cfg, kern, static_cast<KArgs>(args)...);
+}
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), unsigned grid, unsigned block,
+                              cudaStream_t s, Args... args) {
+  return launch_pdl_w(L2Window(), kern, grid, block, s, args...);
 }
 
 // ---- launchers (defined in the .cu files) ----
@@ -231,6 +264,7 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
 cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch, uint32_t batch);
 cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, int count_mode);
 cudaError_t launch_fixup(glb_ctx* c, uint32_t hop);
+cudaError_t launch_table_reset(glb_ctx* c);
 cudaError_t launch_mark(glb_ctx* c, const uint32_t* vertices, uint64_t n);
 // Gather rows: hits src_hit[list.y] -> out[list.x], misses src_miss[list.y] -> out[list.x];
 // fill_src (non-null) replaces miss_list with (r, fill_src[r]) (identity destination).

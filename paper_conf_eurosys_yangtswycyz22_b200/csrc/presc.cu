@@ -244,8 +244,7 @@ __global__ void k_vmap_reset(VEntry* __restrict__ vmap, const int32_t* __restric
        i += (uint64_t)gridDim.x * blockDim.x) {
     VEntry e;
     e.gp = ~0ull;
-    e.slot = slot[i];
-    e.pad = 0;
+    e.aux = (unsigned long long)(uint32_t)slot[i];
     vmap[i] = e;
   }
 }
@@ -389,6 +388,7 @@ cudaError_t launch_assign_slots(glb_ctx* c, const uint32_t* order, uint64_t C) {
 }
 
 cudaError_t launch_vmap_reset(glb_ctx* c) {
+  if (!c->vmap) return cudaSuccess;
   k_vmap_reset<<<grid_for(c), kThreads, 0, c->stream>>>(c->vmap, c->slot, c->V);
   count_launch(c);
   return cudaGetLastError();

@@ -60,6 +60,71 @@ __device__ __forceinline__ unsigned long long vmap_insert(VEntry* vmap, uint32_t
   return old;  // <= e: an earlier position (or a lid) of this generation already held u
 }
 
+// The relabel table.  Dense mode: entry index = gid (V entries; aux = cache slot).
+// Hash mode (large V): open addressing with linear probing over mask+1 entries
+// sized from the batch's unique-vertex bound, so the table stays L2-resident;
+// aux = (gen << 32 | gid) -- entries of older generations count as free, so the
+// table is never cleared -- and the claimer of an entry copies the vertex's cache
+// slot into hslot[index].  Both modes share gp semantics and every later step
+// addresses entries by index.
+struct Table {
+  VEntry* e;
+  int32_t* hslot;       // hash mode: cache slot per entry
+  const int32_t* slot;  // [V] cache slot map
+  uint32_t mask;        // hash mode: capacity - 1
+  uint32_t gen;
+};
+
+__device__ __forceinline__ uint32_t hash32(uint32_t x) {  // lowbias32 mixer
+  x ^= x >> 16;
+  x *= 0x7feb352du;
+  x ^= x >> 15;
+  x *= 0x846ca68bu;
+  x ^= x >> 16;
+  return x;
+}
+
+// Find or claim gid's entry for this generation; kEmpty if the table is full.
+__device__ __forceinline__ uint32_t hclaim(const Table& T, uint32_t gid, bool& claimed) {
+  const unsigned long long key = ((unsigned long long)T.gen << 32) | gid;
+  uint32_t h = hash32(gid) & T.mask;
+  claimed = false;
+  // bounded probing: a run this long means the table is (nearly) full -> ENOMEM
+  const uint32_t max_probe = T.mask < 1023u ? T.mask : 1023u;
+  for (uint32_t probe = 0, tries = 0; probe <= max_probe && tries < 4096u; ++tries) {
+    unsigned long long* kp = &T.e[h].aux;
+    const unsigned long long kg = __ldcg(kp);
+    if (kg == key) return h;
+    if ((uint32_t)(kg >> 32) != T.gen) {  // free in this generation: try to claim it
+      const unsigned long long prev = atomicCAS(kp, kg, key);
+      if (prev == kg) {
+        claimed = true;
+        return h;
+      }
+      if (prev == key) return h;
+      if ((uint32_t)(prev >> 32) != T.gen) continue;  // lost to nothing we know: retry slot
+    }
+    h = (h + 1) & T.mask;
+    ++probe;
+  }
+  return kEmpty;
+}
+
+// Entry index of gid (dense: gid; hash: found / claimed, the claimer records
+// the cache slot).  kEmpty (and an error flag) when the hash table is full.
+template <bool HASH>
+__device__ __forceinline__ uint32_t entry_of(const Table& T, uint32_t gid, DevState* st) {
+  if (!HASH) return gid;
+  bool claimed;
+  const uint32_t h = hclaim(T, gid, claimed);
+  if (h == kEmpty) {
+    atomicOr(&st->err, kErrCapacity);
+    return kEmpty;
+  }
+  if (claimed) T.hslot[h] = __ldg(T.slot + gid);
+  return h;
+}
+
 // Encoded pick: the gid, or -- when the sampler already found u relabelled by an
 // earlier hop / as a seed (table value (gen, lid) with lid < base) -- lid | kOld,
 // so the compaction needs no table access for it.  gids and lids are < 2^31.
@@ -70,9 +135,9 @@ __device__ __forceinline__ uint32_t encode_pick(uint32_t u, unsigned long long o
   return u;
 }
 
-constexpr uint32_t kDefer = 0x80000000u;  // deferred src lid marker (gids < 2^31, glb_load_graph)
+constexpr uint32_t kDefer = 0x80000000u;  // deferred src lid marker (indices < 2^31)
 
-// Resolve deferred src lids of block `hop` (entries gid | kDefer).
+// Resolve deferred src lids of block `hop` (entries = table index | kDefer).
 __device__ __forceinline__ void fixup_block(uint32_t nnz, const VEntry* vmap,
                                             uint32_t* __restrict__ bindices) {
   for (uint32_t e = blockIdx.x * blockDim.x + threadIdx.x; e < nnz; e += gridDim.x * blockDim.x) {
@@ -96,10 +161,10 @@ struct StatusArgs {  // look-back status arrays to clear for this batch
 };
 
 // ---------------------------------------------------------------- seeds
+template <bool HASH>
 __global__ void __launch_bounds__(kThreads)
     k_seed_init(const uint32_t* __restrict__ seeds, uint32_t n0, uint64_t V, DevState* st,
-                uint32_t* __restrict__ uniq, VEntry* vmap, uint32_t gen, MarkArgs mk,
-                StatusArgs za) {
+                uint32_t* __restrict__ uniq, Table T, MarkArgs mk, StatusArgs za) {
   pdl_enter();
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     st->n[0] = n0;
@@ -122,7 +187,18 @@ __global__ void __launch_bounds__(kThreads)
         u = 0;  // keep later kernels in bounds; the batch is reported invalid
       }
       uniq[i] = u;
-      atomicMin(&vmap[u].gp, enc_pos(gen, i));  // a seed's position is its lid
+      if (HASH) {
+        bool claimed;
+        const uint32_t h = hclaim(T, u, claimed);
+        if (h == kEmpty) atomicOr(&st->err, kErrCapacity);
+        else {
+          if (!claimed) atomicOr(&st->err, kErrDupSeed);  // key already inserted this batch
+          T.hslot[h] = __ldg(T.slot + u);
+          atomicMin(&T.e[h].gp, enc_pos(T.gen, i));  // a seed's position is its lid
+        }
+      } else {
+        atomicMin(&T.e[u].gp, enc_pos(T.gen, i));
+      }
       s = __ldg(mk.slot + u);
       mk.lidslot[i] = s;
       if (mk.count) atomicAdd(mk.count + u, 1u);
@@ -144,13 +220,15 @@ __global__ void __launch_bounds__(kThreads)
 // ---------------------------------------------------------------- k-hop (k lanes / vertex)
 // Fanout k <= 32: floor(32/k) frontier vertices per warp, lane s of a group
 // owns Floyd slot s.
+template <bool HASH>
 __global__ void __launch_bounds__(kThreads)
-    k_khop(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch, uint32_t gen,
+    k_khop(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch, Table T,
            const DevState* __restrict__ st, DevState* st_w, const uint64_t* __restrict__ indptr,
            const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
-           VEntry* vmap, uint32_t* __restrict__ picks, uint32_t* fix_ind) {
+           uint32_t* __restrict__ picks, uint32_t* __restrict__ pidx, uint32_t* fix_ind) {
   pdl_enter();
-  if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);  // deferred lids of block hop-1
+  if (fix_ind) fixup_block(st->nnz[hop - 1], T.e, fix_ind);  // deferred lids of block hop-1
+  const uint32_t gen = T.gen;
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
   const uint32_t c3 = ctr3(epoch, hop, kDomKhop);
@@ -170,7 +248,8 @@ __global__ void __launch_bounds__(kThreads)
       v = uniq[d];
       lo = indptr[v];
       deg = (uint32_t)(indptr[v + 1] - lo);
-      if (hop == 0 && s == 0 && __ldcg(&vmap[v].gp) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
+      if (!HASH && hop == 0 && s == 0 && __ldcg(&T.e[v].gp) != enc_pos(gen, d))
+        atomicOr(&st_w->err, kErrDupSeed);
     }
     const bool big = active && deg > k;
     uint32_t t = 0, j = 0;
@@ -199,26 +278,36 @@ __global__ void __launch_bounds__(kThreads)
       if (big) sel = disp ? j : t;
     }
     if (!big && active && s < deg) sel = s;
-    uint32_t u = kEmpty;
+    uint32_t u = kEmpty, idx = kEmpty;
     if (sel != kEmpty) {
       u = __ldg(indices + lo + sel);
-      const unsigned long long e = enc_pos(gen, base + d * k + s);
-      u = encode_pick(u, vmap_insert(vmap, u, e), e, base);
+      idx = entry_of<HASH>(T, u, st_w);
+      if (idx != kEmpty) {
+        const unsigned long long e = enc_pos(gen, base + d * k + s);
+        u = encode_pick(u, vmap_insert(T.e, idx, e), e, base);
+      } else {
+        u = kEmpty;
+      }
     }
-    if (active) picks[(size_t)d * k + s] = u;
+    if (active) {
+      picks[(size_t)d * k + s] = u;
+      if (HASH) pidx[(size_t)d * k + s] = idx;
+    }
   }
 }
 
 // Fanout > 32: one warp per vertex, Floyd run sequentially by lane 0 in shared memory.
+template <bool HASH>
 __global__ void __launch_bounds__(kThreads)
     k_khop_wide(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch,
-                uint32_t gen, const DevState* __restrict__ st, DevState* st_w,
+                Table T, const DevState* __restrict__ st, DevState* st_w,
                 const uint64_t* __restrict__ indptr, const uint32_t* __restrict__ indices,
-                const uint32_t* __restrict__ uniq, VEntry* vmap,
-                uint32_t* __restrict__ picks, uint32_t* fix_ind) {
+                const uint32_t* __restrict__ uniq, uint32_t* __restrict__ picks,
+                uint32_t* __restrict__ pidx, uint32_t* fix_ind) {
   pdl_enter();
   __shared__ uint32_t chosen[kThreads / 32][kMaxFanout];
-  if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);
+  if (fix_ind) fixup_block(st->nnz[hop - 1], T.e, fix_ind);
+  const uint32_t gen = T.gen;
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
   const uint32_t c3 = ctr3(epoch, hop, kDomKhop);
@@ -230,7 +319,8 @@ __global__ void __launch_bounds__(kThreads)
     const uint32_t v = uniq[d];
     const uint64_t lo = indptr[v];
     const uint32_t deg = (uint32_t)(indptr[v + 1] - lo);
-    if (hop == 0 && lane == 0 && __ldcg(&vmap[v].gp) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
+    if (!HASH && hop == 0 && lane == 0 && __ldcg(&T.e[v].gp) != enc_pos(gen, d))
+      atomicOr(&st_w->err, kErrDupSeed);
     if (deg > k) {
       if (lane == 0) {
         for (uint32_t s = 0; s < k; ++s) {
@@ -247,12 +337,18 @@ __global__ void __launch_bounds__(kThreads)
       uint32_t sel = kEmpty;
       if (deg > k) sel = ch[s];
       else if (s < deg) sel = s;
-      uint32_t u = sel != kEmpty ? __ldg(indices + lo + sel) : kEmpty;
+      uint32_t u = sel != kEmpty ? __ldg(indices + lo + sel) : kEmpty, idx = kEmpty;
       if (u != kEmpty) {
-        const unsigned long long e = enc_pos(gen, base + d * k + s);
-        u = encode_pick(u, vmap_insert(vmap, u, e), e, base);
+        idx = entry_of<HASH>(T, u, st_w);
+        if (idx != kEmpty) {
+          const unsigned long long e = enc_pos(gen, base + d * k + s);
+          u = encode_pick(u, vmap_insert(T.e, idx, e), e, base);
+        } else {
+          u = kEmpty;
+        }
       }
       picks[(size_t)d * k + s] = u;
+      if (HASH) pidx[(size_t)d * k + s] = idx;
     }
     __syncwarp();
   }
@@ -262,16 +358,17 @@ __global__ void __launch_bounds__(kThreads)
 // PinSAGE (L209, L353): G >= walks lanes per frontier vertex, one walk per lane.
 // PinSAGE (L209, L353): G >= walks lanes per frontier vertex, one walk per lane;
 // LEN >= walk length (register arrays; 3 for PinSAGE).
-template <int G, int LEN>
+template <int G, int LEN, bool HASH>
 __global__ void __launch_bounds__(kThreads)
     k_rwalk(uint32_t hop, uint32_t walks, uint32_t len, uint32_t topk, uint64_t seed,
-            uint32_t epoch, uint32_t batch, uint32_t gen, const DevState* __restrict__ st,
+            uint32_t epoch, uint32_t batch, Table T, const DevState* __restrict__ st,
             DevState* st_w, const uint64_t* __restrict__ indptr,
             const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
-            VEntry* vmap, uint32_t* __restrict__ picks, uint32_t* __restrict__ pickw,
-            uint32_t* fix_ind) {
+            uint32_t* __restrict__ picks, uint32_t* __restrict__ pickw,
+            uint32_t* __restrict__ pidx, uint32_t* fix_ind) {
   pdl_enter();
-  if (fix_ind) fixup_block(st->nnz[hop - 1], vmap, fix_ind);
+  if (fix_ind) fixup_block(st->nnz[hop - 1], T.e, fix_ind);
+  const uint32_t gen = T.gen;
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
   const uint32_t c3 = ctr3(epoch, hop, kDomRwalk);
@@ -290,7 +387,8 @@ __global__ void __launch_bounds__(kThreads)
     for (int t = 0; t < LEN; ++t) vis[t] = kEmpty;
     if (active) {
       v = uniq[d];
-      if (hop == 0 && w == 0 && __ldcg(&vmap[v].gp) != enc_pos(gen, d)) atomicOr(&st_w->err, kErrDupSeed);
+      if (!HASH && hop == 0 && w == 0 && __ldcg(&T.e[v].gp) != enc_pos(gen, d))
+        atomicOr(&st_w->err, kErrDupSeed);
       if (w < walks) {
         uint32_t cur = v;
 #pragma unroll
@@ -352,7 +450,9 @@ __global__ void __launch_bounds__(kThreads)
         if (vis[t] != kEmpty && first[t] && rank[t] < topk) {
           const uint32_t f = d * topk + rank[t];
           const unsigned long long e = enc_pos(gen, base + f);
-          picks[f] = encode_pick(vis[t], vmap_insert(vmap, vis[t], e), e, base);
+          const uint32_t idx = entry_of<HASH>(T, vis[t], st_w);
+          picks[f] = idx == kEmpty ? kEmpty : encode_pick(vis[t], vmap_insert(T.e, idx, e), e, base);
+          if (HASH) pidx[f] = idx;
           pickw[f] = cnt[t];
         }
       }
@@ -412,11 +512,11 @@ __device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
 //  monotone (later atomicMins never replace it) and a concurrent reader sees
 //  either value, both of which it resolves correctly.
 
-template <bool W>
+template <bool W, bool HASH>
 __global__ void __launch_bounds__(kThreads, 3)
-    k_compact(uint32_t hop, uint32_t k, uint32_t gen, DevState* st,
+    k_compact(uint32_t hop, uint32_t k, Table T, DevState* st,
               const uint32_t* __restrict__ picks, const uint32_t* __restrict__ pickw,
-              VEntry* vmap,
+              const uint32_t* __restrict__ pidx,
               uint32_t* __restrict__ uniq, uint32_t* __restrict__ bindptr,
               uint32_t* __restrict__ bindices, uint32_t* __restrict__ bweights,
               unsigned long long* status, MarkArgs mk, uint32_t num_sms) {
@@ -427,8 +527,10 @@ __global__ void __launch_bounds__(kThreads, 3)
   __shared__ uint32_t s_whm[NW];            // per warp (hit | miss << 16), then exclusive
   __shared__ unsigned long long s_excl;
   __shared__ uint32_t s_hbase, s_mbase;
+  // per position: the cache slot of a new vertex (phase 1 -> 3), then its lid (3 -> 4)
   __shared__ uint32_t s_lid[kCompactTile];
-  __shared__ int32_t s_slot[kCompactTile];
+  __shared__ uint32_t s_idx[HASH ? kCompactTile : 1];  // hash mode: table index per position
+  const uint32_t gen = T.gen;
   const uint32_t n_l = st->n[hop];
   const uint32_t base = st->base[hop];
   const uint32_t flat = n_l * k;
@@ -471,13 +573,15 @@ __global__ void __launch_bounds__(kThreads, 3)
         if (u[i] & kOld) {
           p[i] = u[i] & ~kOld;  // the sampler resolved it: a lid < base
         } else {
-          // one 16-byte load: (gen, position-or-lid) and the cache slot
-          const ulonglong2 ent = __ldcg(reinterpret_cast<const ulonglong2*>(vmap + u[i]));
+          // dense: one 16-byte load gives (gen, position-or-lid) and the cache slot
+          const uint32_t idx = HASH ? pidx[t0 + loc0 + i * 32] : u[i];
+          if (HASH) s_idx[loc0 + i * 32] = idx;
+          const ulonglong2 ent = __ldcg(reinterpret_cast<const ulonglong2*>(T.e + idx));
           p[i] = (uint32_t)ent.x;
           if (ent.x == enc_pos(gen, base + t0 + loc0 + i * 32)) {
             nmask |= 1u << i;
-            const int32_t sl = (int32_t)(uint32_t)ent.y;
-            s_slot[loc0 + i * 32] = sl;
+            const int32_t sl = HASH ? __ldcg(T.hslot + idx) : (int32_t)(uint32_t)ent.y;
+            s_lid[loc0 + i * 32] = (uint32_t)sl;
             if (sl >= 0) hmask |= 1u << i;
           }
         }
@@ -568,9 +672,9 @@ __global__ void __launch_bounds__(kThreads, 3)
         if (isn) {
           const uint32_t loc = loc0 + i * 32;
           const uint32_t lid = n_l + rn + __popc(nb & lt);
-          const int32_t sl = s_slot[loc];
+          const int32_t sl = (int32_t)s_lid[loc];
           uniq[lid] = u[i];
-          __stcg(&vmap[u[i]].gp, enc_pos(gen, lid));  // relabelled: later readers get the lid
+          __stcg(&T.e[HASH ? s_idx[loc] : u[i]].gp, enc_pos(gen, lid));  // relabelled: readers get the lid
           mk.lidslot[lid] = sl;
           if (ish) mk.hit_list[rh + __popc(hb & lt)] = make_uint2(lid, (uint32_t)sl);
           else mk.miss_list[rm + __popc(mb & lt)] = make_uint2(lid, u[i]);
@@ -595,7 +699,7 @@ __global__ void __launch_bounds__(kThreads, 3)
           if ((nmask >> i) & 1u) lid[i] = s_lid[loc0 + i * 32];
           else if (p[i] < base) lid[i] = p[i];                   // relabelled earlier (lid)
           else if (fp >= t0) lid[i] = s_lid[fp - t0];           // earlier in this tile
-          else lid[i] = u[i] | kDefer;                          // earlier tile: fixup
+          else lid[i] = (HASH ? s_idx[loc0 + i * 32] : u[i]) | kDefer;  // earlier tile: fixup
         }
       }
       uint32_t rv = (uint32_t)ex;
@@ -636,6 +740,15 @@ __global__ void k_validate(const uint64_t* __restrict__ indptr, const uint32_t* 
   if (bad) atomicOr(&st->err, kErrBadGraph);
 }
 
+// Hash mode: every entry free (generation 0 is never used) with gp = max.
+__global__ void k_table_reset(VEntry* __restrict__ t, uint64_t n) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (uint64_t)gridDim.x * blockDim.x) {
+    t[i].gp = ~0ull;
+    t[i].aux = 0ull;
+  }
+}
+
 inline int grid_for(glb_ctx* c, int per_sm = 8) { return c->num_sms * per_sm; }
 
 MarkArgs mark_args(glb_ctx* c, int count_mode) {
@@ -648,6 +761,16 @@ MarkArgs mark_args(glb_ctx* c, int count_mode) {
             : count_mode == GLB_COUNT_ACCESS  ? c->access
                                               : nullptr;
   return m;
+}
+
+Table table_of(glb_ctx* c) {
+  Table T;
+  T.e = c->hash_mode ? c->htab : c->vmap;
+  T.hslot = c->hslot;
+  T.slot = c->slot;
+  T.mask = c->hmask;
+  T.gen = c->gen;
+  return T;
 }
 
 }  // namespace
@@ -668,8 +791,13 @@ cudaError_t launch_seed_init(glb_ctx* c, const uint32_t* seeds, uint32_t n0, int
     za.p[l] = c->sb.status[l];
     za.n[l] = (uint32_t)c->sb.ntiles[l];
   }
-  const cudaError_t e = launch_pdl(k_seed_init, blocks, kThreads, c->stream, seeds, n0, c->V, c->st,
-                                   c->sb.uniq, c->vmap, c->gen, mark_args(c, count_mode), za);
+  const Table T = table_of(c);
+  const cudaError_t e =
+      c->hash_mode
+          ? launch_pdl_w(c->pin, k_seed_init<true>, blocks, kThreads, c->stream, seeds, n0, c->V, c->st,
+                       c->sb.uniq, T, mark_args(c, count_mode), za)
+          : launch_pdl_w(c->pin, k_seed_init<false>, blocks, kThreads, c->stream, seeds, n0, c->V, c->st,
+                       c->sb.uniq, T, mark_args(c, count_mode), za);
   count_launch(c);
   return e;
 }
@@ -683,13 +811,16 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
   const uint64_t* ip = c->indptr;
   const uint32_t* ix = c->indices;
   const uint32_t* uq = b.uniq;
+  const Table T = table_of(c);
   cudaError_t e;
+#define GLB_KH_ARGS hop, k, seed, epoch, batch, T, stc, c->st, ip, ix, uq, b.picks, b.pidx, fix
   if (k <= 32)
-    e = launch_pdl(k_khop, grid, kThreads, c->stream, hop, k, seed, epoch, batch, c->gen, stc,
-                   c->st, ip, ix, uq, c->vmap, b.picks, fix);
+    e = c->hash_mode ? launch_pdl_w(c->pin, k_khop<true>, grid, kThreads, c->stream, GLB_KH_ARGS)
+                     : launch_pdl_w(c->pin, k_khop<false>, grid, kThreads, c->stream, GLB_KH_ARGS);
   else
-    e = launch_pdl(k_khop_wide, grid, kThreads, c->stream, hop, k, seed, epoch, batch, c->gen, stc,
-                   c->st, ip, ix, uq, c->vmap, b.picks, fix);
+    e = c->hash_mode ? launch_pdl_w(c->pin, k_khop_wide<true>, grid, kThreads, c->stream, GLB_KH_ARGS)
+                     : launch_pdl_w(c->pin, k_khop_wide<false>, grid, kThreads, c->stream, GLB_KH_ARGS);
+#undef GLB_KH_ARGS
   count_launch(c);
   return e;
 }
@@ -697,19 +828,21 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
 cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch, uint32_t batch) {
   const int grid = grid_for(c);
   const SampleBufs& b = c->sb;
-#define GLB_RW_ARGS                                                                     \
-  hop, c->rw_walks, c->rw_len, c->rw_topk, seed, epoch, batch, c->gen, stc, c->st, ip, ix, uq, \
-      c->vmap, b.picks, b.pickw, fix
+#define GLB_RW_ARGS                                                                            \
+  hop, c->rw_walks, c->rw_len, c->rw_topk, seed, epoch, batch, T, stc, c->st, ip, ix, uq, b.picks, \
+      b.pickw, b.pidx, fix
   uint32_t* fix = hop ? b.bindices[hop - 1] : nullptr;
   const uint32_t w = c->rw_walks;
   const DevState* stc = c->st;
   const uint64_t* ip = c->indptr;
   const uint32_t* ix = c->indices;
   const uint32_t* uq = b.uniq;
+  const Table T = table_of(c);
   cudaError_t e;
-#define GLB_RW_G(GG)                                                                    \
-  (c->rw_len <= 3 ? launch_pdl(k_rwalk<GG, 3>, grid, kThreads, c->stream, GLB_RW_ARGS) \
-                  : launch_pdl(k_rwalk<GG, kMaxWalkLen>, grid, kThreads, c->stream, GLB_RW_ARGS))
+#define GLB_RW_L(GG, LL)                                                                       \
+  (c->hash_mode ? launch_pdl_w(c->pin, k_rwalk<GG, LL, true>, grid, kThreads, c->stream, GLB_RW_ARGS)  \
+                : launch_pdl_w(c->pin, k_rwalk<GG, LL, false>, grid, kThreads, c->stream, GLB_RW_ARGS))
+#define GLB_RW_G(GG) (c->rw_len <= 3 ? GLB_RW_L(GG, 3) : GLB_RW_L(GG, kMaxWalkLen))
   if (w <= 1) e = GLB_RW_G(1);
   else if (w <= 2) e = GLB_RW_G(2);
   else if (w <= 4) e = GLB_RW_G(4);
@@ -717,6 +850,7 @@ cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch
   else if (w <= 16) e = GLB_RW_G(16);
   else e = GLB_RW_G(32);
 #undef GLB_RW_G
+#undef GLB_RW_L
 #undef GLB_RW_ARGS
   count_launch(c);
   return e;
@@ -724,8 +858,8 @@ cudaError_t launch_rwalk(glb_ctx* c, uint32_t hop, uint64_t seed, uint32_t epoch
 
 cudaError_t launch_fixup(glb_ctx* c, uint32_t hop) {
   const DevState* stc = c->st;
-  const VEntry* vm = c->vmap;
-  const cudaError_t e = launch_pdl(k_fixup, grid_for(c), kThreads, c->stream, hop, stc, vm,
+  const VEntry* vm = table_of(c).e;
+  const cudaError_t e = launch_pdl_w(c->pin, k_fixup, grid_for(c), kThreads, c->stream, hop, stc, vm,
                                    c->sb.bindices[hop]);
   count_launch(c);
   return e;
@@ -736,18 +870,32 @@ cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, 
   const int grid = grid_for(c, 3);
   const uint32_t* pk = b.picks;
   const uint32_t* pw = b.pickw;
+  const uint32_t* pi = b.pidx;
   const uint32_t nsm = (uint32_t)c->num_sms;
+  const Table T = table_of(c);
+  const MarkArgs mk = mark_args(c, count_mode);
   cudaError_t e;
+#define GLB_CP_ARGS(W)                                                                          \
+  hop, k, T, c->st, pk, pw, pi, b.uniq, b.bindptr[hop], b.bindices[hop],                        \
+      (W) ? b.bweights[hop] : (uint32_t*)nullptr, b.status[hop], mk, nsm
   if (weighted)
-    e = launch_pdl(k_compact<true>, grid, kThreads, c->stream, hop, k, c->gen, c->st, pk, pw,
-                   c->vmap, b.uniq, b.bindptr[hop], b.bindices[hop], b.bweights[hop],
-                   b.status[hop], mark_args(c, count_mode), nsm);
+    e = c->hash_mode ? launch_pdl_w(c->pin, k_compact<true, true>, grid, kThreads, c->stream, GLB_CP_ARGS(1))
+                     : launch_pdl_w(c->pin, k_compact<true, false>, grid, kThreads, c->stream, GLB_CP_ARGS(1));
   else
-    e = launch_pdl(k_compact<false>, grid, kThreads, c->stream, hop, k, c->gen, c->st, pk,
-                   (const uint32_t*)nullptr, c->vmap, b.uniq, b.bindptr[hop], b.bindices[hop],
-                   (uint32_t*)nullptr, b.status[hop], mark_args(c, count_mode), nsm);
+    e = c->hash_mode ? launch_pdl_w(c->pin, k_compact<false, true>, grid, kThreads, c->stream, GLB_CP_ARGS(0))
+                     : launch_pdl_w(c->pin, k_compact<false, false>, grid, kThreads, c->stream, GLB_CP_ARGS(0));
+#undef GLB_CP_ARGS
   count_launch(c);
   return e;
+}
+
+cudaError_t launch_table_reset(glb_ctx* c) {
+  if (c->hash_mode && c->htab) {
+    const uint64_t n = (uint64_t)c->hmask + 1;
+    k_table_reset<<<grid_for(c), kThreads, 0, c->stream>>>(c->htab, n);
+    count_launch(c);
+  }
+  return cudaGetLastError();
 }
 
 }  // namespace glb

@@ -31,11 +31,17 @@ def assert_same_sample(gs, os_, weighted=False):
             assert np.array_equal(u32(gs.weights[l]), os_.weights[l]), f"weights hop {l}"
 
 
-def make_ctx(g, kind="khop", fanouts=(10, 5), max_batch=None, layers=None):
+MODES = ["dense", "hash"]
+
+
+def make_ctx(g, kind="khop", fanouts=(10, 5), max_batch=None, layers=None, mode="auto"):
     ctx = glb.Context(0)
     ctx.load_graph(g.indptr, g.indices, g.features)
+    ctx.set_relabel_mode(mode)
     ctx.set_sampler(kind, fanouts=fanouts, layers=layers,
                     max_batch=max_batch or g.shape.batch)
+    if mode != "auto":
+        assert ctx.relabel_mode == mode
     ctx.set_train_set(g.train, g.shape.batch, g.seed)
     return ctx
 
@@ -78,10 +84,11 @@ def test_worked_example_on_gpu():
     assert ctx.permutation(8).tolist() == gold["shuffle"]["epoch1"]
 
 
-def test_tiny_every_batch_bit_exact(tiny):
+@pytest.mark.parametrize("mode", MODES)
+def test_tiny_every_batch_bit_exact(tiny, mode):
     g, go = tiny
     sh = g.shape
-    ctx = make_ctx(g, fanouts=sh.fanouts)
+    ctx = make_ctx(g, fanouts=sh.fanouts, mode=mode)
     for e in [0, 1]:
         ob = oracle.epoch_batches(g.train, sh.batch, g.seed, e)
         ctx.shuffle(e)
@@ -105,10 +112,11 @@ def test_host_and_device_seed_paths(tiny):
 
 
 @pytest.mark.parametrize("fanouts", [(25, 10), (15, 10, 5), (3,), (1, 1, 1), (32, 2), (40, 33)])
-def test_fanout_variants_power_law(fanouts):
+@pytest.mark.parametrize("mode", MODES)
+def test_fanout_variants_power_law(fanouts, mode):
     g = synth.small_graph(6000, 90000, 2.1, 8, 700, seed=11)
     go = oracle.GraphOracle(g.indptr, g.indices)
-    ctx = make_ctx(g, fanouts=fanouts, max_batch=300)
+    ctx = make_ctx(g, fanouts=fanouts, max_batch=300, mode=mode)
     for b, n0 in enumerate([1, 37, 300]):
         seeds = g.train[b * 200:b * 200 + n0]
         assert_same_sample(ctx.sample(seeds, seed=5, epoch=b, batch=b),
@@ -132,9 +140,10 @@ def test_empty_batch_zero_hops_and_degree_zero():
     assert s.sizes == [2] and u32(s.uniq).tolist() == [2, 1]
 
 
-def test_errors():
+@pytest.mark.parametrize("mode", MODES)
+def test_errors(mode):
     g = synth.small_graph(500, 3000, 2.2, 4, 50, seed=8)
-    ctx = make_ctx(g, fanouts=(3, 2), max_batch=16)
+    ctx = make_ctx(g, fanouts=(3, 2), max_batch=16, mode=mode)
     with pytest.raises(glb.GlbError) as e:
         ctx.sample(np.array([1, 2, 1], np.uint32))
     assert e.value.code == glb.EINVAL
@@ -165,11 +174,13 @@ def test_errors():
 
 @pytest.mark.parametrize("layers,walks,length,topk", [(3, 4, 3, 5), (2, 4, 3, 5), (1, 2, 5, 3),
                                                       (2, 8, 2, 7)])
-def test_random_walk_parity(layers, walks, length, topk):
+@pytest.mark.parametrize("mode", MODES)
+def test_random_walk_parity(layers, walks, length, topk, mode):
     g = synth.small_graph(8000, 60000, 2.5, 8, 600, seed=21)
     go = oracle.GraphOracle(g.indptr, g.indices)
     ctx = glb.Context(0)
     ctx.load_graph(g.indptr, g.indices, None)
+    ctx.set_relabel_mode(mode)
     ctx.set_sampler("rwalk", layers=layers, walks=walks, walk_len=length, topk=topk, max_batch=200)
     for b, n0 in enumerate([1, 64, 200]):
         seeds = g.train[b * 200:b * 200 + n0]
@@ -178,10 +189,11 @@ def test_random_walk_parity(layers, walks, length, topk):
         assert_same_sample(gs, os_, weighted=True)
 
 
-def test_presample_cache_and_hit_stats(tiny):
+@pytest.mark.parametrize("mode", MODES)
+def test_presample_cache_and_hit_stats(tiny, mode):
     g, go = tiny
     sh = g.shape
-    ctx = make_ctx(g, fanouts=sh.fanouts)
+    ctx = make_ctx(g, fanouts=sh.fanouts, mode=mode)
     for K in [1, 2]:
         ctx.reset_counts(glb.COUNT_PRESAMPLE)
         ctx.presample(K)
@@ -212,11 +224,12 @@ def test_presample_cache_and_hit_stats(tiny):
         assert hs["hits"] <= hs["optimal_hits"]
 
 
+@pytest.mark.parametrize("mode", MODES)
 @pytest.mark.parametrize("alpha", [0.0, 0.1, 0.5, 1.0])
-def test_extract_sample_bytes(tiny, alpha):
+def test_extract_sample_bytes(tiny, alpha, mode):
     g, go = tiny
     sh = g.shape
-    ctx = make_ctx(g, fanouts=sh.fanouts)
+    ctx = make_ctx(g, fanouts=sh.fanouts, mode=mode)
     ctx.presample(1)
     ctx.build_cache(alpha)
     slot = ctx.cache_slots()
@@ -304,12 +317,13 @@ def test_pr_full_size_parity(pr):
 
 
 @pytest.mark.parametrize("alpha", [1.0, 0.3])
-def test_pipeline_depth2_bit_exact(tiny, alpha):
+@pytest.mark.parametrize("mode", MODES)
+def test_pipeline_depth2_bit_exact(tiny, alpha, mode):
     """Pipelined Extract || Sample (two streams, double-buffered slots) gives the
     same bytes as the oracle for every batch of an epoch."""
     g, go = tiny
     sh = g.shape
-    ctx = make_ctx(g, fanouts=sh.fanouts)
+    ctx = make_ctx(g, fanouts=sh.fanouts, mode=mode)
     ctx.presample(1)
     ctx.build_cache(alpha)
     ctx.set_pipeline(2)
