@@ -54,6 +54,8 @@ def parse():
                    help="gloo: CPU-staged send/recv (lets N ranks share one GPU for testing)")
     p.add_argument("--relabel", default="auto", choices=["auto", "dense", "hash"],
                    help="relabel table (glb_set_relabel_mode)")
+    p.add_argument("--host-alloc", default="register", choices=["register", "cuda"],
+                   help="host feature memory: pageable + cudaHostRegister, or cudaHostAlloc")
     p.add_argument("--pipeline", type=int, default=1, choices=[1, 2],
                    help="2: extract of batch b overlaps sampling of batch b+1 (two streams)")
     return p.parse_args()
@@ -325,7 +327,11 @@ def main():
     sh = synth.SHAPES[args.config]
 
     t0 = time.perf_counter()
-    g = synth.make_graph(sh)
+    alloc = None
+    if args.host_alloc == "cuda":
+        def alloc(nbytes):  # cudaHostAlloc'ed (pinned, mapped under UVA) via torch
+            return torch.empty(nbytes, dtype=torch.uint8, pin_memory=True).numpy()
+    g = synth.make_graph(sh, feature_alloc=alloc)
     t_gen = time.perf_counter() - t0
 
     ctx = glb.Context(local)

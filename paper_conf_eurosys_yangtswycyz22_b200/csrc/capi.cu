@@ -214,6 +214,8 @@ glb_status glb_create(int device, glb_ctx** out) {
       (e = cudaMalloc(&c->st_x, sizeof(DevState))) != cudaSuccess ||
       (e = cudaMalloc(&c->scratch, 4 * sizeof(unsigned long long))) != cudaSuccess ||
       (e = cudaMalloc(&c->xcount, 2 * sizeof(unsigned long long))) != cudaSuccess ||
+      (e = cudaMalloc(&c->work, 8 * sizeof(unsigned int))) != cudaSuccess ||
+      (e = cudaMemset(c->work, 0, 8 * sizeof(unsigned int))) != cudaSuccess ||
       (e = cudaMallocHost(&c->h_st, sizeof(DevState))) != cudaSuccess ||
       (e = cudaMallocHost(&c->h_xcount, 2 * sizeof(unsigned long long))) != cudaSuccess ||
       (e = cudaMemset(c->sts[0], 0, sizeof(DevState))) != cudaSuccess ||
@@ -241,6 +243,7 @@ glb_status glb_destroy(glb_ctx* c) {
   dfree(c->xb.hit_list); dfree(c->xb.miss_list);
   dfree(c->train); dfree(c->perm); dfree(c->shuf_keys); dfree(c->shuf_vals);
   dfree(c->sts[0]); dfree(c->sts[1]); dfree(c->st_x); dfree(c->scratch); dfree(c->xcount);
+  dfree(c->work);
   for (int i = 0; i < 2; ++i) {
     if (c->ev_sampled[i]) cudaEventDestroy(c->ev_sampled[i]);
     if (c->ev_extracted[i]) cudaEventDestroy(c->ev_extracted[i]);
@@ -305,7 +308,13 @@ glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* in
   }
   if (features) {
     const size_t bytes = (size_t)V * D * sizeof(float);
-    cudaError_t e = cudaHostRegister((void*)features, bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+    cudaPointerAttributes pa;
+    const bool pinned = cudaPointerGetAttributes(&pa, features) == cudaSuccess &&
+                        pa.type == cudaMemoryTypeHost;  // e.g. cudaHostAlloc'ed by the caller
+    (void)cudaGetLastError();
+    cudaError_t e = pinned ? cudaErrorHostMemoryAlreadyRegistered
+                           : cudaHostRegister((void*)features, bytes,
+                                              cudaHostRegisterMapped | cudaHostRegisterPortable);
     if (e == cudaErrorHostMemoryAlreadyRegistered) {
       (void)cudaGetLastError();
       c->registered = false;

@@ -73,48 +73,59 @@ template <typename T>
 __device__ __forceinline__ void st_row(T* p, T v) { __stcs(p, v); }
 
 // T = float4 (row bytes % 16 == 0) or float.  U = T-units per row.
+// Work: hit chunks first (HBM, fast), then miss chunks (host, PCIe); chunks are
+// handed out by two device counters, so every block works on hits while there
+// are any and then every block keeps PCIe requests in flight.
 template <typename T>
 __global__ void __launch_bounds__(kThreads, 4)
     k_gather(T* __restrict__ out, const T* __restrict__ src_hit, const T* __restrict__ src_miss,
              const uint2* __restrict__ hit_list, const uint2* __restrict__ miss_list,
              const uint32_t* __restrict__ fill_src, const uint32_t* __restrict__ dev_counts,
              uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t R,
-             unsigned long long* xcount) {
+             unsigned long long* xcount, unsigned int* work) {
   pdl_enter();
   __shared__ uint2 ent[2][kThreads];
+  __shared__ unsigned int s_next;
   const uint64_t nh = dev_counts ? dev_counts[0] : nh_host;
   const uint64_t nm = dev_counts ? dev_counts[1] : nm_host;
-  const uint32_t G = gridDim.x;
-  uint32_t miss_blocks = 0;
-  if (nm) miss_blocks = nh ? max(1u, G / 4) : G;
-  const bool is_miss = blockIdx.x >= G - miss_blocks;
-  const uint32_t rb = is_miss ? blockIdx.x - (G - miss_blocks) : blockIdx.x;
-  const uint32_t nrb = is_miss ? miss_blocks : G - miss_blocks;
-  const uint64_t n = is_miss ? nm : nh;
-  const uint2* list = is_miss ? miss_list : hit_list;
-  const uint32_t* fsrc = is_miss ? fill_src : nullptr;
-  const T* src = is_miss ? src_miss : src_hit;
   if (xcount && blockIdx.x == 0 && threadIdx.x == 0) {
     xcount[0] = nh;
     xcount[1] = nm;
   }
-  if (n == 0) return;
   const uint32_t t = threadIdx.x;
-  const uint64_t nchunks = (n + R - 1) / R;
+  const uint64_t nch = (nh + R - 1) / R, ncm = (nm + R - 1) / R;  // hit / miss chunks
   const float inv_u = 1.0f / (float)U;
-  auto load_ent = [&](uint64_t chunk) -> uint2 {
-    const uint64_t r = chunk * R + t;
-    if (t < R && chunk < nchunks && r < n)
-      return fsrc ? make_uint2((uint32_t)r, __ldg(fsrc + r)) : __ldg(list + r);
-    return make_uint2(0u, 0u);
-  };
-  uint2 e = load_ent(rb);
-  int buf = 0;
-  for (uint64_t c = rb; c < nchunks; c += nrb) {
-    if (t < R) ent[buf][t] = e;
+  // chunk id g: g < nch -> hit chunk g; else miss chunk g - nch
+  auto claim = [&]() -> uint64_t {
+    if (t == 0) {
+      unsigned int g = atomicAdd(&work[0], 1u);
+      if (g >= nch) g = (unsigned int)nch + atomicAdd(&work[1], 1u);
+      s_next = g;
+    }
     __syncthreads();
-    e = load_ent(c + nrb);  // prefetch the next chunk's entries
-    const uint64_t rows = min((uint64_t)R, n - c * R);
+    const uint64_t g = s_next;
+    __syncthreads();
+    return g;
+  };
+  auto load_ent = [&](uint64_t g) -> uint2 {
+    if (g >= nch + ncm || t >= R) return make_uint2(0u, 0u);
+    const bool miss = g >= nch;
+    const uint64_t r = (miss ? g - nch : g) * R + t;
+    if (r >= (miss ? nm : nh)) return make_uint2(0u, 0u);
+    if (!miss) return __ldg(hit_list + r);
+    return fill_src ? make_uint2((uint32_t)r, __ldg(fill_src + r)) : __ldg(miss_list + r);
+  };
+  uint64_t g = claim();
+  uint2 e = load_ent(g);
+  int buf = 0;
+  while (g < nch + ncm) {
+    if (t < R) ent[buf][t] = e;
+    const uint64_t gn = claim();  // (its barrier also publishes ent[buf])
+    e = load_ent(gn);             // prefetch the next chunk's entries
+    const bool miss = g >= nch;
+    const T* src = miss ? src_miss : src_hit;
+    const uint64_t c = miss ? g - nch : g;
+    const uint64_t rows = min((uint64_t)R, (miss ? nm : nh) - c * R);
     const uint32_t total = (uint32_t)rows * U;
     for (uint32_t base = 0; base < total; base += kChunkUnits) {
       T x[kVecPerThread];
@@ -137,6 +148,16 @@ __global__ void __launch_bounds__(kThreads, 4)
       }
     }
     buf ^= 1;
+    g = gn;
+  }
+  // the last block out re-arms the counters for the next launch on this stream
+  if (t == 0) {
+    __threadfence();
+    if (atomicAdd(&work[2], 1u) == gridDim.x - 1) {
+      work[0] = 0u;
+      work[1] = 0u;
+      work[2] = 0u;
+    }
   }
 }
 
@@ -162,14 +183,17 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   if (R > (uint32_t)kThreads) R = kThreads;
   if (R < 1) R = 1;
   const int grid = c->num_sms * c->gather_bps;
+  // chunk counters of the launching stream (this ctx's gathers are serial on it; each
+  // launch leaves them zeroed for the next)
+  unsigned int* work = c->stream == c->xstream ? c->work + 4 : c->work;
   cudaError_t e;
   if (vec)
     e = launch_pdl(k_gather<float4>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount);
+                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work);
   else
     e = launch_pdl(k_gather<float>, grid, kThreads, c->stream, out, src_hit, src_miss, hit_list,
-                   miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R, c->xcount);
+                   miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work);
   count_launch(c);
   return e;
 }

@@ -175,6 +175,7 @@ struct glb_ctx {
   cudaEvent_t ev_sampled[2] = {nullptr, nullptr};
   cudaEvent_t ev_extracted[2] = {nullptr, nullptr};
   int gather_bps = 4;            // gather blocks per SM
+  unsigned int* work = nullptr;  // device [8]: gather chunk counters (main, extract stream)
   bool timing = false;           // record per-extract kernel events
   std::vector<cudaEvent_t> tev;  // pairs (start, end) of recorded extracts
   size_t tev_used = 0;

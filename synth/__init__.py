@@ -142,8 +142,13 @@ def gen_topology(V: int, E: int, gamma_out: float, gamma_in: float, seed: int, c
     return indptr, indices
 
 
-def gen_features(V: int, D: int, seed: int, threads: int = 0) -> np.ndarray:
-    f = aligned_empty(V * D, np.float32).reshape(V, D)
+def gen_features(V: int, D: int, seed: int, threads: int = 0, alloc=None) -> np.ndarray:
+    """alloc(nbytes) -> writable uint8 numpy buffer (e.g. CUDA pinned memory); default:
+    2 MB-aligned pageable memory that glb_load_graph registers."""
+    if alloc is None:
+        f = aligned_empty(V * D, np.float32).reshape(V, D)
+    else:
+        f = alloc(V * D * 4).view(np.float32)[:V * D].reshape(V, D)
     lib().synth_features(V, D, seed, f.ctypes.data, threads)
     return f
 
@@ -157,7 +162,7 @@ def gen_trainset(V: int, n: int, seed: int) -> np.ndarray:
 
 
 def make_graph(shape: Shape | str, seed: int | None = None, features: bool = True,
-               threads: int = 0) -> Graph:
+               threads: int = 0, feature_alloc=None) -> Graph:
     if isinstance(shape, str):
         shape = SHAPES[shape]
     seed = seed_for(shape) if seed is None else seed
@@ -165,7 +170,7 @@ def make_graph(shape: Shape | str, seed: int | None = None, features: bool = Tru
     indptr, indices = gen_topology(shape.V, shape.E, shape.gamma_out, shape.gamma_in, seed, cap,
                                    threads)
     train = gen_trainset(shape.V, shape.n_train, seed)
-    feats = gen_features(shape.V, shape.D, seed, threads) if features else None
+    feats = gen_features(shape.V, shape.D, seed, threads, feature_alloc) if features else None
     return Graph(shape, seed, indptr, indices, train, feats)
 
 
