@@ -68,7 +68,7 @@ void free_sample_bufs(glb_ctx* c) {
     for (int l = 0; l < GLB_MAX_HOPS; ++l) {
       dfree(b.bindptr[l]); dfree(b.bindices[l]); dfree(b.bweights[l]); dfree(b.status[l]);
     }
-    dfree(b.hit_list); dfree(b.miss_list);
+    dfree(b.hit_list); dfree(b.miss_list); dfree(b.miss_sorted);
     b = SampleBufs();
   }
   c->sb = SampleBufs();
@@ -240,7 +240,8 @@ glb_status glb_destroy(glb_ctx* c) {
   if (c->xstream) cudaStreamSynchronize(c->xstream);
   free_sample_bufs(c);
   free_graph(c);
-  dfree(c->xb.hit_list); dfree(c->xb.miss_list);
+  dfree(c->xb.hit_list); dfree(c->xb.miss_list); dfree(c->xb.miss_sorted);
+  dfree(c->miss_bins);
   dfree(c->train); dfree(c->perm); dfree(c->shuf_keys); dfree(c->shuf_vals);
   dfree(c->sts[0]); dfree(c->sts[1]); dfree(c->st_x); dfree(c->scratch); dfree(c->xcount);
   dfree(c->work);
@@ -330,6 +331,11 @@ glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* in
     c->h_features = features;
     c->features_mapped = (const float*)dp;
     c->D = D;
+    uint32_t shift = 0;
+    while ((4ull * D << (shift + 1)) <= (2ull << 20)) ++shift;
+    dfree(c->miss_bins);
+    c->miss_bins_cap = (uint32_t)((V >> shift) + 1);
+    CK(dalloc(&c->miss_bins, c->miss_bins_cap));
   }
   return GLB_OK;
 }
@@ -422,6 +428,7 @@ glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32
     }
     CK(dalloc(&bs.hit_list, un));
     CK(dalloc(&bs.miss_list, un));
+    CK(dalloc(&bs.miss_sorted, un));
   }
   use_slot(c, 0);
   c->kind = kind;
@@ -701,15 +708,21 @@ glb_status glb_extract(glb_ctx* c, const uint32_t* vertices, uint64_t n, void* o
   if (n >= 0xFFFFFFFFull) return set_err(c, GLB_EINVAL, "n too large");
   if (n > c->xb.cap) {
     CK(cudaStreamSynchronize(c->stream));
-    dfree(c->xb.hit_list); dfree(c->xb.miss_list);
+    dfree(c->xb.hit_list); dfree(c->xb.miss_list); dfree(c->xb.miss_sorted);
     c->xb.cap = 0;
     CK(dalloc(&c->xb.hit_list, n));
     CK(dalloc(&c->xb.miss_list, n));
+    CK(dalloc(&c->xb.miss_sorted, n));
     c->xb.cap = n;
   }
   CK(cudaMemsetAsync(&c->st_x->nhit, 0, 2 * sizeof(uint32_t), c->stream));
   if (n) CK(launch_mark(c, vertices, n));
-  CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->xb.hit_list, c->xb.miss_list,
+  const uint2* misses = c->xb.miss_list;
+  if (n && c->C < c->V) {  // some rows may come over PCIe: order them by host page
+    CK(launch_sort_misses(c, c->xb.miss_list, &c->st_x->nmiss, c->xb.miss_sorted));
+    misses = c->xb.miss_sorted;
+  }
+  CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->xb.hit_list, misses,
                    nullptr, &c->st_x->nhit, 0, 0));
   if (stats) {
     CK(cudaMemcpyAsync(c->h_xcount, c->xcount, 2 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
@@ -747,8 +760,15 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
     c->tev_used += 2;
     cudaEventRecord(t0, c->stream);
   }
-  cudaError_t e = launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_list,
-                                c->sb.miss_list, nullptr, &c->st->nhit, 0, 0);
+  const uint2* misses = c->sb.miss_list;
+  cudaError_t e = cudaSuccess;
+  if (c->C < c->V) {  // some rows may come over PCIe: order them by host page
+    e = launch_sort_misses(c, c->sb.miss_list, &c->st->nmiss, c->sb.miss_sorted);
+    misses = c->sb.miss_sorted;
+  }
+  if (e == cudaSuccess)
+    e = launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_list, misses,
+                      nullptr, &c->st->nhit, 0, 0);
   if (e == cudaSuccess && t1) e = cudaEventRecord(t1, c->stream);
   if (e == cudaSuccess && stats) {
     e = cudaMemcpyAsync(c->h_xcount, c->xcount, 2 * sizeof(unsigned long long),

@@ -113,12 +113,14 @@ struct SampleBufs {
   uint64_t ntiles[GLB_MAX_HOPS] = {};
   uint2* hit_list = nullptr;          // extract work lists: (dst row, cache slot)
   uint2* miss_list = nullptr;         //                     (dst row, gid)
+  uint2* miss_sorted = nullptr;       // miss_list ordered by host page
 };
 
 struct ExtractBufs {
   uint64_t cap = 0;
   uint2* hit_list = nullptr;
   uint2* miss_list = nullptr;
+  uint2* miss_sorted = nullptr;
 };
 
 }  // namespace glb
@@ -176,6 +178,8 @@ struct glb_ctx {
   cudaEvent_t ev_extracted[2] = {nullptr, nullptr};
   int gather_bps = 4;            // gather blocks per SM
   unsigned int* work = nullptr;  // device [8]: gather chunk counters (main, extract stream)
+  unsigned int* miss_bins = nullptr;  // [miss_bins_cap] host-page histogram of misses
+  uint32_t miss_bins_cap = 0;
   bool timing = false;           // record per-extract kernel events
   std::vector<cudaEvent_t> tev;  // pairs (start, end) of recorded extracts
   size_t tev_used = 0;
@@ -273,6 +277,8 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
                           const uint2* hit_list, const uint2* miss_list, const uint32_t* fill_src,
                           const uint32_t* dev_counts /* [nhit, nmiss] on device or null */,
                           uint64_t nhit_host, uint64_t nmiss_host);
+cudaError_t launch_sort_misses(glb_ctx* c, const uint2* miss, const uint32_t* nmiss_dev,
+                               uint2* sorted);
 cudaError_t launch_shuffle_keys(glb_ctx* c, uint32_t epoch, unsigned long long* keys, uint32_t* vals);
 cudaError_t radix_sort_pairs_u64(glb_ctx* c, unsigned long long* keys, uint32_t* vals,
                                  unsigned long long* keys_alt, uint32_t* vals_alt, uint64_t n,
