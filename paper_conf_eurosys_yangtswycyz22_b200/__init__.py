@@ -76,11 +76,14 @@ def lib(auto_build: bool = True):
     global _lib
     if _lib is not None:
         return _lib
-    if auto_build:
-        build()
-    if not os.path.exists(_SO):
-        raise RuntimeError(f"{_SO} missing: run __graft_entry__.build()")
-    L = ctypes.CDLL(_SO)
+    so = os.environ.get("GLB_LIBRARY")  # A/B builds (tools/ab_build.sh)
+    if so is None:
+        if auto_build:
+            build()
+        so = _SO
+    if not os.path.exists(so):
+        raise RuntimeError(f"{so} missing: run __graft_entry__.build()")
+    L = ctypes.CDLL(so)
     vp, u32, u64, i32, dbl = (ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int,
                               ctypes.c_double)
     sig = {
