@@ -498,21 +498,38 @@ def main():
     # ---- hit rate vs Optimal (accesses recorded over measured epochs, untimed)
     result_hit = None
     sweep = []
+    similarity = None
     if not args.no_sweep:
-        ctx.reset_counts(glb.COUNT_ACCESS)
-        ctx.set_count_mode(glb.COUNT_ACCESS)
+        def reduce_counts(t):
+            if world > 1:
+                c = t if args.backend == "nccl" else t.cpu()
+                par.allreduce_counts(c)
+                if c is not t:
+                    t.copy_(c)
+            return t
+
+        # per-epoch access footprints of the measured epochs (Table 2 / Optimal, L148 fn4)
+        per_epoch = []
         for e in range(sh.K, sh.K + args.measure_epochs):
+            ctx.reset_counts(glb.COUNT_ACCESS)
+            ctx.set_count_mode(glb.COUNT_ACCESS)
             for b in range(rank, nb, world):
                 ctx.sample_batch(e, b)
-        ctx.set_count_mode(glb.COUNT_NONE)
-        ctx.sync()
-        if world > 1:
-            t_acc = ctx.counts_tensor(glb.COUNT_ACCESS)
-            c = t_acc if args.backend == "nccl" else t_acc.cpu()
-            par.allreduce_counts(c)
-            if c is not t_acc:
-                t_acc.copy_(c)
+            ctx.set_count_mode(glb.COUNT_NONE)
+            ctx.sync()
+            per_epoch.append(reduce_counts(ctx.counts_tensor(glb.COUNT_ACCESS)).clone())
+        ctx.counts_tensor(glb.COUNT_ACCESS).copy_(sum(per_epoch))
+        if len(per_epoch) >= 2:
+            v, num, den = ctx.footprint_similarity(per_epoch[0], per_epoch[1], 0.1)
+            similarity = {"epochs": [sh.K, sh.K + 1], "top_frac": 0.1, "value": v,
+                          "numerator": num, "denominator": den, "source": "Table 2 (L329)"}
         for a in sorted(set(sh.alphas) | {args.alpha}):
+            policies = {}
+            if 0.0 < a < 1.0:  # Fig 10 analog: Degree / Random vs PreSC vs Optimal
+                for pol in ("degree", "random"):
+                    ctx.build_cache_policy(a, pol, seed=g.seed)
+                    hs = ctx.hit_stats()
+                    policies[pol] = hs["hits"] / hs["total"] if hs["total"] else 0.0
             ctx.build_cache(a)
             hs = ctx.hit_stats()
             H = hs["hits"] / hs["total"] if hs["total"] else 0.0
@@ -534,6 +551,8 @@ def main():
             sweep.append({"alpha": a, "cache_rows": hs["cache_rows"], "hit_rate": H,
                           "optimal_hit_rate": Hs,
                           "presc_vs_optimal_pct": (100.0 * H / Hs) if Hs > 0 else None,
+                          "degree_hit_rate": policies.get("degree"),
+                          "random_hit_rate": policies.get("random"),
                           "seeds_per_s": sd * world / (ms / 1e3)})
             if a == args.alpha:
                 result_hit = sweep[-1]
@@ -572,6 +591,7 @@ def main():
             "clocks": clk,
             "hit_rate": result_hit,
             "alpha_sweep": sweep,
+            "footprint_similarity": similarity,
             "units": {"mean_n_L": statistics.mean(nL), "mean_hits": statistics.mean(hits),
                       "mean_misses": statistics.mean(misses)},
             "preprocess_s": {"generate_inputs": t_gen, "load_graph": t_load,

@@ -158,6 +158,22 @@ glb_status glb_get_counts(glb_ctx* ctx, int which, uint32_t* host_out /* V */);
  * the PreSC counts, else a device u32[V] hotness map (e.g. degree).  Synchronous. */
 glb_status glb_build_cache(glb_ctx* ctx, double alpha, const uint32_t* hotness);
 glb_status glb_get_cache_slots(glb_ctx* ctx, int32_t* host_out /* V */);
+
+/* Caching policies compared in the paper (L79, L301, L339-L343, Fig 10/12): fill a
+ * device u32[V] hotness map for glb_build_cache.  GLB_POLICY_PRESC copies the PreSC
+ * counts; GLB_POLICY_DEGREE = out-degree (PaGraph; saturated to 2^32-1);
+ * GLB_POLICY_RANDOM = hi32(draw64(v, 0, 0, c3(0,0,POLICY=7), 0)) under `seed`, a
+ * random order of the vertices.  hotness_out: device, caller-owned. */
+enum { GLB_POLICY_PRESC = 0, GLB_POLICY_DEGREE = 1, GLB_POLICY_RANDOM = 2 };
+glb_status glb_policy_hotness(glb_ctx* ctx, int policy, uint64_t seed, uint32_t* hotness_out);
+
+/* Footprint similarity of epoch i to epoch j (Table 2; reading Q16):
+ *   sum_{v in T_i and T_j} min(f_i(v), f_j(v)) / sum_{v in T_j} f_j(v),
+ * T_x = the floor(top_frac*V) vertices ranked first by (f_x desc, gid asc).
+ * f_i, f_j: device u32[V] per-epoch visit counts.  Exact integer sums (num, den)
+ * are returned; out = num/den (0 if den == 0).  Synchronous. */
+glb_status glb_footprint_similarity(glb_ctx* ctx, const uint32_t* f_i, const uint32_t* f_j,
+                                    double top_frac, uint64_t* num, uint64_t* den, double* out);
 glb_status glb_cache_size(const glb_ctx* ctx, uint64_t* out);
 
 /* Hit-rate statistics over the recorded accesses (GLB_COUNT_ACCESS) for the

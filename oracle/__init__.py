@@ -74,6 +74,8 @@ def lib():
         L.orc_sample_rwalk.restype = i32
         L.orc_extract.argtypes = [vp, u64, u32, vp, u64, vp]
         L.orc_extract.restype = i32
+        L.orc_policy_random.argtypes = [u64, u64, vp]
+        L.orc_policy_random.restype = None
         _lib = L
     return _lib
 
@@ -282,6 +284,35 @@ def cache_slots(counts: np.ndarray, alpha: float) -> np.ndarray:
     order = cache_rank(counts)
     slot[order[:C]] = np.arange(C, dtype=np.int32)
     return slot
+
+
+# ---------------------------------------------------------------- policies (Fig 10)
+def hotness_degree(indptr: np.ndarray) -> np.ndarray:
+    """Degree policy (PaGraph; L79, L301): h_v = out-degree."""
+    d = np.diff(indptr.astype(np.uint64))
+    return np.minimum(d, np.uint64(0xFFFFFFFF)).astype(np.uint32)
+
+
+def hotness_random(seed: int, V: int) -> np.ndarray:
+    """Random policy (L442): a uniformly random order, one draw per vertex."""
+    out = np.empty(V, np.uint32)
+    lib().orc_policy_random(seed, V, _p(out))
+    return out
+
+
+def footprint_similarity(f_i: np.ndarray, f_j: np.ndarray, top_frac: float = 0.1):
+    """Table 2 (L329, reading Q16): sum_{v in T_i & T_j} min(f_i, f_j) / sum_{v in T_j} f_j,
+    T_x = the floor(top_frac*V) vertices ranked first by (f_x desc, gid asc).
+    Returns (value, numerator, denominator)."""
+    C = cache_size(top_frac, f_i.shape[0])
+    ti = np.zeros(f_i.shape[0], bool)
+    tj = np.zeros(f_j.shape[0], bool)
+    ti[cache_rank(f_i)[:C]] = True
+    tj[cache_rank(f_j)[:C]] = True
+    both = ti & tj
+    num = int(np.minimum(f_i[both], f_j[both]).astype(np.uint64).sum())
+    den = int(f_j[tj].astype(np.uint64).sum())
+    return (num / den if den else 0.0), num, den
 
 
 # ---------------------------------------------------------------- metric

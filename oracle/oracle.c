@@ -289,6 +289,15 @@ int orc_sample_rwalk(const uint64_t* indptr, const uint32_t* indices, uint64_t V
 }
 
 /* ---------------------------------------------------------------------------
+ * Random caching policy (L442 §7.4 "Random"): each vertex's hotness is the high
+ * word of its own draw, domain POLICY = 7 -- a uniformly random order.
+ * ------------------------------------------------------------------------- */
+void orc_policy_random(uint64_t seed, uint64_t V, uint32_t* out) {
+  uint32_t c3 = orc_c3(0, 0, 7);
+  for (uint64_t v = 0; v < V; ++v) out[v] = (uint32_t)(orc_draw64(seed, (uint32_t)v, 0, 0, c3, 0) >> 32);
+}
+
+/* ---------------------------------------------------------------------------
  * a7: extract (L79, L241, L252).  A byte copy of each requested row; whether
  * a row comes from the GPU cache or from host memory does not change its
  * bytes, so the oracle reads every row from the feature matrix.

@@ -64,6 +64,9 @@ int orc_sample_rwalk(const uint64_t* indptr, const uint32_t* indices, uint64_t V
                      uint32_t* blk_indices, uint32_t* blk_weights, uint64_t indices_cap,
                      uint64_t* nnz);
 
+/* Random policy hotness (L442): hi32(draw64(v,0,0,c3(0,0,7),0)) for every vertex. */
+void orc_policy_random(uint64_t seed, uint64_t V, uint32_t* out);
+
 /* Extract (Fig 9): out[i,:] = features[vertices[i],:]. */
 int orc_extract(const float* features, uint64_t V, uint32_t D, const uint32_t* vertices,
                 uint64_t n, float* out);

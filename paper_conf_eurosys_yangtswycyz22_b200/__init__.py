@@ -21,6 +21,7 @@ import numpy as np
 from .build import SO as _SO, build  # noqa: F401
 
 KHOP, RWALK = 0, 1
+POLICY_PRESC, POLICY_DEGREE, POLICY_RANDOM = 0, 1, 2
 COUNT_NONE, COUNT_PRESAMPLE, COUNT_ACCESS = 0, 1, 2
 MAX_HOPS = 8
 OK, EINVAL, ENOMEM, ECUDA, ESTATE, ERANGE = 0, -1, -2, -3, -4, -5
@@ -35,7 +36,7 @@ EXPORTS = [
     "glb_get_counts", "glb_build_cache", "glb_get_cache_slots", "glb_cache_size",
     "glb_hit_stats_get", "glb_extract", "glb_extract_sample", "glb_kernel_launches",
     "glb_set_pipeline", "glb_extract_stream", "glb_set_timing", "glb_extract_times",
-    "glb_set_relabel_mode", "glb_relabel_mode",
+    "glb_set_relabel_mode", "glb_relabel_mode", "glb_policy_hotness", "glb_footprint_similarity",
 ]
 
 
@@ -119,6 +120,9 @@ def lib(auto_build: bool = True):
         "glb_extract_times": ([vp, vp, u64, ctypes.POINTER(u64)], i32),
         "glb_set_relabel_mode": ([vp, i32], i32),
         "glb_relabel_mode": ([vp, ctypes.POINTER(i32)], i32),
+        "glb_policy_hotness": ([vp, i32, u64, vp], i32),
+        "glb_footprint_similarity": ([vp, vp, vp, dbl, ctypes.POINTER(u64), ctypes.POINTER(u64),
+                                      ctypes.POINTER(dbl)], i32),
     }
     for name, (a, r) in sig.items():
         f = getattr(L, name)
@@ -335,6 +339,27 @@ class Context:
             assert hotness.is_cuda and hotness.numel() == self.V and hotness.is_contiguous()
             hp = hotness.data_ptr()
         self._ck(self._lib.glb_build_cache(self._h, float(alpha), hp))
+
+    def policy_hotness(self, policy: str, seed: int = 0):
+        """Hotness map of a caching policy ('presc' | 'degree' | 'random'), CUDA int32 [V]
+        (u32 values), for build_cache (L79, L301, Fig 10)."""
+        import torch
+        pid = {"presc": POLICY_PRESC, "degree": POLICY_DEGREE, "random": POLICY_RANDOM}[policy]
+        out = torch.empty(self.V, dtype=torch.int32, device=self.device)
+        self._ck(self._lib.glb_policy_hotness(self._h, pid, seed, out.data_ptr()))
+        return out
+
+    def build_cache_policy(self, alpha: float, policy: str, seed: int = 0):
+        self.build_cache(alpha, hotness=self.policy_hotness(policy, seed))
+
+    def footprint_similarity(self, f_i, f_j, top_frac: float = 0.1):
+        """Table 2 (L329): similarity of epoch i's footprint to epoch j's; f_*: CUDA int32
+        [V] visit counts.  Returns (value, numerator, denominator) -- exact integers."""
+        num, den, out = ctypes.c_uint64(), ctypes.c_uint64(), ctypes.c_double()
+        self._ck(self._lib.glb_footprint_similarity(self._h, f_i.data_ptr(), f_j.data_ptr(),
+                                                    float(top_frac), ctypes.byref(num),
+                                                    ctypes.byref(den), ctypes.byref(out)))
+        return out.value, num.value, den.value
 
     def cache_slots(self) -> np.ndarray:
         out = np.empty(self.V, np.int32)

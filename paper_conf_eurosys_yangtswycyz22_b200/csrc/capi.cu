@@ -613,6 +613,25 @@ glb_status glb_get_counts(glb_ctx* c, int which, uint32_t* host_out) {
   return GLB_OK;
 }
 
+// Order all vertices by (hotness desc, gid asc) (reading Q10): a stable LSD radix sort
+// of maxc - h over gid order.  tmp: device u32[4V]; returns the order (inside tmp).
+static glb_status rank_vertices(glb_ctx* c, const uint32_t* hot, uint32_t* tmp, uint32_t** order_out) {
+  const uint64_t V = c->V;
+  uint32_t *k0 = tmp, *v0 = tmp + V, *k1 = tmp + 2 * V, *v1 = tmp + 3 * V;
+  uint32_t* dmax = (uint32_t*)c->scratch;
+  CK(cudaMemsetAsync(dmax, 0, sizeof(uint32_t), c->stream));
+  CK(launch_max_u32(c, hot, V, dmax));
+  uint32_t maxc = 0;
+  CK(cudaMemcpyAsync(&maxc, dmax, sizeof(uint32_t), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  int bits = 0;
+  while (bits < 32 && (maxc >> bits)) ++bits;
+  CK(launch_rank_keys(c, hot, maxc, k0, v0));
+  uint32_t* ko = nullptr;
+  CK(radix_sort_pairs_u32(c, k0, v0, k1, v1, V, bits, &ko, order_out));
+  return GLB_OK;
+}
+
 glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
   ENTER(c);
   if (!c->V) return set_err(c, GLB_ESTATE, "build_cache before load_graph");
@@ -624,18 +643,9 @@ glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
   CK(sync_all(c));  // an in-flight extract may still read the old cache
   uint32_t* tmp = nullptr;
   CK(dalloc(&tmp, 4 * V));
-  uint32_t *k0 = tmp, *v0 = tmp + V, *k1 = tmp + 2 * V, *v1 = tmp + 3 * V;
-  uint32_t* dmax = (uint32_t*)c->scratch;
-  CK(cudaMemsetAsync(dmax, 0, sizeof(uint32_t), c->stream));
-  CK(launch_max_u32(c, hot, V, dmax));
-  uint32_t maxc = 0;
-  CK(cudaMemcpyAsync(&maxc, dmax, sizeof(uint32_t), cudaMemcpyDeviceToHost, c->stream));
-  CK(cudaStreamSynchronize(c->stream));
-  int bits = 0;
-  while (bits < 32 && (maxc >> bits)) ++bits;
-  CK(launch_rank_keys(c, hot, maxc, k0, v0));
-  uint32_t *ko = nullptr, *order = nullptr;
-  CK(radix_sort_pairs_u32(c, k0, v0, k1, v1, V, bits, &ko, &order));
+  uint32_t* order = nullptr;
+  glb_status s = rank_vertices(c, hot, tmp, &order);
+  if (s != GLB_OK) { cudaFree(tmp); return s; }
   CK(cudaMemsetAsync(c->slot, 0xFF, sizeof(int32_t) * V, c->stream));
   CK(launch_assign_slots(c, order, C));
   CK(launch_vmap_reset(c));  // dense mode: copy the slots into the relabel entries
@@ -650,6 +660,47 @@ glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
   CK(cudaStreamSynchronize(c->stream));
   cudaFree(tmp);
   c->have_sample = false;  // marks of an earlier sample refer to the old cache
+  return GLB_OK;
+}
+
+glb_status glb_policy_hotness(glb_ctx* c, int policy, uint64_t seed, uint32_t* out) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "no graph");
+  if (!out) return set_err(c, GLB_EINVAL, "null out");
+  if (policy < GLB_POLICY_PRESC || policy > GLB_POLICY_RANDOM) return set_err(c, GLB_EINVAL, "bad policy");
+  CK(launch_policy_hotness(c, policy, seed, out));
+  return GLB_OK;
+}
+
+glb_status glb_footprint_similarity(glb_ctx* c, const uint32_t* fi, const uint32_t* fj,
+                                    double top_frac, uint64_t* num, uint64_t* den, double* out) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "no graph");
+  if (!fi || !fj) return set_err(c, GLB_EINVAL, "null counts");
+  if (!(top_frac >= 0.0 && top_frac <= 1.0)) return set_err(c, GLB_EINVAL, "top_frac not in [0,1]");
+  const uint64_t V = c->V;
+  const uint64_t C = (uint64_t)std::floor(top_frac * (double)V);
+  uint32_t* tmp = nullptr;
+  uint8_t* flags = nullptr;
+  CK(dalloc(&tmp, 4 * V));
+  CK(dalloc(&flags, 2 * V));
+  CK(cudaMemsetAsync(flags, 0, 2 * V, c->stream));
+  for (int x = 0; x < 2; ++x) {
+    uint32_t* order = nullptr;
+    glb_status s = rank_vertices(c, x == 0 ? fi : fj, tmp, &order);
+    if (s != GLB_OK) { cudaFree(tmp); cudaFree(flags); return s; }
+    CK(launch_topmark(c, order, C, flags + x * V));
+  }
+  CK(cudaMemsetAsync(c->scratch, 0, 2 * sizeof(unsigned long long), c->stream));
+  CK(launch_similarity(c, fi, fj, flags, flags + V, c->scratch));
+  unsigned long long h2[2];
+  CK(cudaMemcpyAsync(h2, c->scratch, sizeof(h2), cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  cudaFree(tmp);
+  cudaFree(flags);
+  if (num) *num = h2[0];
+  if (den) *den = h2[1];
+  if (out) *out = h2[1] ? (double)h2[0] / (double)h2[1] : 0.0;
   return GLB_OK;
 }
 

@@ -27,7 +27,7 @@ constexpr int kMaxFanout = 1024;
 constexpr int kMaxWalkLen = 8;
 
 // RNG domains (reading Q4): counter word 3 = epoch<<16 | hop<<8 | domain
-enum : uint32_t { kDomShuffle = 1, kDomKhop = 2, kDomRwalk = 3 };
+enum : uint32_t { kDomShuffle = 1, kDomKhop = 2, kDomRwalk = 3, kDomPolicy = 7 };
 
 // device error bits (DevState::err)
 enum : uint32_t { kErrDupSeed = 1u, kErrRange = 2u, kErrCapacity = 4u, kErrBadGraph = 8u };
@@ -293,6 +293,10 @@ cudaError_t launch_rank_keys(glb_ctx* c, const uint32_t* hot, uint32_t maxc, uin
                              uint32_t* vals);
 cudaError_t launch_assign_slots(glb_ctx* c, const uint32_t* order, uint64_t C);
 cudaError_t launch_vmap_reset(glb_ctx* c);   // gp = ~0, slot = c->slot[v]
+cudaError_t launch_policy_hotness(glb_ctx* c, int policy, uint64_t seed, uint32_t* out);
+cudaError_t launch_topmark(glb_ctx* c, const uint32_t* order, uint64_t C, uint8_t* flag);
+cudaError_t launch_similarity(glb_ctx* c, const uint32_t* fi, const uint32_t* fj,
+                              const uint8_t* ti, const uint8_t* tj, unsigned long long* out2);
 cudaError_t launch_hit_stats(glb_ctx* c, unsigned long long* out3 /* total,hits,max */);
 cudaError_t launch_value_hist(glb_ctx* c, const uint32_t* a, uint64_t n, unsigned long long* bins,
                               uint32_t nbins);

@@ -249,6 +249,54 @@ __global__ void k_vmap_reset(VEntry* __restrict__ vmap, const int32_t* __restric
   }
 }
 
+__global__ void k_policy_hotness(int policy, uint64_t seed, const uint64_t* __restrict__ indptr,
+                                 const uint32_t* __restrict__ counts, uint64_t n,
+                                 uint32_t* __restrict__ out) {
+  const uint32_t c3 = ctr3(0, 0, kDomPolicy);
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n;
+       v += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t h;
+    if (policy == GLB_POLICY_DEGREE) {
+      const uint64_t d = indptr[v + 1] - indptr[v];
+      h = d > 0xFFFFFFFFull ? 0xFFFFFFFFu : (uint32_t)d;
+    } else if (policy == GLB_POLICY_RANDOM) {
+      h = (uint32_t)(draw64(seed, (uint32_t)v, 0, 0, c3, 0) >> 32);
+    } else {
+      h = counts[v];
+    }
+    out[v] = h;
+  }
+}
+
+__global__ void k_topmark(const uint32_t* __restrict__ order, uint64_t C, uint8_t* __restrict__ flag) {
+  for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < C;
+       i += (uint64_t)gridDim.x * blockDim.x)
+    flag[order[i]] = 1;
+}
+
+// num = sum over T_i and T_j of min(f_i, f_j); den = sum over T_j of f_j
+__global__ void k_similarity(const uint32_t* __restrict__ fi, const uint32_t* __restrict__ fj,
+                             const uint8_t* __restrict__ ti, const uint8_t* __restrict__ tj,
+                             uint64_t n, unsigned long long* out2) {
+  unsigned long long num = 0, den = 0;
+  for (uint64_t v = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; v < n;
+       v += (uint64_t)gridDim.x * blockDim.x) {
+    if (tj[v]) {
+      den += fj[v];
+      if (ti[v]) num += min(fi[v], fj[v]);
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    num += __shfl_xor_sync(kFull, num, o);
+    den += __shfl_xor_sync(kFull, den, o);
+  }
+  if ((threadIdx.x & 31) == 0) {
+    if (num) atomicAdd(out2 + 0, num);
+    if (den) atomicAdd(out2 + 1, den);
+  }
+}
+
 __global__ void k_hit_stats(const uint32_t* __restrict__ acc, const int32_t* __restrict__ slot,
                             uint64_t n, unsigned long long* out3) {
   unsigned long long tot = 0, hit = 0;
@@ -390,6 +438,27 @@ cudaError_t launch_assign_slots(glb_ctx* c, const uint32_t* order, uint64_t C) {
 cudaError_t launch_vmap_reset(glb_ctx* c) {
   if (!c->vmap) return cudaSuccess;
   k_vmap_reset<<<grid_for(c), kThreads, 0, c->stream>>>(c->vmap, c->slot, c->V);
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_policy_hotness(glb_ctx* c, int policy, uint64_t seed, uint32_t* out) {
+  k_policy_hotness<<<grid_for(c), kThreads, 0, c->stream>>>(policy, seed, c->indptr, c->counts,
+                                                             c->V, out);
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_topmark(glb_ctx* c, const uint32_t* order, uint64_t C, uint8_t* flag) {
+  if (C == 0) return cudaSuccess;
+  k_topmark<<<grid_for(c), kThreads, 0, c->stream>>>(order, C, flag);
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_similarity(glb_ctx* c, const uint32_t* fi, const uint32_t* fj,
+                              const uint8_t* ti, const uint8_t* tj, unsigned long long* out2) {
+  k_similarity<<<grid_for(c), kThreads, 0, c->stream>>>(fi, fj, ti, tj, c->V, out2);
   count_launch(c);
   return cudaGetLastError();
 }

@@ -13,7 +13,8 @@
  *     are apportioned by cumulative flooring F(r)=floor(E' P_r / P), so
  *     sum(deg) == E exactly.
  *   - Targets: Vose alias table over in-weights (q+1)^(-1/(g_in-1)), in-rank q
- *     is vertex perm_in(q).  Edge (u, j) uses Philox counter
+ *     is vertex perm(q) -- the same permutation as the out-ranks (correlated
+ *     in/out degrees).  Edge (u, j) uses Philox counter
  *     (u, j, 0, c3(0,0,GEN_GRAPH)).  Rows unsorted; multi-edges and
  *     self-loops allowed (PAPER.md L67 does not exclude them).
  *   - Features f(v,d) = ((draw64(v,d,0,c3(0,0,FEATURES),0) >> 40) * 2^-23) - 1,
@@ -33,8 +34,11 @@
 #define SY_GEN_GRAPH 4u
 #define SY_TRAINSET 5u
 #define SY_FEATURES 6u
+/* One rank permutation for both directions: a vertex's out-degree rank equals its
+ * in-weight rank, so in- and out-degree are correlated as in real graphs (for the
+ * undirected ogbn-products they are equal) -- the premise of the Degree policy. */
 #define SY_PERM_OUT 7u
-#define SY_PERM_IN 8u
+#define SY_PERM_IN SY_PERM_OUT
 
 static inline void sy_philox(uint32_t c[4], uint32_t k0, uint32_t k1) {
   for (int r = 0; r < 10; ++r) {

@@ -344,3 +344,32 @@ def test_pipeline_depth2_bit_exact(tiny, alpha, mode):
     # the current sample is still readable after the pipeline drained
     assert_same_sample(ctx.sample_result(),
                        go.sample_khop(ob[-1], sh.fanouts, g.seed, e, len(ob) - 1))
+
+
+def test_policies_and_similarity(tiny):
+    g, go = tiny
+    sh = g.shape
+    ctx = make_ctx(g, fanouts=sh.fanouts)
+    deg = ctx.policy_hotness("degree")
+    assert np.array_equal(u32(deg), oracle.hotness_degree(g.indptr))
+    rnd = ctx.policy_hotness("random", seed=77)
+    assert np.array_equal(u32(rnd), oracle.hotness_random(77, g.V))
+    for pol, h in [("degree", oracle.hotness_degree(g.indptr)),
+                   ("random", oracle.hotness_random(77, g.V))]:
+        for a in [0.05, 0.3]:
+            ctx.build_cache_policy(a, pol, seed=77)
+            assert np.array_equal(ctx.cache_slots(), oracle.cache_slots(h, a)), (pol, a)
+    # footprint similarity between epochs 1 and 2 (Table 2 analog)
+    fs = []
+    for e in [1, 2]:
+        ctx.reset_counts(glb.COUNT_ACCESS)
+        ctx.set_count_mode(glb.COUNT_ACCESS)
+        for b in range(ctx.num_batches):
+            ctx.sample_batch(e, b)
+        ctx.set_count_mode(glb.COUNT_NONE)
+        ctx.sync()
+        fs.append(ctx.counts_tensor(glb.COUNT_ACCESS).clone())
+    got = ctx.footprint_similarity(fs[0], fs[1], 0.1)
+    f1 = go.visit_counts("khop", g.train, sh.batch, sh.fanouts, g.seed, [1])
+    f2 = go.visit_counts("khop", g.train, sh.batch, sh.fanouts, g.seed, [2])
+    assert got[1:] == oracle.footprint_similarity(f1, f2, 0.1)[1:]

@@ -117,3 +117,59 @@ def test_extract_matches_closed_form_features():
     # duplicates allowed: one row per entry
     out2 = go.extract(np.array([5, 5, 0], np.uint32))
     assert np.array_equal(out2[0], out2[1])
+
+
+def test_footprint_similarity_pins():
+    # identical footprints -> 1; disjoint top sets -> 0
+    f = np.array([5, 0, 3, 9, 1, 0, 7, 2, 0, 4], np.uint32)
+    assert oracle.footprint_similarity(f, f, 0.3)[0] == 1.0
+    g = np.array([0, 6, 0, 0, 0, 8, 0, 0, 5, 0], np.uint32)
+    assert oracle.footprint_similarity(f, g, 0.3)[0] == 0.0
+    # hand-computed (L329): T_i = {3, 6, 0} (9, 7, 5), T_j = {0, 3, 1} (8, 6, 5 with tie -> gid)
+    h = np.array([8, 5, 0, 6, 0, 0, 2, 0, 0, 5], np.uint32)
+    v, num, den = oracle.footprint_similarity(f, h, 0.3)
+    assert (num, den) == (min(5, 8) + min(9, 6), 8 + 6 + 5) and v == pytest.approx(11 / 19)
+    # brute force against the definition on random small inputs
+    rng = np.random.default_rng(4)
+    for _ in range(50):
+        V = int(rng.integers(2, 15))
+        fi = rng.integers(0, 6, V).astype(np.uint32)
+        fj = rng.integers(0, 6, V).astype(np.uint32)
+        frac = float(rng.choice([0.1, 0.3, 0.5, 1.0]))
+        C = oracle.cache_size(frac, V)
+        ti = set(brute_rank(fi)[:C])
+        tj = set(brute_rank(fj)[:C])
+        num = sum(min(int(fi[v]), int(fj[v])) for v in ti & tj)
+        den = sum(int(fj[v]) for v in tj)
+        assert oracle.footprint_similarity(fi, fj, frac)[1:] == (num, den)
+
+
+def test_policy_hotness_pins():
+    indptr = np.array([0, 3, 3, 7, 8], np.uint64)
+    assert oracle.hotness_degree(indptr).tolist() == [3, 0, 4, 1]
+    r1 = oracle.hotness_random(5, 20000)
+    assert np.array_equal(r1, oracle.hotness_random(5, 20000))
+    assert not np.array_equal(r1, oracle.hotness_random(6, 20000))
+    # high words of the draw: roughly uniform over 16 buckets
+    from scipy import stats
+    assert stats.chisquare(np.bincount(r1 >> 28, minlength=16)).pvalue > 1e-3
+    # equals the definition for a few vertices
+    for v in [0, 7, 19999]:
+        assert r1[v] == oracle.draw64(5, v, 0, 0, oracle.c3(0, 0, 7), 0) >> 32
+
+
+def test_presc_vs_degree_and_random_on_tiny():
+    """Fig 10 / L339-L343 shape check at alpha = 10% (properties of these seeded
+    inputs, not paper values): PreSC far above Random, and on this power-law graph
+    with correlated in/out degrees Degree comes close to PreSC (L339-L341: Degree
+    is competitive only on power-law graphs)."""
+    g = synth.make_graph("tiny")
+    go = oracle.GraphOracle(g.indptr, g.indices)
+    sh = g.shape
+    counts = go.presample("khop", g.train, sh.batch, sh.fanouts, g.seed, 1)
+    acc = go.visit_counts("khop", g.train, sh.batch, sh.fanouts, g.seed, [1, 2])
+    h = {p: oracle.hit_rate(acc, oracle.cache_slots(x, 0.1)) for p, x in
+         [("presc", counts), ("degree", oracle.hotness_degree(g.indptr)),
+          ("random", oracle.hotness_random(g.seed, g.V))]}
+    assert h["presc"] > 2 * h["random"]
+    assert h["presc"] > 0.95 * h["degree"]
