@@ -74,6 +74,9 @@ def lib():
         L.orc_sample_rwalk.restype = i32
         L.orc_extract.argtypes = [vp, u64, u32, vp, u64, vp]
         L.orc_extract.restype = i32
+        L.orc_sample_khop_weighted.argtypes = [vp, vp, vp, u64, vp, u64, vp, u32, u64, u32, u32,
+                                               vp, vp, u64, vp, vp, u64, vp, u64, vp]
+        L.orc_sample_khop_weighted.restype = i32
         L.orc_policy_random.argtypes = [u64, u64, vp]
         L.orc_policy_random.restype = None
         _lib = L
@@ -190,6 +193,31 @@ class GraphOracle:
         return self._split(uniq, sizes, bptr, bidx, nnz, L, None,
                            picks=picks, fanouts=list(fan) if want_picks else None)
 
+    # NEXT-1 weighted k-hop + a3
+    def sample_khop_weighted(self, weights, seeds, fanouts, seed, epoch, batch) -> Sample:
+        w = np.ascontiguousarray(weights, dtype=np.uint32)
+        seeds = np.ascontiguousarray(seeds, dtype=np.uint32)
+        fan = np.ascontiguousarray(fanouts, dtype=np.uint32)
+        L = fan.shape[0]
+        ub = [seeds.shape[0]]
+        for k in fan:
+            ub.append(min(ub[-1] * (1 + int(k)), self.V))
+        ucap = max(ub[-1], 1)
+        pcap = sum(ub[l] + 1 for l in range(L)) + 1
+        icap = sum(ub[l] * int(k) for l, k in enumerate(fan)) + 1
+        uniq = np.empty(ucap, np.uint32)
+        sizes = np.zeros(L + 1, np.uint64)
+        bptr = np.empty(pcap, np.uint32)
+        bidx = np.empty(icap, np.uint32)
+        nnz = np.zeros(max(L, 1), np.uint64)
+        rc = lib().orc_sample_khop_weighted(_p(self.indptr), _p(self.indices), _p(w), self.V,
+                                            _p(seeds), seeds.shape[0], _p(fan), L, seed, epoch,
+                                            batch, _p(self.lid), _p(uniq), ucap, _p(sizes),
+                                            _p(bptr), pcap, _p(bidx), icap, _p(nnz))
+        if rc:
+            raise OracleError(rc)
+        return self._split(uniq, sizes, bptr, bidx, nnz, L, None)
+
     # a2' + a3
     def sample_rwalk(self, seeds, layers, seed, epoch, batch, walks=4, walk_len=3,
                      topk=5) -> Sample:
@@ -229,9 +257,11 @@ class GraphOracle:
         return Sample(uniq[:sizes[-1]].copy(), sizes, ips, ixs, ws if bw is not None else None,
                       pks if picks is not None else None)
 
-    def sample(self, sampler: str, seeds, fanouts, seed, epoch, batch) -> Sample:
+    def sample(self, sampler: str, seeds, fanouts, seed, epoch, batch, weights=None) -> Sample:
         if sampler == "khop":
             return self.sample_khop(seeds, fanouts, seed, epoch, batch)
+        if sampler == "weighted":
+            return self.sample_khop_weighted(weights, seeds, fanouts, seed, epoch, batch)
         return self.sample_rwalk(seeds, len(fanouts), seed, epoch, batch, topk=fanouts[0])
 
     # a7
@@ -248,18 +278,19 @@ class GraphOracle:
     # a5: PreSC#K (L333: "records the visit count of the sampled vertices";
     # reading Q8/Q9: one visit per (batch, unique vertex), epochs 0..K-1)
     def visit_counts(self, sampler, train, batch_size, fanouts, seed, epochs,
-                     batch_filter=None) -> np.ndarray:
+                     batch_filter=None, weights=None) -> np.ndarray:
         counts = np.zeros(self.V, np.uint32)
         for e in epochs:
             for b, seeds in enumerate(epoch_batches(train, batch_size, seed, e)):
                 if batch_filter is not None and not batch_filter(e, b):
                     continue
-                s = self.sample(sampler, seeds, fanouts, seed, e, b)
+                s = self.sample(sampler, seeds, fanouts, seed, e, b, weights)
                 counts[s.uniq] += 1       # uniq is duplicate-free
         return counts
 
-    def presample(self, sampler, train, batch_size, fanouts, seed, K) -> np.ndarray:
-        return self.visit_counts(sampler, train, batch_size, fanouts, seed, range(K))
+    def presample(self, sampler, train, batch_size, fanouts, seed, K, weights=None) -> np.ndarray:
+        return self.visit_counts(sampler, train, batch_size, fanouts, seed, range(K),
+                                 weights=weights)
 
 
 # ---------------------------------------------------------------- a6

@@ -208,6 +208,66 @@ int orc_sample_khop(const uint64_t* indptr, const uint32_t* indices, uint64_t V,
 }
 
 /* ---------------------------------------------------------------------------
+ * NEXT-1: k-hop WEIGHTED neighbourhood sampling (L81 fn1 "non-uniform (e.g., in
+ * proportion to the edge weight)", L148 fn5, L136, L434 Fig 12 "GCN (W.)";
+ * reading Q19): for a frontier vertex v whose row carries weights w_0..w_{n-1}
+ * (W = their sum), slot s = 0..k-1 draws WITH replacement:
+ *   x = floor(draw64(v, s>>1, batch, c3(epoch,l,WEIGHTED=8), s&1) * W / 2^64),
+ *   pick = the first position p with w_0 + ... + w_p > x   (inverse CDF).
+ * A row with W = 0 yields no picks.  Relabel exactly as in k-hop.
+ * ------------------------------------------------------------------------- */
+int orc_sample_khop_weighted(const uint64_t* indptr, const uint32_t* indices,
+                             const uint32_t* weights, uint64_t V, const uint32_t* seeds,
+                             uint64_t n0, const uint32_t* fanouts, uint32_t L, uint64_t seed,
+                             uint32_t epoch, uint32_t batch, int32_t* lid_scratch,
+                             uint32_t* uniq, uint64_t uniq_cap, uint64_t* sizes,
+                             uint32_t* blk_indptr, uint64_t indptr_cap,
+                             uint32_t* blk_indices, uint64_t indices_cap, uint64_t* nnz) {
+  if (epoch > 0xFFFFu || L > 0xFFu) return ORC_ERANGE;
+  for (uint32_t l = 0; l < L; ++l)
+    if (fanouts[l] == 0 || fanouts[l] > 1024) return ORC_EINVAL;
+  orc_relabel r = {lid_scratch, uniq, 0, uniq_cap};
+  int rc = orc_insert_seeds(&r, seeds, n0, V);
+  if (rc != ORC_OK) { orc_relabel_reset(&r); return rc; }
+  sizes[0] = r.n;
+  uint64_t ip_off = 0, ix_off = 0;
+  for (uint32_t l = 0; l < L; ++l) {
+    uint32_t k = fanouts[l];
+    uint64_t n_l = r.n;
+    uint32_t c3 = orc_c3(epoch, l, 8);
+    if (ip_off + n_l + 1 > indptr_cap) { orc_relabel_reset(&r); return ORC_ENOMEM; }
+    uint32_t* bptr = blk_indptr + ip_off;
+    uint64_t e = 0;
+    for (uint64_t d = 0; d < n_l; ++d) {
+      uint32_t v = r.uniq[d];
+      uint64_t lo = indptr[v], hi = indptr[v + 1];
+      unsigned __int128 W = 0;
+      for (uint64_t q = lo; q < hi; ++q) W += weights[q];
+      bptr[d] = (uint32_t)e;
+      if (W == 0) continue;
+      for (uint32_t s = 0; s < k; ++s) {
+        uint64_t rr = orc_draw64(seed, v, s >> 1, batch, c3, (int)(s & 1u));
+        unsigned __int128 x = ((unsigned __int128)rr * W) >> 64;
+        uint64_t p = lo;
+        unsigned __int128 cum = weights[p];
+        while (cum <= x) { ++p; cum += weights[p]; }
+        int64_t lu = orc_lid_of(&r, indices[p]);
+        if (lu < 0 || ix_off + e >= indices_cap) { orc_relabel_reset(&r); return ORC_ENOMEM; }
+        blk_indices[ix_off + e] = (uint32_t)lu;
+        e += 1;
+      }
+    }
+    bptr[n_l] = (uint32_t)e;
+    nnz[l] = e;
+    sizes[l + 1] = r.n;
+    ip_off += n_l + 1;
+    ix_off += e;
+  }
+  orc_relabel_reset(&r);
+  return ORC_OK;
+}
+
+/* ---------------------------------------------------------------------------
  * a2': PinSAGE random-walk selection (L209, L353; reading Q13).  For each
  * frontier vertex v: `walks` walks of `walk_len` steps from v; step t of
  * walk w at vertex cur picks CSR position

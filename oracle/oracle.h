@@ -53,6 +53,16 @@ int orc_sample_khop(const uint64_t* indptr, const uint32_t* indices, uint64_t V,
                     uint32_t* blk_indices, uint64_t indices_cap, uint64_t* nnz,
                     uint32_t* picks, uint64_t picks_cap);
 
+/* k-hop WEIGHTED sampling with replacement by inverse CDF over the row's edge
+ * weights (L81, L148 fn5; reading Q19); weights: u32[E]. */
+int orc_sample_khop_weighted(const uint64_t* indptr, const uint32_t* indices,
+                             const uint32_t* weights, uint64_t V, const uint32_t* seeds,
+                             uint64_t n0, const uint32_t* fanouts, uint32_t L, uint64_t seed,
+                             uint32_t epoch, uint32_t batch, int32_t* lid_scratch,
+                             uint32_t* uniq, uint64_t uniq_cap, uint64_t* sizes,
+                             uint32_t* blk_indptr, uint64_t indptr_cap,
+                             uint32_t* blk_indices, uint64_t indices_cap, uint64_t* nnz);
+
 /* PinSAGE random-walk neighbour selection ("random
  * walks to select 5 neighbors from 4 paths of length 3"; reading Q13) +
  * the same relabel.  blk_weights parallels blk_indices (visit counts). */

@@ -53,6 +53,8 @@ def lib():
         L.synth_trainset.restype = i32
         L.synth_perm.argtypes = [u64, u64, u32, u64]
         L.synth_perm.restype = u64
+        L.synth_edge_weights.argtypes = [u64, vp, u32, u64, vp, i32]
+        L.synth_edge_weights.restype = i32
         _lib = L
     return _lib
 
@@ -151,6 +153,15 @@ def gen_features(V: int, D: int, seed: int, threads: int = 0, alloc=None) -> np.
         f = alloc(V * D * 4).view(np.float32)[:V * D].reshape(V, D)
     lib().synth_features(V, D, seed, f.ctypes.data, threads)
     return f
+
+
+def gen_edge_weights(indices: np.ndarray, seed: int, levels: int = 16, threads: int = 0):
+    """Per-edge weight = the target's "year registered" (1..levels): weighted sampling
+    prefers newer neighbours."""
+    w = aligned_empty(indices.shape[0], np.uint32)
+    lib().synth_edge_weights(indices.shape[0], indices.ctypes.data, levels, seed,
+                             w.ctypes.data, threads)
+    return w
 
 
 def gen_trainset(V: int, n: int, seed: int) -> np.ndarray:

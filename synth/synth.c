@@ -246,3 +246,22 @@ int synth_trainset(uint64_t V, uint64_t n, uint64_t seed, uint32_t* out) {
   qsort(out, n, sizeof(uint32_t), sy_cmp_u32);
   return 0;
 }
+
+/* ---- edge weights (weighted sampling input: "The weight of a vertex
+ * represents the year registered, and the sampling algorithm prefers to select the
+ * newer neighbors"): w(u->t) = year(t), year(t) in 1..levels drawn per vertex. ---- */
+typedef struct { const uint32_t* indices; uint32_t* w; uint32_t levels; uint32_t k0, k1; } sy_w_ctx;
+static void sy_w_body(void* vc, uint64_t lo, uint64_t hi) {
+  sy_w_ctx* c = (sy_w_ctx*)vc;
+  for (uint64_t e = lo; e < hi; ++e) {
+    uint32_t w[4] = {c->indices[e], 0u, 0u, sy_c3(0, 0, 9u)};
+    sy_philox(w, c->k0, c->k1);
+    c->w[e] = 1u + (uint32_t)(((uint64_t)w[0] * c->levels) >> 32);
+  }
+}
+int synth_edge_weights(uint64_t E, const uint32_t* indices, uint32_t levels, uint64_t seed,
+                       uint32_t* out, int threads) {
+  sy_w_ctx c = {indices, out, levels ? levels : 1u, (uint32_t)seed, (uint32_t)(seed >> 32)};
+  sy_parallel(sy_w_body, &c, E, 1 << 16, threads);
+  return 0;
+}
