@@ -69,8 +69,9 @@ def dist_env():
 
 
 def workload_name(sh, alpha):
-    samp = (f"k-hop {list(sh.fanouts)}" if sh.sampler == "khop"
-            else f"random walk {len(sh.fanouts)}x(4 walks, len 3, top-{sh.fanouts[0]})")
+    samp = {"khop": f"k-hop {list(sh.fanouts)}",
+            "weighted": f"weighted k-hop {list(sh.fanouts)} (edge weight = target year)",
+            "rwalk": f"random walk {len(sh.fanouts)}x(4 walks, len 3, top-{sh.fanouts[0]})"}[sh.sampler]
     return (f"{sh.name}-shaped synthetic power-law graph (V={sh.V}, E={sh.E}, feat {sh.D}), "
             f"{samp}, batch {sh.batch}, PreSC#{sh.K}, alpha={alpha}")
 
@@ -162,7 +163,7 @@ def reference_arm(args):
             batches[e] = oracle.epoch_batches(g.train, sh.batch, g.seed, e)
         seeds = batches[e][b]
         t0 = time.perf_counter()
-        s = go.sample(sh.sampler, seeds, sh.fanouts, g.seed, e, b)
+        s = go.sample(sh.sampler, seeds, sh.fanouts, g.seed, e, b, g.weights)
         go.extract(s.uniq)
         return time.perf_counter() - t0, len(seeds)
 
@@ -197,7 +198,7 @@ def cpu_baseline(g, sh, budget_s):
     t_tot, seeds, nb = 0.0, 0, 0
     while t_tot < budget_s and nb < len(bs):
         t0 = time.perf_counter()
-        s = go.sample(sh.sampler, bs[nb], sh.fanouts, g.seed, sh.K, nb)
+        s = go.sample(sh.sampler, bs[nb], sh.fanouts, g.seed, sh.K, nb, g.weights)
         go.extract(s.uniq)
         t_tot += time.perf_counter() - t0
         seeds += len(bs[nb])
@@ -342,8 +343,10 @@ def main():
     t_load = time.perf_counter() - t0
     kind = sh.sampler
     ctx.set_relabel_mode(args.relabel)
-    if kind == "khop":
-        ctx.set_sampler("khop", fanouts=sh.fanouts, max_batch=sh.batch)
+    if g.weights is not None:
+        ctx.load_edge_weights(g.weights)
+    if kind in ("khop", "weighted"):
+        ctx.set_sampler(kind, fanouts=sh.fanouts, max_batch=sh.batch)
     else:
         ctx.set_sampler("rwalk", layers=len(sh.fanouts), walks=synth.RW_WALKS,
                         walk_len=synth.RW_LEN, topk=sh.fanouts[0], max_batch=sh.batch)

@@ -43,7 +43,9 @@ enum {
 /* sampler kinds */
 enum {
   GLB_KHOP_UNIFORM = 0, /* k-hop uniform neighbourhood sampling (L67, Fig 7) */
-  GLB_RANDOM_WALK = 1   /* PinSAGE random walks: "5 neighbors from 4 paths of length 3" (L353) */
+  GLB_RANDOM_WALK = 1,  /* PinSAGE random walks: "5 neighbors from 4 paths of length 3" (L353) */
+  GLB_KHOP_WEIGHTED = 2 /* k-hop weighted: k draws with replacement, P(edge) = w / row sum
+                           (L81 fn1, L148 fn5, L136; reading Q19); needs glb_load_edge_weights */
 };
 
 /* visit-count recording targets (glb_set_count_mode) */
@@ -74,6 +76,11 @@ glb_status glb_sync(glb_ctx* ctx); /* cudaStreamSynchronize + deferred device er
 glb_status glb_load_graph(glb_ctx* ctx, uint64_t num_vertices, uint64_t num_edges,
                           const uint64_t* indptr, const uint32_t* indices,
                           const void* features, uint32_t feat_dim);
+
+/* Edge weights for GLB_KHOP_WEIGHTED: host u32[E] parallel to `indices` (e.g. the
+ * target's "year registered", L136).  Copied; their inclusive u64 prefix over all edges
+ * is kept in HBM (8 B per edge).  Synchronous. */
+glb_status glb_load_edge_weights(glb_ctx* ctx, const uint32_t* weights);
 
 /* Sampler used by glb_sample_batch / glb_presample, and the capacity of the
  * per-batch buffers.  kind GLB_KHOP_UNIFORM: fanouts[0..num_hops-1] (hop order

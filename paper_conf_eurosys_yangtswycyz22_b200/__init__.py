@@ -20,7 +20,7 @@ import numpy as np
 
 from .build import SO as _SO, build  # noqa: F401
 
-KHOP, RWALK = 0, 1
+KHOP, RWALK, KHOP_WEIGHTED = 0, 1, 2
 POLICY_PRESC, POLICY_DEGREE, POLICY_RANDOM = 0, 1, 2
 COUNT_NONE, COUNT_PRESAMPLE, COUNT_ACCESS = 0, 1, 2
 MAX_HOPS = 8
@@ -37,6 +37,7 @@ EXPORTS = [
     "glb_hit_stats_get", "glb_extract", "glb_extract_sample", "glb_kernel_launches",
     "glb_set_pipeline", "glb_extract_stream", "glb_set_timing", "glb_extract_times",
     "glb_set_relabel_mode", "glb_relabel_mode", "glb_policy_hotness", "glb_footprint_similarity",
+    "glb_load_edge_weights",
 ]
 
 
@@ -121,6 +122,7 @@ def lib(auto_build: bool = True):
         "glb_set_relabel_mode": ([vp, i32], i32),
         "glb_relabel_mode": ([vp, ctypes.POINTER(i32)], i32),
         "glb_policy_hotness": ([vp, i32, u64, vp], i32),
+        "glb_load_edge_weights": ([vp, vp], i32),
         "glb_footprint_similarity": ([vp, vp, vp, dbl, ctypes.POINTER(u64), ctypes.POINTER(u64),
                                       ctypes.POINTER(dbl)], i32),
     }
@@ -226,10 +228,15 @@ class Context:
         self._keep = [features]  # borrowed host memory must outlive the ctx registration
         self.V, self.D = V, D
 
+    def load_edge_weights(self, weights: np.ndarray):
+        """u32 per-edge weights (parallel to indices) for the 'weighted' sampler."""
+        w = np.ascontiguousarray(weights, dtype=np.uint32)
+        self._ck(self._lib.glb_load_edge_weights(self._h, _np_ptr(w)))
+
     def set_sampler(self, kind: str = "khop", fanouts=(25, 10), walks=4, walk_len=3, topk=5,
                     layers=None, max_batch=8000):
-        k = KHOP if kind == "khop" else RWALK
-        if k == KHOP:
+        k = {"khop": KHOP, "rwalk": RWALK, "weighted": KHOP_WEIGHTED}[kind]
+        if k in (KHOP, KHOP_WEIGHTED):
             fan = np.ascontiguousarray(fanouts, dtype=np.uint32)
             L = fan.shape[0]
         else:

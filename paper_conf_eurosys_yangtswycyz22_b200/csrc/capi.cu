@@ -89,7 +89,7 @@ cudaError_t sync_all(glb_ctx* c) {
 }
 
 void free_graph(glb_ctx* c) {
-  dfree(c->indptr); dfree(c->indices); dfree(c->vmap); dfree(c->htab);
+  dfree(c->indptr); dfree(c->indices); dfree(c->wprefix); dfree(c->vmap); dfree(c->htab);
   c->hslot = nullptr;
   c->hmask = 0;
   c->hash_mode = false;
@@ -145,6 +145,7 @@ glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, in
   CK(launch_seed_init(c, seeds_dev, n0, mode));
   for (uint32_t l = 0; l < L; ++l) {
     if (kind == GLB_KHOP_UNIFORM) CK(launch_khop(c, l, k[l], seed, epoch, batch));
+    else if (kind == GLB_KHOP_WEIGHTED) CK(launch_khop_weighted(c, l, k[l], seed, epoch, batch));
     else CK(launch_rwalk(c, l, seed, epoch, batch));
     CK(launch_compact(c, l, k[l], kind == GLB_RANDOM_WALK, mode));
   }
@@ -340,13 +341,31 @@ glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* in
   return GLB_OK;
 }
 
+glb_status glb_load_edge_weights(glb_ctx* c, const uint32_t* weights) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "edge weights before load_graph");
+  if (c->E && !weights) return set_err(c, GLB_EINVAL, "null weights");
+  CK(sync_all(c));
+  dfree(c->wprefix);
+  uint32_t* dw = nullptr;
+  CK(dalloc(&dw, c->E));
+  CK(dalloc(&c->wprefix, c->E));
+  if (c->E) CK(cudaMemcpy(dw, weights, sizeof(uint32_t) * c->E, cudaMemcpyHostToDevice));
+  cudaError_t e = scan_inclusive_u64(c, dw, c->E, c->wprefix);
+  cudaFree(dw);
+  if (e != cudaSuccess) return cuda_fail(c, e, "weight prefix scan");
+  return GLB_OK;
+}
+
 glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32_t L,
                            uint32_t walks, uint32_t len, uint32_t topk, uint32_t max_batch) {
   ENTER(c);
   if (!c->V) return set_err(c, GLB_ESTATE, "set_sampler before load_graph");
   if (L > GLB_MAX_HOPS) return set_err(c, GLB_EINVAL, "num_hops %u > %d", L, GLB_MAX_HOPS);
   uint32_t k[GLB_MAX_HOPS] = {};
-  if (kind == GLB_KHOP_UNIFORM) {
+  if (kind == GLB_KHOP_WEIGHTED && !c->wprefix)
+    return set_err(c, GLB_ESTATE, "weighted sampler before glb_load_edge_weights");
+  if (kind == GLB_KHOP_UNIFORM || kind == GLB_KHOP_WEIGHTED) {
     if (L && !fanouts) return set_err(c, GLB_EINVAL, "null fanouts");
     for (uint32_t l = 0; l < L; ++l) {
       if (fanouts[l] == 0 || fanouts[l] > (uint32_t)kMaxFanout)
@@ -529,7 +548,7 @@ glb_status glb_sample(glb_ctx* c, const uint32_t* seeds, uint32_t n0, const uint
   if (!c->sampler_set) return set_err(c, GLB_ESTATE, "sample before set_sampler");
   if (n0 && !seeds) return set_err(c, GLB_EINVAL, "null seeds");
   const uint32_t* k = c->fanouts;
-  if (c->kind == GLB_KHOP_UNIFORM && fanouts) {
+  if ((c->kind == GLB_KHOP_UNIFORM || c->kind == GLB_KHOP_WEIGHTED) && fanouts) {
     for (uint32_t l = 0; l < L; ++l)
       if (fanouts[l] == 0) return set_err(c, GLB_EINVAL, "fanout 0");
     k = fanouts;

@@ -27,7 +27,7 @@ constexpr int kMaxFanout = 1024;
 constexpr int kMaxWalkLen = 8;
 
 // RNG domains (reading Q4): counter word 3 = epoch<<16 | hop<<8 | domain
-enum : uint32_t { kDomShuffle = 1, kDomKhop = 2, kDomRwalk = 3, kDomPolicy = 7 };
+enum : uint32_t { kDomShuffle = 1, kDomKhop = 2, kDomRwalk = 3, kDomPolicy = 7, kDomWeighted = 8 };
 
 // device error bits (DevState::err)
 enum : uint32_t { kErrDupSeed = 1u, kErrRange = 2u, kErrCapacity = 4u, kErrBadGraph = 8u };
@@ -138,6 +138,7 @@ struct glb_ctx {
   uint64_t V = 0, E = 0;
   uint64_t* indptr = nullptr;
   uint32_t* indices = nullptr;
+  unsigned long long* wprefix = nullptr;  // [E] inclusive prefix of edge weights (weighted k-hop)
   const void* h_features = nullptr;
   const float* features_mapped = nullptr;  // device alias of the registered host matrix
   bool registered = false;
@@ -279,6 +280,9 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
                           uint64_t nhit_host, uint64_t nmiss_host);
 cudaError_t launch_sort_misses(glb_ctx* c, const uint2* miss, const uint32_t* nmiss_dev,
                                uint2* sorted);
+cudaError_t scan_inclusive_u64(glb_ctx* c, const uint32_t* a, uint64_t n, unsigned long long* out);
+cudaError_t launch_khop_weighted(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed,
+                                 uint32_t epoch, uint32_t batch);
 cudaError_t launch_shuffle_keys(glb_ctx* c, uint32_t epoch, unsigned long long* keys, uint32_t* vals);
 cudaError_t radix_sort_pairs_u64(glb_ctx* c, unsigned long long* keys, uint32_t* vals,
                                  unsigned long long* keys_alt, uint32_t* vals_alt, uint64_t n,

@@ -330,6 +330,89 @@ __global__ void k_value_hist(const uint32_t* __restrict__ a, uint64_t n,
   }
 }
 
+// ---- inclusive u64 prefix of u32 values (edge weights; 3 phases, any length) ----
+__global__ void __launch_bounds__(kThreads)
+    k_scan64_reduce(const uint32_t* __restrict__ a, uint64_t n, unsigned long long* __restrict__ sums) {
+  __shared__ unsigned long long red[kWarps];
+  const uint64_t b = (uint64_t)blockIdx.x * kScanChunk;
+  unsigned long long s = 0;
+  for (int i = threadIdx.x; i < kScanChunk; i += kThreads)
+    if (b + i < n) s += a[b + i];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(kFull, s, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned long long t = 0;
+    for (int w = 0; w < kWarps; ++w) t += red[w];
+    sums[blockIdx.x] = t;
+  }
+}
+
+__device__ __forceinline__ unsigned long long block_excl_scan64(unsigned long long x,
+                                                                unsigned long long* total) {
+  __shared__ unsigned long long s[kWarps];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  unsigned long long inc = x;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const unsigned long long y = __shfl_up_sync(kFull, inc, o);
+    if (lane >= o) inc += y;
+  }
+  if (lane == 31) s[w] = inc;
+  __syncthreads();
+  if (w == 0) {
+    unsigned long long t = lane < kWarps ? s[lane] : 0, ti = t;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned long long y = __shfl_up_sync(kFull, ti, o);
+      if (lane >= o) ti += y;
+    }
+    if (lane < kWarps) s[lane] = ti - t;
+    if (lane == kWarps - 1) *total = ti;
+  }
+  __syncthreads();
+  const unsigned long long res = s[w] + inc - x;
+  __syncthreads();
+  return res;
+}
+
+__global__ void __launch_bounds__(kThreads) k_scan64_sums(unsigned long long* sums, uint64_t m) {
+  __shared__ unsigned long long total;
+  unsigned long long carry = 0;
+  for (uint64_t b = 0; b < m; b += kThreads) {
+    const uint64_t i = b + threadIdx.x;
+    const unsigned long long x = i < m ? sums[i] : 0ull;
+    const unsigned long long ex = block_excl_scan64(x, &total);
+    if (i < m) sums[i] = carry + ex;
+    carry += total;
+    __syncthreads();
+  }
+}
+
+__global__ void __launch_bounds__(kThreads)
+    k_scan64_down(const uint32_t* __restrict__ a, uint64_t n,
+                  const unsigned long long* __restrict__ sums, unsigned long long* __restrict__ out) {
+  __shared__ unsigned long long total;
+  const uint64_t b = (uint64_t)blockIdx.x * kScanChunk;
+  constexpr int kPer = kScanChunk / kThreads;
+  uint32_t x[kPer];
+  unsigned long long s = 0;
+#pragma unroll
+  for (int q = 0; q < kPer; ++q) {
+    const uint64_t i = b + (uint64_t)threadIdx.x * kPer + q;
+    x[q] = i < n ? a[i] : 0u;
+    s += x[q];
+  }
+  unsigned long long run = sums[blockIdx.x] + block_excl_scan64(s, &total);
+#pragma unroll
+  for (int q = 0; q < kPer; ++q) {
+    const uint64_t i = b + (uint64_t)threadIdx.x * kPer + q;
+    run += x[q];
+    if (i < n) out[i] = run;  // inclusive
+  }
+}
+
 cudaError_t scan_exclusive_u32(glb_ctx* c, const uint32_t* a, uint64_t n, uint32_t* out,
                                uint32_t* sums) {
   const uint64_t m = (n + kScanChunk - 1) / kScanChunk;
@@ -399,6 +482,21 @@ cudaError_t radix_sort_pairs_u32(glb_ctx* c, uint32_t* keys, uint32_t* vals, uin
                                  uint32_t** vals_out) {
   return radix_sort_pairs<uint32_t>(c, keys, vals, keys_alt, vals_alt, n, bits, keys_out,
                                     vals_out);
+}
+
+cudaError_t scan_inclusive_u64(glb_ctx* c, const uint32_t* a, uint64_t n, unsigned long long* out) {
+  const uint64_t m = (n + kScanChunk - 1) / kScanChunk;
+  if (m == 0) return cudaSuccess;
+  unsigned long long* sums = nullptr;
+  cudaError_t e = cudaMalloc(&sums, sizeof(unsigned long long) * m);
+  if (e != cudaSuccess) return e;
+  k_scan64_reduce<<<(unsigned)m, kThreads, 0, c->stream>>>(a, n, sums);
+  k_scan64_sums<<<1, kThreads, 0, c->stream>>>(sums, m);
+  k_scan64_down<<<(unsigned)m, kThreads, 0, c->stream>>>(a, n, sums, out);
+  count_launch(c, 3);
+  e = cudaStreamSynchronize(c->stream);
+  cudaFree(sums);
+  return e == cudaSuccess ? cudaGetLastError() : e;
 }
 
 cudaError_t launch_shuffle_keys(glb_ctx* c, uint32_t epoch, unsigned long long* keys,

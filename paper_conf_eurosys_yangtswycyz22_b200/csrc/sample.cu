@@ -296,6 +296,67 @@ __global__ void __launch_bounds__(kThreads)
   }
 }
 
+// ---------------------------------------------------------------- weighted k-hop (NEXT-1)
+// L81 fn1 / L148 fn5 / L136; reading Q19: slot s of frontier vertex v draws with
+// replacement x = floor(r * W / 2^64) over the row's total weight W and picks the
+// first position whose inclusive weight prefix exceeds x.  The prefix is global over
+// all edges (wprefix, u64), so the row's prefix is wprefix - wprefix[lo - 1].  One
+// lane per slot; slots beyond 32 loop.  Binary search over the row.
+template <bool HASH>
+__global__ void __launch_bounds__(kThreads)
+    k_khop_weighted(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch,
+                    Table T, const DevState* __restrict__ st, DevState* st_w,
+                    const uint64_t* __restrict__ indptr, const uint32_t* __restrict__ indices,
+                    const unsigned long long* __restrict__ wprefix,
+                    const uint32_t* __restrict__ uniq, uint32_t* __restrict__ picks,
+                    uint32_t* __restrict__ pidx, uint32_t* fix_ind) {
+  pdl_enter();
+  if (fix_ind) fixup_block(st->nnz[hop - 1], T.e, fix_ind);
+  const uint32_t gen = T.gen;
+  const uint32_t n_l = st->n[hop];
+  const uint32_t base = st->base[hop];
+  const uint32_t c3 = ctr3(epoch, hop, kDomWeighted);
+  const uint32_t G = k < 32 ? k : 32;         // lanes per vertex
+  const int lane = threadIdx.x & 31;
+  const uint32_t gpw = 32 / G;
+  const uint32_t gi = (uint32_t)lane / G;
+  const uint32_t sl = (uint32_t)lane - gi * G;
+  const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  for (uint32_t w0 = warp_global * gpw; w0 < n_l; w0 += nwarps * gpw) {
+    const uint32_t d = w0 + gi;
+    if (gi >= gpw || d >= n_l) continue;
+    const uint32_t v = uniq[d];
+    const uint64_t lo = indptr[v], hi = indptr[v + 1];
+    const unsigned long long pbase = lo ? wprefix[lo - 1] : 0ull;
+    const unsigned long long W = hi > lo ? wprefix[hi - 1] - pbase : 0ull;
+    for (uint32_t s = sl; s < k; s += G) {
+      uint32_t u = kEmpty, idx = kEmpty;
+      if (W) {
+        const unsigned long long x =
+            __umul64hi(draw64(seed, v, s >> 1, batch, c3, s & 1u), W);  // floor(r*W/2^64)
+        const unsigned long long target = pbase + x;
+        uint64_t a = lo, b = hi - 1;  // first p in [lo, hi) with wprefix[p] > target
+        while (a < b) {
+          const uint64_t m = a + ((b - a) >> 1);
+          if (__ldg(wprefix + m) > target) b = m;
+          else a = m + 1;
+        }
+        u = __ldg(indices + a);
+        idx = entry_of<HASH>(T, u, st_w);
+        if (idx != kEmpty) {
+          const unsigned long long e = enc_pos(gen, base + d * k + s);
+          u = encode_pick(u, vmap_insert(T.e, idx, e), e, base);
+        } else {
+          u = kEmpty;
+        }
+      }
+      picks[(size_t)d * k + s] = u;
+      if (HASH) pidx[(size_t)d * k + s] = idx;
+    }
+  }
+}
+
 // Fanout > 32: one warp per vertex, Floyd run sequentially by lane 0 in shared memory.
 template <bool HASH>
 __global__ void __launch_bounds__(kThreads)
@@ -821,6 +882,26 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
     e = c->hash_mode ? launch_pdl_w(c->pin, k_khop_wide<true>, grid, kThreads, c->stream, GLB_KH_ARGS)
                      : launch_pdl_w(c->pin, k_khop_wide<false>, grid, kThreads, c->stream, GLB_KH_ARGS);
 #undef GLB_KH_ARGS
+  count_launch(c);
+  return e;
+}
+
+cudaError_t launch_khop_weighted(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed,
+                                 uint32_t epoch, uint32_t batch) {
+  const int grid = grid_for(c);
+  const SampleBufs& b = c->sb;
+  uint32_t* fix = hop ? b.bindices[hop - 1] : nullptr;
+  const DevState* stc = c->st;
+  const uint64_t* ip = c->indptr;
+  const uint32_t* ix = c->indices;
+  const unsigned long long* wp = c->wprefix;
+  const uint32_t* uq = b.uniq;
+  const Table T = table_of(c);
+  cudaError_t e;
+#define GLB_KW_ARGS hop, k, seed, epoch, batch, T, stc, c->st, ip, ix, wp, uq, b.picks, b.pidx, fix
+  e = c->hash_mode ? launch_pdl_w(c->pin, k_khop_weighted<true>, grid, kThreads, c->stream, GLB_KW_ARGS)
+                   : launch_pdl_w(c->pin, k_khop_weighted<false>, grid, kThreads, c->stream, GLB_KW_ARGS);
+#undef GLB_KW_ARGS
   count_launch(c);
   return e;
 }

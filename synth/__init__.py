@@ -88,8 +88,14 @@ SHAPES = {
                 (5, 5, 5), 1, (0.22, 0.05, 0.10)),
     "UK": Shape("UK", 77_741_046, 2_965_197_340, 3.0, 2.1, 256, 1_000_000, 8000, "khop", (25, 10),
                 1, (0.18, 1.0)),
+    # NEXT-1 (not a BASELINE config): Twitter with 3-hop WEIGHTED sampling, edge weight =
+    # the target's "year registered" (Fig 5(b), Fig 12 "GCN (W.)").
+    "TWW": Shape("TWW", 41_652_230, 1_468_365_182, 2.1, 2.1, 256, 417_000, 8000, "weighted",
+                 (15, 10, 5), 1, (0.25, 0.10, 1.0)),
+    "PRW": Shape("PRW", 2_449_029, 123_718_280, 2.5, 2.5, 100, 196_615, 8000, "weighted",
+                 (25, 10), 1, (0.05, 0.10, 0.25, 1.0)),
 }
-CONFIG_INDEX = {"tiny": 0, "PR": 1, "TW": 2, "PA": 3, "UK": 4}
+CONFIG_INDEX = {"tiny": 0, "PR": 1, "TW": 2, "PA": 3, "UK": 4, "TWW": 2, "PRW": 1}
 
 # PinSAGE random walk: 4 paths of length 3, keep 5.
 RW_WALKS, RW_LEN, RW_TOPK = 4, 3, 5
@@ -116,6 +122,7 @@ class Graph:
     indices: np.ndarray    # u32[E]
     train: np.ndarray      # u32[n_train], sorted
     features: np.ndarray | None  # f32[V, D] (None if not generated)
+    weights: np.ndarray | None = None  # u32[E] edge weights (weighted sampler shapes)
 
     @property
     def V(self):
@@ -182,7 +189,8 @@ def make_graph(shape: Shape | str, seed: int | None = None, features: bool = Tru
                                    threads)
     train = gen_trainset(shape.V, shape.n_train, seed)
     feats = gen_features(shape.V, shape.D, seed, threads, feature_alloc) if features else None
-    return Graph(shape, seed, indptr, indices, train, feats)
+    w = gen_edge_weights(indices, seed, threads=threads) if shape.sampler == "weighted" else None
+    return Graph(shape, seed, indptr, indices, train, feats, w)
 
 
 def small_graph(V: int, E: int, gamma: float, D: int, n_train: int, seed: int,

@@ -373,3 +373,27 @@ def test_policies_and_similarity(tiny):
     f1 = go.visit_counts("khop", g.train, sh.batch, sh.fanouts, g.seed, [1])
     f2 = go.visit_counts("khop", g.train, sh.batch, sh.fanouts, g.seed, [2])
     assert got[1:] == oracle.footprint_similarity(f1, f2, 0.1)[1:]
+
+
+@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("fanouts", [(10, 5), (15, 10, 5), (40,)])
+def test_weighted_khop_parity(fanouts, mode):
+    g = synth.small_graph(6000, 90000, 2.1, 8, 700, seed=13)
+    w = synth.gen_edge_weights(g.indices, 13)
+    w[::7] = 0                                              # some zero-weight edges
+    go = oracle.GraphOracle(g.indptr, g.indices)
+    ctx = glb.Context(0)
+    ctx.load_graph(g.indptr, g.indices, g.features)
+    ctx.load_edge_weights(w)
+    ctx.set_relabel_mode(mode)
+    ctx.set_sampler("weighted", fanouts=fanouts, max_batch=300)
+    for b, n0 in enumerate([1, 37, 300]):
+        seeds = g.train[b * 200:b * 200 + n0]
+        assert_same_sample(ctx.sample(seeds, seed=5, epoch=b, batch=b),
+                           go.sample_khop_weighted(w, seeds, fanouts, 5, b, b))
+    # PreSC with the weighted sampler (Fig 11(a)/Table 2 "3-hop weighted" analog)
+    ctx.set_sampler("weighted", fanouts=fanouts, max_batch=64)
+    ctx.set_train_set(g.train, 64, g.seed)
+    ctx.presample(1)
+    exp = go.presample("weighted", g.train, 64, fanouts, g.seed, 1, weights=w)
+    assert np.array_equal(ctx.get_counts(glb.COUNT_PRESAMPLE), exp)
