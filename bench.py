@@ -56,6 +56,9 @@ def parse():
                    help="relabel table (glb_set_relabel_mode)")
     p.add_argument("--host-alloc", default="register", choices=["register", "cuda"],
                    help="host feature memory: pageable + cudaHostRegister, or cudaHostAlloc")
+    p.add_argument("--cache", default="replicated", choices=["replicated", "sharded"],
+                   help="sharded: each rank caches alpha*V distinct rows, peers read them over "
+                        "NVLink (NEXT-3; glb_build_cache_sharded)")
     p.add_argument("--pipeline", type=int, default=1, choices=[1, 2],
                    help="2: extract of batch b overlaps sampling of batch b+1 (two streams)")
     return p.parse_args()
@@ -373,10 +376,14 @@ def main():
     torch.cuda.synchronize()
     t_pre = time.perf_counter() - t0
     t0 = time.perf_counter()
-    ctx.build_cache(args.alpha)
+    if args.cache == "sharded":
+        par.build_sharded_cache(ctx, args.alpha, rank, world)
+    else:
+        ctx.build_cache(args.alpha)
     torch.cuda.synchronize()
     t_cache = time.perf_counter() - t0
 
+    ctx_cache_rows = ctx.cache_size
     ub = sh.batch
     for k in sh.fanouts:
         ub = min(ub * (1 + k), sh.V)
@@ -502,6 +509,12 @@ def main():
     result_hit = None
     sweep = []
     similarity = None
+    peer_share = None
+    if args.cache == "sharded":
+        # share of extracted rows served by another rank's shard (last replayed batch)
+        k = ctx.last_extract_counts()
+        peer_share = k["peer_hits"] / max(1, k["hits"] + k["misses"])
+        barrier()  # peers may still read this rank's shard: nobody rebuilds before here
     if not args.no_sweep:
         def reduce_counts(t):
             if world > 1:
@@ -577,6 +590,8 @@ def main():
                        "l2": "inputs larger than L2 (CSR %.2f GB, feature cache %.2f GB vs 126 MB L2)"
                              % ((8 * (sh.V + 1) + 4 * sh.E) / 1e9, 4 * sh.D * sh.V * args.alpha / 1e9)},
             "pipeline_depth": args.pipeline,
+            "cache": {"layout": args.cache, "rows_cached": ctx_cache_rows,
+                      "peer_hit_share": peer_share},
             "relabel_table": ctx.relabel_mode,
             "host_wall_ms_timed_region": wall_ms,
             "host_enqueue_ms_timed_region": enqueue_ms,

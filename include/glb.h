@@ -183,6 +183,39 @@ glb_status glb_footprint_similarity(glb_ctx* ctx, const uint32_t* f_i, const uin
                                     double top_frac, uint64_t* num, uint64_t* den, double* out);
 glb_status glb_cache_size(const glb_ctx* ctx, uint64_t* out);
 
+/* ------------------------------------------------ NEXT-3: peer-sharded cache over NVLink
+ * The paper's GPUs cache the same hot rows each, and a cross-GPU access is "74x slower"
+ * than local (L516 §9); NVSwitch gives every B200 ~900 GB/s to every peer, so `world`
+ * GPUs can instead cache world x as many distinct rows.
+ * glb_build_cache_sharded: C = min(V, world * floor(alpha*V)) global rows, ranked as in
+ * glb_build_cache (slot[v] = global rank i, reading Q10); this ctx (shard `rank`) stores
+ * the rows i with i % world == rank at local row i / world.  world == 1 is
+ * glb_build_cache.  Every ctx of the group must build with the same hotness, alpha and
+ * world.  Synchronous.  Errors: EINVAL (world > GLB_MAX_SHARDS, rank >= world),
+ * ESTATE (no graph / no features).
+ * Until every other shard is attached (glb_attach_peer_cache), extract returns ESTATE. */
+#define GLB_MAX_SHARDS 16
+#define GLB_IPC_HANDLE_BYTES 64
+glb_status glb_build_cache_sharded(glb_ctx* ctx, double alpha, const uint32_t* hotness,
+                                   uint32_t rank, uint32_t world);
+/* device pointer of this ctx's cache rows f32[rows][D] (rows = its shard's row count) */
+glb_status glb_cache_device_ptr(glb_ctx* ctx, void** out, uint64_t* rows);
+/* CUDA IPC handle (GLB_IPC_HANDLE_BYTES opaque bytes) of this ctx's shard, for another
+ * process (e.g. all-gathered over torch.distributed).  ESTATE if there is no shard. */
+glb_status glb_cache_ipc_handle(glb_ctx* ctx, void* handle_out);
+/* Map shard `peer`'s rows for reading by this ctx's extract: exactly one of
+ *  ipc_handle -- from glb_cache_ipc_handle in another process (opened with
+ *                cudaIpcOpenMemHandle; closed on the next build or destroy), or
+ *  dev_ptr    -- glb_cache_device_ptr of a ctx in THIS process (same GPU, or another
+ *                GPU: peer access is enabled; EINVAL if the GPUs cannot access each other).
+ * The peer must keep its shard alive (no rebuild / destroy) while this ctx extracts.
+ * Synchronous.  Errors: ESTATE (cache not sharded), EINVAL (peer == own rank, >= world). */
+glb_status glb_attach_peer_cache(glb_ctx* ctx, uint32_t peer, const void* ipc_handle,
+                                 const void* dev_ptr);
+/* Counts of the last extract: out[0] = cache hits (local + peer shards), out[1] = host
+ * misses, out[2] = hits served by another GPU's shard (0 unless sharded).  Synchronous. */
+glb_status glb_last_extract_counts(glb_ctx* ctx, uint64_t* out3);
+
 /* Hit-rate statistics over the recorded accesses (GLB_COUNT_ACCESS) for the
  * current cache: total accesses, accesses served by the cache (H = hits/total),
  * and the Optimal policy's hits: the C largest access counts (L148 fn4, L339).

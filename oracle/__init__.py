@@ -317,6 +317,31 @@ def cache_slots(counts: np.ndarray, alpha: float) -> np.ndarray:
     return slot
 
 
+# ---------------------------------------------------------------- NEXT-3 sharded cache
+def sharded_cache(counts: np.ndarray, alpha: float, world: int):
+    """Peer-sharded load_cache (the paper's cross-GPU access, L516 §9):
+    `world` GPUs each hold floor(alpha*V) rows, so C = min(V, world*floor(alpha*V))
+    distinct rows are cached; the vertex of rank i < C (ranking of L301, reading Q10) has
+    global slot i and lives on shard i % world at row i // world.
+    Returns (slot i32[V], [rows of shard r: vertex ids in row order, r < world])."""
+    V = counts.shape[0]
+    C = min(V, world * cache_size(alpha, V))
+    order = cache_rank(counts)
+    slot = np.full(V, -1, np.int32)
+    slot[order[:C]] = np.arange(C, dtype=np.int32)
+    shards = [order[:C][r::world] for r in range(world)]
+    return slot, shards
+
+
+def extract_counts(vertices: np.ndarray, slot: np.ndarray, rank: int = 0, world: int = 1):
+    """(hits, misses, peer_hits) of one extract on shard `rank`: a hit is a cached vertex
+    (L252); a peer hit is one whose row lives on another GPU's shard."""
+    s = slot[np.asarray(vertices, dtype=np.int64)]
+    hit = s >= 0
+    peer = hit & ((s % world) != rank)
+    return int(hit.sum()), int((~hit).sum()), int(peer.sum())
+
+
 # ---------------------------------------------------------------- policies (Fig 10)
 def hotness_degree(indptr: np.ndarray) -> np.ndarray:
     """Degree policy (PaGraph; L79, L301): h_v = out-degree."""

@@ -37,8 +37,11 @@ EXPORTS = [
     "glb_hit_stats_get", "glb_extract", "glb_extract_sample", "glb_kernel_launches",
     "glb_set_pipeline", "glb_extract_stream", "glb_set_timing", "glb_extract_times",
     "glb_set_relabel_mode", "glb_relabel_mode", "glb_policy_hotness", "glb_footprint_similarity",
-    "glb_load_edge_weights",
+    "glb_load_edge_weights", "glb_build_cache_sharded", "glb_cache_device_ptr",
+    "glb_cache_ipc_handle", "glb_attach_peer_cache", "glb_last_extract_counts",
 ]
+MAX_SHARDS = 16
+IPC_HANDLE_BYTES = 64
 
 
 class GlbError(RuntimeError):
@@ -123,6 +126,11 @@ def lib(auto_build: bool = True):
         "glb_relabel_mode": ([vp, ctypes.POINTER(i32)], i32),
         "glb_policy_hotness": ([vp, i32, u64, vp], i32),
         "glb_load_edge_weights": ([vp, vp], i32),
+        "glb_build_cache_sharded": ([vp, dbl, vp, u32, u32], i32),
+        "glb_cache_device_ptr": ([vp, ctypes.POINTER(vp), ctypes.POINTER(u64)], i32),
+        "glb_cache_ipc_handle": ([vp, vp], i32),
+        "glb_attach_peer_cache": ([vp, u32, vp, vp], i32),
+        "glb_last_extract_counts": ([vp, ctypes.POINTER(u64)], i32),
         "glb_footprint_similarity": ([vp, vp, vp, dbl, ctypes.POINTER(u64), ctypes.POINTER(u64),
                                       ctypes.POINTER(dbl)], i32),
     }
@@ -367,6 +375,43 @@ class Context:
                                                     float(top_frac), ctypes.byref(num),
                                                     ctypes.byref(den), ctypes.byref(out)))
         return out.value, num.value, den.value
+
+    # ---------------------------------------------------- NEXT-3: peer-sharded cache
+    def build_cache_sharded(self, alpha: float, rank: int, world: int, hotness=None):
+        """Cache world*floor(alpha*V) rows over ``world`` GPUs; this ctx holds shard ``rank``
+        (global rank i -> shard i % world, row i // world).  Attach the other shards next."""
+        hp = None
+        if hotness is not None:
+            assert hotness.is_cuda and hotness.numel() == self.V and hotness.is_contiguous()
+            hp = hotness.data_ptr()
+        self._ck(self._lib.glb_build_cache_sharded(self._h, float(alpha), hp, rank, world))
+
+    def cache_device_ptr(self):
+        """(device pointer, rows) of this ctx's own cache rows."""
+        p, n = ctypes.c_void_p(), ctypes.c_uint64()
+        self._ck(self._lib.glb_cache_device_ptr(self._h, ctypes.byref(p), ctypes.byref(n)))
+        return p.value, n.value
+
+    def cache_ipc_handle(self) -> bytes:
+        buf = ctypes.create_string_buffer(IPC_HANDLE_BYTES)
+        self._ck(self._lib.glb_cache_ipc_handle(self._h, buf))
+        return buf.raw
+
+    def attach_peer_cache(self, peer: int, ipc_handle: bytes | None = None,
+                          dev_ptr: int | None = None):
+        """Map shard ``peer``: an IPC handle from another process, or a device pointer of a
+        ctx in this process."""
+        h = None
+        if ipc_handle is not None:
+            assert len(ipc_handle) == IPC_HANDLE_BYTES
+            h = ctypes.create_string_buffer(ipc_handle, IPC_HANDLE_BYTES)
+        self._ck(self._lib.glb_attach_peer_cache(self._h, peer, h, dev_ptr))
+
+    def last_extract_counts(self) -> dict:
+        """Synchronous: hits (local + peer), misses and peer-shard hits of the last extract."""
+        a = (ctypes.c_uint64 * 3)()
+        self._ck(self._lib.glb_last_extract_counts(self._h, a))
+        return {"hits": a[0], "misses": a[1], "peer_hits": a[2]}
 
     def cache_slots(self) -> np.ndarray:
         out = np.empty(self.V, np.int32)

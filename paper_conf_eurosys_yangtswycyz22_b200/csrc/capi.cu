@@ -88,7 +88,21 @@ cudaError_t sync_all(glb_ctx* c) {
   return e;
 }
 
+// Drop the peer-shard mapping (IPC-opened peers are closed); the cache becomes local.
+void close_shards(glb_ctx* c) {
+  for (int r = 0; r < kMaxShards; ++r) {
+    if (c->shard_ipc[r]) cudaIpcCloseMemHandle(c->shard_ipc[r]);
+    c->shard_ipc[r] = nullptr;
+    c->shard_base[r] = nullptr;
+  }
+  c->shard_rank = 0;
+  c->shard_world = 1;
+  c->shard_attached = 0;
+  c->C_local = 0;
+}
+
 void free_graph(glb_ctx* c) {
+  close_shards(c);
   dfree(c->indptr); dfree(c->indices); dfree(c->wprefix); dfree(c->vmap); dfree(c->htab);
   c->hslot = nullptr;
   c->hmask = 0;
@@ -104,6 +118,10 @@ void free_graph(glb_ctx* c) {
   c->D = 0;
   c->gen = 0;
   c->have_sample = false;
+}
+
+bool shards_ready(const glb_ctx* c) {
+  return c->shard_world < 2 || c->shard_attached == (uint32_t)((1ull << c->shard_world) - 1);
 }
 
 glb_status check_dev_err(glb_ctx* c, DevState* st) {
@@ -214,11 +232,12 @@ glb_status glb_create(int device, glb_ctx** out) {
       (e = cudaMalloc(&c->sts[1], sizeof(DevState))) != cudaSuccess ||
       (e = cudaMalloc(&c->st_x, sizeof(DevState))) != cudaSuccess ||
       (e = cudaMalloc(&c->scratch, 4 * sizeof(unsigned long long))) != cudaSuccess ||
-      (e = cudaMalloc(&c->xcount, 2 * sizeof(unsigned long long))) != cudaSuccess ||
+      (e = cudaMalloc(&c->xcount, 3 * sizeof(unsigned long long))) != cudaSuccess ||
+      (e = cudaMemset(c->xcount, 0, 3 * sizeof(unsigned long long))) != cudaSuccess ||
       (e = cudaMalloc(&c->work, 8 * sizeof(unsigned int))) != cudaSuccess ||
       (e = cudaMemset(c->work, 0, 8 * sizeof(unsigned int))) != cudaSuccess ||
       (e = cudaMallocHost(&c->h_st, sizeof(DevState))) != cudaSuccess ||
-      (e = cudaMallocHost(&c->h_xcount, 2 * sizeof(unsigned long long))) != cudaSuccess ||
+      (e = cudaMallocHost(&c->h_xcount, 3 * sizeof(unsigned long long))) != cudaSuccess ||
       (e = cudaMemset(c->sts[0], 0, sizeof(DevState))) != cudaSuccess ||
       (e = cudaMemset(c->sts[1], 0, sizeof(DevState))) != cudaSuccess ||
       (e = cudaMemset(c->st_x, 0, sizeof(DevState))) != cudaSuccess) {
@@ -651,17 +670,17 @@ static glb_status rank_vertices(glb_ctx* c, const uint32_t* hot, uint32_t* tmp, 
   return GLB_OK;
 }
 
-glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
-  ENTER(c);
-  if (!c->V) return set_err(c, GLB_ESTATE, "build_cache before load_graph");
-  if (!(alpha >= 0.0 && alpha <= 1.0)) return set_err(c, GLB_EINVAL, "alpha %g not in [0,1]", alpha);
+// load_cache (L301) for a cache of C global rows split over `world` shards: the
+// vertex of global rank i is cached iff i < C, slot[v] = i; shard i % world holds it
+// at row i / world (world == 1: the whole cache is local, row = rank).
+static glb_status build_cache_impl(glb_ctx* c, uint64_t C, const uint32_t* hotness, uint32_t rank,
+                                   uint32_t world) {
   const uint64_t V = c->V;
-  uint64_t C = (uint64_t)std::floor(alpha * (double)V);
-  if (C > V) C = V;
   const uint32_t* hot = hotness ? hotness : c->counts;
   CK(sync_all(c));  // an in-flight extract may still read the old cache
+  close_shards(c);
   uint32_t* tmp = nullptr;
-  CK(dalloc(&tmp, 4 * V));
+  CK(dalloc(&tmp, 5 * V));
   uint32_t* order = nullptr;
   glb_status s = rank_vertices(c, hot, tmp, &order);
   if (s != GLB_OK) { cudaFree(tmp); return s; }
@@ -670,15 +689,120 @@ glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
   CK(launch_vmap_reset(c));  // dense mode: copy the slots into the relabel entries
   dfree(c->cache);
   c->C = C;
-  if (c->features_mapped && C) {
-    CK(dalloc(&c->cache, C * (uint64_t)c->D));
+  c->shard_rank = rank;
+  c->shard_world = world;
+  const uint64_t Cl = C > rank ? (C - rank + world - 1) / world : 0;  // rows i = j*world + rank
+  c->C_local = Cl;
+  if (c->features_mapped && (Cl || world > 1)) {
+    CK(dalloc(&c->cache, Cl * (uint64_t)c->D));  // >= 1 element: a shard always has a base
+    const uint32_t* rows = order;
+    if (world > 1) {
+      uint32_t* sub = tmp + 4 * V;
+      CK(launch_shard_rows(c, order, world, rank, Cl, sub));
+      rows = sub;
+    }
     // cache rows come over PCIe from the mapped host matrix (zero copy)
-    CK(launch_gather(c, c->cache, nullptr, c->features_mapped, nullptr, nullptr, order, nullptr,
-                     0, C));
+    if (Cl)
+      CK(launch_gather(c, c->cache, nullptr, c->features_mapped, nullptr, nullptr, rows, nullptr,
+                       0, Cl));
   }
+  c->shard_base[rank] = c->cache;
+  c->shard_attached = 1u << rank;
   CK(cudaStreamSynchronize(c->stream));
   cudaFree(tmp);
   c->have_sample = false;  // marks of an earlier sample refer to the old cache
+  return GLB_OK;
+}
+
+glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "build_cache before load_graph");
+  if (!(alpha >= 0.0 && alpha <= 1.0)) return set_err(c, GLB_EINVAL, "alpha %g not in [0,1]", alpha);
+  uint64_t C = (uint64_t)std::floor(alpha * (double)c->V);
+  if (C > c->V) C = c->V;
+  return build_cache_impl(c, C, hotness, 0, 1);
+}
+
+glb_status glb_build_cache_sharded(glb_ctx* c, double alpha, const uint32_t* hotness,
+                                   uint32_t rank, uint32_t world) {
+  ENTER(c);
+  if (!c->V) return set_err(c, GLB_ESTATE, "build_cache before load_graph");
+  if (!(alpha >= 0.0 && alpha <= 1.0)) return set_err(c, GLB_EINVAL, "alpha %g not in [0,1]", alpha);
+  if (world < 1 || world > (uint32_t)kMaxShards || rank >= world)
+    return set_err(c, GLB_EINVAL, "shard rank %u / world %u (world <= %d)", rank, world, kMaxShards);
+  uint64_t C = (uint64_t)std::floor(alpha * (double)c->V) * world;
+  if (C > c->V) C = c->V;
+  if (world > 1 && !c->features_mapped)
+    return set_err(c, GLB_ESTATE, "a sharded cache needs a graph with features");
+  return build_cache_impl(c, C, hotness, rank, world);
+}
+
+glb_status glb_cache_device_ptr(glb_ctx* c, void** out, uint64_t* rows) {
+  ENTER(c);
+  if (!out) return set_err(c, GLB_EINVAL, "null out");
+  *out = c->cache;
+  if (rows) *rows = c->C_local;
+  return GLB_OK;
+}
+
+glb_status glb_cache_ipc_handle(glb_ctx* c, void* handle_out) {
+  ENTER(c);
+  if (!handle_out) return set_err(c, GLB_EINVAL, "null out");
+  if (!c->cache) return set_err(c, GLB_ESTATE, "no cache shard (build_cache_sharded first)");
+  static_assert(sizeof(cudaIpcMemHandle_t) == GLB_IPC_HANDLE_BYTES, "IPC handle size");
+  cudaIpcMemHandle_t h;
+  CK(cudaIpcGetMemHandle(&h, c->cache));
+  memcpy(handle_out, &h, sizeof(h));
+  return GLB_OK;
+}
+
+glb_status glb_attach_peer_cache(glb_ctx* c, uint32_t peer, const void* ipc_handle,
+                                 const void* dev_ptr) {
+  ENTER(c);
+  if (c->shard_world < 2) return set_err(c, GLB_ESTATE, "cache is not sharded");
+  if (peer >= c->shard_world || peer == c->shard_rank)
+    return set_err(c, GLB_EINVAL, "peer %u (rank %u of %u)", peer, c->shard_rank, c->shard_world);
+  if (!ipc_handle == !dev_ptr) return set_err(c, GLB_EINVAL, "pass exactly one of ipc_handle, dev_ptr");
+  CK(sync_all(c));  // an in-flight extract may read the old mapping
+  if (c->shard_ipc[peer]) {
+    cudaIpcCloseMemHandle(c->shard_ipc[peer]);
+    c->shard_ipc[peer] = nullptr;
+  }
+  const void* base = dev_ptr;
+  if (ipc_handle) {
+    cudaIpcMemHandle_t h;
+    memcpy(&h, ipc_handle, sizeof(h));
+    void* p = nullptr;
+    CK(cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess));
+    c->shard_ipc[peer] = p;
+    base = p;
+  } else {
+    cudaPointerAttributes a;
+    CK(cudaPointerGetAttributes(&a, dev_ptr));
+    if (a.type != cudaMemoryTypeDevice) return set_err(c, GLB_EINVAL, "dev_ptr is not device memory");
+    if (a.device != c->device) {  // same process, another GPU: NVLink peer access
+      int ok = 0;
+      CK(cudaDeviceCanAccessPeer(&ok, c->device, a.device));
+      if (!ok) return set_err(c, GLB_EINVAL, "device %d cannot access device %d", c->device, a.device);
+      cudaError_t e = cudaDeviceEnablePeerAccess(a.device, 0);
+      if (e == cudaErrorPeerAccessAlreadyEnabled) cudaGetLastError();
+      else if (e != cudaSuccess) return cuda_fail(c, e, "cudaDeviceEnablePeerAccess");
+    }
+  }
+  c->shard_base[peer] = (const float*)base;
+  c->shard_attached |= 1u << peer;
+  return GLB_OK;
+}
+
+glb_status glb_last_extract_counts(glb_ctx* c, uint64_t* out3) {
+  ENTER(c);
+  if (!out3) return set_err(c, GLB_EINVAL, "null out");
+  CK(sync_all(c));
+  unsigned long long h[3];
+  CK(cudaMemcpy(h, c->xcount, sizeof(h), cudaMemcpyDeviceToHost));
+  out3[0] = h[0];
+  out3[1] = h[1];
+  out3[2] = c->shard_world > 1 ? h[2] : 0;
   return GLB_OK;
 }
 
@@ -774,6 +898,7 @@ glb_status glb_extract(glb_ctx* c, const uint32_t* vertices, uint64_t n, void* o
                        glb_extract_stats* stats) {
   ENTER(c);
   if (!c->V || !c->features_mapped) return set_err(c, GLB_ESTATE, "extract needs a graph with features");
+  if (!shards_ready(c)) return set_err(c, GLB_ESTATE, "peer cache shards not all attached");
   if (n && (!vertices || !out)) return set_err(c, GLB_EINVAL, "null pointer");
   if (n >= 0xFFFFFFFFull) return set_err(c, GLB_EINVAL, "n too large");
   if (n > c->xb.cap) {
@@ -795,7 +920,7 @@ glb_status glb_extract(glb_ctx* c, const uint32_t* vertices, uint64_t n, void* o
   CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->xb.hit_list, misses,
                    nullptr, &c->st_x->nhit, 0, 0));
   if (stats) {
-    CK(cudaMemcpyAsync(c->h_xcount, c->xcount, 2 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
+    CK(cudaMemcpyAsync(c->h_xcount, c->xcount, 3 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
     c->pending_stats = stats;
   }
   return GLB_OK;
@@ -805,6 +930,7 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
   ENTER(c);
   if (!c->have_sample) return set_err(c, GLB_ESTATE, "extract_sample without a current sample");
   if (!c->features_mapped) return set_err(c, GLB_ESTATE, "graph loaded without features");
+  if (!shards_ready(c)) return set_err(c, GLB_ESTATE, "peer cache shards not all attached");
   if (!out) return set_err(c, GLB_EINVAL, "null out");
   cudaStream_t main = c->stream;
   const int slot = c->cur;
@@ -841,7 +967,7 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
                       nullptr, &c->st->nhit, 0, 0);
   if (e == cudaSuccess && t1) e = cudaEventRecord(t1, c->stream);
   if (e == cudaSuccess && stats) {
-    e = cudaMemcpyAsync(c->h_xcount, c->xcount, 2 * sizeof(unsigned long long),
+    e = cudaMemcpyAsync(c->h_xcount, c->xcount, 3 * sizeof(unsigned long long),
                         cudaMemcpyDeviceToHost, c->stream);
     c->pending_stats = stats;
   }

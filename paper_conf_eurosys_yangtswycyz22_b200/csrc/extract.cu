@@ -28,6 +28,11 @@ constexpr unsigned kFull = 0xFFFFFFFFu;
 constexpr int kVecPerThread = 8;
 constexpr int kChunkUnits = kThreads * kVecPerThread;  // vectors per chunk
 
+struct ShardTab {
+  const void* base[kMaxShards];
+  uint32_t W, rank;
+};
+
 __device__ __forceinline__ uint32_t lanemask_lt() {
   uint32_t m;
   asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
@@ -76,16 +81,24 @@ __device__ __forceinline__ void st_row(T* p, T v) { __stcs(p, v); }
 // Work: hit chunks first (HBM, fast), then miss chunks (host, PCIe); chunks are
 // handed out by two device counters, so every block works on hits while there
 // are any and then every block keeps PCIe requests in flight.
-template <typename T>
+//
+// SHARD (NEXT-3, peer-sharded cache): a hit's slot is a global cache rank i, owned
+// by shard i % W at row i / W; tab.base[w] is shard w's rows (this GPU's own HBM or
+// a peer's, mapped over NVLink).  The owner is resolved once per entry when the
+// entry is staged, so the per-vector loop only indexes the shard table.
+template <typename T, bool SHARD>
 __global__ void __launch_bounds__(kThreads, 4)
     k_gather(T* __restrict__ out, const T* __restrict__ src_hit, const T* __restrict__ src_miss,
              const uint2* __restrict__ hit_list, const uint2* __restrict__ miss_list,
              const uint32_t* __restrict__ fill_src, const uint32_t* __restrict__ dev_counts,
              uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t R,
-             unsigned long long* xcount, unsigned int* work) {
+             unsigned long long* xcount, unsigned int* work, ShardTab tab) {
   pdl_enter();
   __shared__ uint2 ent[2][kThreads];
+  __shared__ const T* rowp[SHARD ? 2 : 1][SHARD ? kThreads : 1];  // SHARD: hit row address
   __shared__ unsigned int s_next;
+  uint32_t npeer = 0;
+  const T* e_row = nullptr;
   const uint64_t nh = dev_counts ? dev_counts[0] : nh_host;
   const uint64_t nm = dev_counts ? dev_counts[1] : nm_host;
   if (xcount && blockIdx.x == 0 && threadIdx.x == 0) {
@@ -112,14 +125,25 @@ __global__ void __launch_bounds__(kThreads, 4)
     const bool miss = g >= nch;
     const uint64_t r = (miss ? g - nch : g) * R + t;
     if (r >= (miss ? nm : nh)) return make_uint2(0u, 0u);
-    if (!miss) return __ldg(hit_list + r);
+    if (!miss) {
+      uint2 h = __ldg(hit_list + r);
+      if (SHARD) {
+        const uint32_t w = h.y % tab.W;
+        e_row = (const T*)tab.base[w] + (uint64_t)(h.y / tab.W) * U;
+        npeer += w != tab.rank;
+      }
+      return h;
+    }
     return fill_src ? make_uint2((uint32_t)r, __ldg(fill_src + r)) : __ldg(miss_list + r);
   };
   uint64_t g = claim();
   uint2 e = load_ent(g);
   int buf = 0;
   while (g < nch + ncm) {
-    if (t < R) ent[buf][t] = e;
+    if (t < R) {
+      ent[buf][t] = e;
+      if (SHARD) rowp[buf][t] = e_row;
+    }
     const uint64_t gn = claim();  // (its barrier also publishes ent[buf])
     e = load_ent(gn);             // prefetch the next chunk's entries
     const bool miss = g >= nch;
@@ -137,7 +161,8 @@ __global__ void __launch_bounds__(kThreads, 4)
           uint32_t row = (uint32_t)(((float)v + 0.5f) * inv_u);  // exact for v < 2^20
           const uint32_t col = v - row * U;
           const uint2 en = ent[buf][row];
-          x[q] = ld_row(src + (uint64_t)en.y * U + col);
+          if (SHARD && !miss) x[q] = ld_row(rowp[buf][row] + col);
+          else x[q] = ld_row(src + (uint64_t)en.y * U + col);
           dst[q] = (uint64_t)en.x * U + col;
         }
       }
@@ -149,6 +174,10 @@ __global__ void __launch_bounds__(kThreads, 4)
     }
     buf ^= 1;
     g = gn;
+  }
+  if (SHARD) {  // rows this launch read from other GPUs' shards
+    const uint32_t wsum = __reduce_add_sync(kFull, npeer);
+    if ((t & 31) == 0 && wsum && xcount) atomicAdd(&xcount[2], (unsigned long long)wsum);
   }
   // the last block out re-arms the counters for the next launch on this stream
   if (t == 0) {
@@ -258,14 +287,31 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   // chunk counters of the launching stream (this ctx's gathers are serial on it; each
   // launch leaves them zeroed for the next)
   unsigned int* work = c->stream == c->xstream ? c->work + 4 : c->work;
+  // sharded only for sample/extract gathers that read the cache (not the cache fill)
+  const bool shard = c->shard_world > 1 && src_hit == c->cache && hit_list;
+  ShardTab tab = {};
+  tab.W = c->shard_world;
+  tab.rank = c->shard_rank;
+  for (uint32_t w = 0; w < c->shard_world; ++w) tab.base[w] = c->shard_base[w];
   cudaError_t e;
-  if (vec)
-    e = launch_pdl(k_gather<float4>, grid, kThreads, c->stream, (float4*)out,
+  if (shard && (e = cudaMemsetAsync(c->xcount + 2, 0, sizeof(unsigned long long), c->stream)) != cudaSuccess)
+    return e;
+  if (vec && shard)
+    e = launch_pdl(k_gather<float4, true>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work);
+                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work, tab);
+  else if (vec)
+    e = launch_pdl(k_gather<float4, false>, grid, kThreads, c->stream, (float4*)out,
+                   (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
+                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work, tab);
+  else if (shard)
+    e = launch_pdl(k_gather<float, true>, grid, kThreads, c->stream, out, src_hit, src_miss,
+                   hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
+                   c->xcount, work, tab);
   else
-    e = launch_pdl(k_gather<float>, grid, kThreads, c->stream, out, src_hit, src_miss, hit_list,
-                   miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work);
+    e = launch_pdl(k_gather<float, false>, grid, kThreads, c->stream, out, src_hit, src_miss,
+                   hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
+                   c->xcount, work, tab);
   count_launch(c);
   return e;
 }

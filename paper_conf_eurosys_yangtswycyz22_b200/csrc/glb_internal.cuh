@@ -24,6 +24,7 @@ __host__ __device__ inline uint32_t compact_items(uint32_t flat, uint32_t num_sm
          : it > (uint32_t)kCompactItems ? (uint32_t)kCompactItems : it;
 }
 constexpr int kMaxFanout = 1024;
+constexpr int kMaxShards = 16;  // GLB_MAX_SHARDS: ranks of a peer-sharded cache (NEXT-3)
 constexpr int kMaxWalkLen = 8;
 
 // RNG domains (reading Q4): counter word 3 = epoch<<16 | hop<<8 | domain
@@ -159,6 +160,13 @@ struct glb_ctx {
   int32_t* slot = nullptr;     // i32[V]
   float* cache = nullptr;      // f32[C][D]
   uint64_t C = 0;
+  // NEXT-3 peer-sharded cache: global rank i < C is owned by shard i % W at row i / W;
+  // shard_base[r] = device pointer (valid in this process) of shard r's rows.
+  uint32_t shard_rank = 0, shard_world = 1;
+  uint64_t C_local = 0;            // rows of this ctx's own shard (== C when W == 1)
+  const float* shard_base[glb::kMaxShards] = {};
+  void* shard_ipc[glb::kMaxShards] = {};  // opened with cudaIpcOpenMemHandle (closed on rebuild)
+  uint32_t shard_attached = 0;     // bitmask of shards with a base pointer
   uint32_t* counts = nullptr;  // u32[V] PreSC hotness
   uint32_t* access = nullptr;  // u32[V] measured accesses
   int count_mode = GLB_COUNT_NONE;
@@ -210,7 +218,7 @@ struct glb_ctx {
   unsigned long long* shuf_keys = nullptr;
   uint32_t* shuf_vals = nullptr;
   glb_extract_stats* pending_stats = nullptr;
-  unsigned long long* xcount = nullptr;      // device [2] hits/misses of the last extract
+  unsigned long long* xcount = nullptr;      // device [3] hits/misses/peer hits of the last extract
   unsigned long long* h_xcount = nullptr;    // pinned mirror
 
   // radix sort scratch
@@ -296,6 +304,9 @@ cudaError_t launch_max_u32(glb_ctx* c, const uint32_t* a, uint64_t n, uint32_t* 
 cudaError_t launch_rank_keys(glb_ctx* c, const uint32_t* hot, uint32_t maxc, uint32_t* keys,
                              uint32_t* vals);
 cudaError_t launch_assign_slots(glb_ctx* c, const uint32_t* order, uint64_t C);
+// out[j] = order[j*W + r] for j < n (the vertices of shard r of a peer-sharded cache)
+cudaError_t launch_shard_rows(glb_ctx* c, const uint32_t* order, uint32_t W, uint32_t r,
+                              uint64_t n, uint32_t* out);
 cudaError_t launch_vmap_reset(glb_ctx* c);   // gp = ~0, slot = c->slot[v]
 cudaError_t launch_policy_hotness(glb_ctx* c, int policy, uint64_t seed, uint32_t* out);
 cudaError_t launch_topmark(glb_ctx* c, const uint32_t* order, uint64_t C, uint8_t* flag);

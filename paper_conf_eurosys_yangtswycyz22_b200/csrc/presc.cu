@@ -238,6 +238,15 @@ __global__ void k_assign_slots(const uint32_t* __restrict__ order, uint64_t C, i
     slot[order[i]] = (int32_t)i;
 }
 
+// NEXT-3: the vertices of shard r of a peer-sharded cache, in local-row order
+// (global rank i = j*W + r is local row j of shard r).
+__global__ void k_shard_rows(const uint32_t* __restrict__ order, uint32_t W, uint32_t r,
+                             uint64_t n, uint32_t* __restrict__ out) {
+  for (uint64_t j = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; j < n;
+       j += (uint64_t)gridDim.x * blockDim.x)
+    out[j] = order[j * W + r];
+}
+
 __global__ void k_vmap_reset(VEntry* __restrict__ vmap, const int32_t* __restrict__ slot,
                              uint64_t n) {
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
@@ -529,6 +538,14 @@ cudaError_t launch_rank_keys(glb_ctx* c, const uint32_t* hot, uint32_t maxc, uin
 cudaError_t launch_assign_slots(glb_ctx* c, const uint32_t* order, uint64_t C) {
   if (C == 0) return cudaSuccess;
   k_assign_slots<<<grid_for(c), kThreads, 0, c->stream>>>(order, C, c->slot);
+  count_launch(c);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_shard_rows(glb_ctx* c, const uint32_t* order, uint32_t W, uint32_t r,
+                              uint64_t n, uint32_t* out) {
+  if (n == 0) return cudaSuccess;
+  k_shard_rows<<<grid_for(c), kThreads, 0, c->stream>>>(order, W, r, n, out);
   count_launch(c);
   return cudaGetLastError();
 }

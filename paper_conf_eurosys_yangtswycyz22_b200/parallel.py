@@ -57,6 +57,25 @@ def presample_dp(ctx, K: int, rank: int, world: int, group=None):
     allreduce_counts(ctx.counts_tensor(1), group)
 
 
+def build_sharded_cache(ctx, alpha: float, rank: int, world: int, group=None):
+    """NEXT-3: each rank caches floor(alpha*V) distinct rows -- the
+    ranks i with i % world == rank of the PreSC order -- and maps every other rank's
+    shard through CUDA IPC (over NVLink on a multi-GPU box), so the group caches
+    world*alpha*|V| rows instead of alpha*|V| replicated ones.  The handles travel as
+    64-byte blobs over the process group; the closing barrier guarantees every shard is
+    mapped before anyone extracts.  Callers must barrier again before any rank rebuilds
+    or frees its shard (peers may still be reading it)."""
+    ctx.build_cache_sharded(alpha, rank, world)
+    if world == 1:
+        return
+    handles = [None] * world
+    dist.all_gather_object(handles, ctx.cache_ipc_handle(), group=group)
+    for p, h in enumerate(handles):
+        if p != rank:
+            ctx.attach_peer_cache(p, ipc_handle=h)
+    dist.barrier(group=group)
+
+
 # ----------------------------------------------------------------------------- factored
 def num_samplers(n_gpus: int, t_sample: float, t_train: float) -> int:
     """Ns = ceil(Ng / (K + 1)), K = Tt / Ts; at least one of each

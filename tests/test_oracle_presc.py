@@ -173,3 +173,35 @@ def test_presc_vs_degree_and_random_on_tiny():
           ("random", oracle.hotness_random(g.seed, g.V))]}
     assert h["presc"] > 2 * h["random"]
     assert h["presc"] > 0.95 * h["degree"]
+
+
+def test_sharded_cache_pins():
+    """NEXT-3: world shards of floor(alpha*V) rows each hold exactly the
+    world*floor(alpha*V) top-ranked vertices (a brute-force sort), disjointly, shard r
+    holding the ranks i = r, r+world, ... in row order; world = 1 is load_cache itself."""
+    rng = np.random.default_rng(9)
+    counts = rng.integers(0, 7, 150).astype(np.uint32)
+    ranked = brute_rank(counts)
+    for alpha in [0.0, 0.02, 0.1, 0.2, 0.5, 1.0]:
+        slot1, sh1 = oracle.sharded_cache(counts, alpha, 1)
+        assert np.array_equal(slot1, oracle.cache_slots(counts, alpha))
+        for world in [2, 3, 8]:
+            slot, shards = oracle.sharded_cache(counts, alpha, world)
+            C = min(150, world * int(alpha * 150))
+            members = [v for s in shards for v in s.tolist()]
+            assert sorted(members) == sorted(ranked[:C])            # the top C, disjoint
+            assert sorted(slot[slot >= 0].tolist()) == list(range(C))
+            for r, s in enumerate(shards):
+                assert s.tolist() == [ranked[i] for i in range(r, C, world)]
+                assert all(int(slot[v]) % world == r for v in s.tolist())
+            if world * alpha >= 1.0:
+                assert C == 150 and np.all(slot >= 0)               # every row cached somewhere
+
+
+def test_extract_counts_pins():
+    slot = np.array([-1, 0, 1, 2, 3, -1, 4], np.int32)              # 5 cached rows over 2 shards
+    ids = np.array([0, 1, 2, 3, 4, 5, 6, 6, 1], np.uint32)
+    assert oracle.extract_counts(ids, slot) == (7, 2, 0)
+    # shard 0 holds slots 0, 2, 4 (vertices 1, 3, 6); shard 1 slots 1, 3 (vertices 2, 4)
+    assert oracle.extract_counts(ids, slot, 0, 2) == (7, 2, 2)      # vertices 2 and 4
+    assert oracle.extract_counts(ids, slot, 1, 2) == (7, 2, 5)      # 1, 3, 6, 6, 1
