@@ -94,11 +94,15 @@ __global__ void __launch_bounds__(kThreads, 4)
              uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t R,
              unsigned long long* xcount, unsigned int* work, ShardTab tab) {
   pdl_enter();
-  __shared__ uint2 ent[2][kThreads];
-  __shared__ const T* rowp[SHARD ? 2 : 1][SHARD ? kThreads : 1];  // SHARD: hit row address
+  // staged work entry: source row address and destination element offset, resolved once
+  // per row so the per-vector loop is one LDS.128 + two adds
+  struct __align__(16) RowEnt {
+    const T* src;
+    unsigned long long dst;
+  };
+  __shared__ RowEnt ent[2][kThreads];
   __shared__ unsigned int s_next;
   uint32_t npeer = 0;
-  const T* e_row = nullptr;
   const uint64_t nh = dev_counts ? dev_counts[0] : nh_host;
   const uint64_t nm = dev_counts ? dev_counts[1] : nm_host;
   if (xcount && blockIdx.x == 0 && threadIdx.x == 0) {
@@ -120,50 +124,54 @@ __global__ void __launch_bounds__(kThreads, 4)
     __syncthreads();
     return g;
   };
+  // raw work-list entry of this thread in chunk g (kept in 2 registers while the current
+  // chunk's rows are in flight) ...
   auto load_ent = [&](uint64_t g) -> uint2 {
     if (g >= nch + ncm || t >= R) return make_uint2(0u, 0u);
     const bool miss = g >= nch;
     const uint64_t r = (miss ? g - nch : g) * R + t;
     if (r >= (miss ? nm : nh)) return make_uint2(0u, 0u);
-    if (!miss) {
-      uint2 h = __ldg(hit_list + r);
-      if (SHARD) {
-        const uint32_t w = h.y % tab.W;
-        e_row = (const T*)tab.base[w] + (uint64_t)(h.y / tab.W) * U;
-        npeer += w != tab.rank;
-      }
-      return h;
-    }
+    if (!miss) return __ldg(hit_list + r);
     return fill_src ? make_uint2((uint32_t)r, __ldg(fill_src + r)) : __ldg(miss_list + r);
+  };
+  // ... and resolved to (source row address, destination offset) when staged
+  auto stage = [&](uint64_t g, uint2 h) -> RowEnt {
+    RowEnt re;
+    if (g >= nch) {
+      re.src = src_miss + (uint64_t)h.y * U;
+    } else if (SHARD) {
+      const uint32_t w = h.y % tab.W;
+      re.src = (const T*)tab.base[w] + (uint64_t)(h.y / tab.W) * U;
+      npeer += (w != tab.rank) && (g * R + t < nh);
+    } else {
+      re.src = src_hit + (uint64_t)h.y * U;
+    }
+    re.dst = (unsigned long long)h.x * U;
+    return re;
   };
   uint64_t g = claim();
   uint2 e = load_ent(g);
   int buf = 0;
   while (g < nch + ncm) {
-    if (t < R) {
-      ent[buf][t] = e;
-      if (SHARD) rowp[buf][t] = e_row;
-    }
+    if (t < R) ent[buf][t] = stage(g, e);
     const uint64_t gn = claim();  // (its barrier also publishes ent[buf])
     e = load_ent(gn);             // prefetch the next chunk's entries
     const bool miss = g >= nch;
-    const T* src = miss ? src_miss : src_hit;
     const uint64_t c = miss ? g - nch : g;
     const uint64_t rows = min((uint64_t)R, (miss ? nm : nh) - c * R);
     const uint32_t total = (uint32_t)rows * U;
     for (uint32_t base = 0; base < total; base += kChunkUnits) {
       T x[kVecPerThread];
-      uint64_t dst[kVecPerThread];
+      unsigned long long dst[kVecPerThread];
 #pragma unroll
       for (int q = 0; q < kVecPerThread; ++q) {
         const uint32_t v = base + q * kThreads + t;
         if (v < total) {
           uint32_t row = (uint32_t)(((float)v + 0.5f) * inv_u);  // exact for v < 2^20
           const uint32_t col = v - row * U;
-          const uint2 en = ent[buf][row];
-          if (SHARD && !miss) x[q] = ld_row(rowp[buf][row] + col);
-          else x[q] = ld_row(src + (uint64_t)en.y * U + col);
-          dst[q] = (uint64_t)en.x * U + col;
+          const RowEnt en = ent[buf][row];
+          x[q] = ld_row(en.src + col);
+          dst[q] = en.dst + col;
         }
       }
 #pragma unroll

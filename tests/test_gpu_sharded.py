@@ -65,8 +65,7 @@ def test_sharded_extract_sample_bit_exact(tiny, world, alpha, mode):
         ptr, rows = c.cache_device_ptr()
         assert rows == shards[r].shape[0]
         if rows:  # the shard's rows are exactly the oracle's feature rows
-            view = torch.as_tensor(glb._CAI(ptr, (rows * g.shape.D,), "<f4", c, None),
-                                   device="cuda:0").view(rows, g.shape.D)
+            view = glb._view(ptr, rows * g.shape.D, "<f4", c, c.device).view(rows, g.shape.D)
             assert np.array_equal(view.cpu().numpy().view(np.uint32),
                                   go.extract(shards[r]).view(np.uint32))
     e = 1

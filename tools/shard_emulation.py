@@ -20,7 +20,7 @@ import synth  # noqa: E402
 ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="PR")
 ap.add_argument("--world", type=int, default=8)
-ap.add_argument("--alpha", type=float, default=0.125)
+ap.add_argument("--alpha", type=float, default=0.126)  # W*floor(alpha*V) >= V: no misses
 ap.add_argument("--steps", type=int, default=200)
 args = ap.parse_args()
 
