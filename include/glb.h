@@ -145,6 +145,13 @@ glb_status glb_sample(glb_ctx* ctx, const uint32_t* seeds, uint32_t num_seeds,
  * Visit counts are recorded per the count mode.  Use glb_sample_result to read
  * sizes (synchronises), or glb_extract_sample to gather features directly. */
 glb_status glb_sample_batch(glb_ctx* ctx, uint32_t epoch, uint32_t batch);
+/* Sample caller-provided seeds with the ctx sampler, ASYNCHRONOUSLY (no host sync): a host
+ * `seeds` buffer is copied to the device on the ctx stream (truly asynchronous when it is
+ * pinned; it must stay unchanged until the stream reaches the copy), a device buffer is
+ * read in place.  Errors found on the device (duplicate seed, id >= V) surface at the next
+ * glb_sync / glb_sample_result.  Errors: ESTATE, EINVAL, ENOMEM (n > max_batch), ERANGE. */
+glb_status glb_sample_async(glb_ctx* ctx, const uint32_t* seeds, uint32_t num_seeds,
+                            uint64_t seed, uint32_t epoch, uint32_t batch);
 glb_status glb_sample_result(glb_ctx* ctx, glb_blocks* out);
 
 /* ---------------------------------------------------------------- PreSC (a5, a6)
@@ -215,6 +222,10 @@ glb_status glb_attach_peer_cache(glb_ctx* ctx, uint32_t peer, const void* ipc_ha
 /* Counts of the last extract: out[0] = cache hits (local + peer shards), out[1] = host
  * misses, out[2] = hits served by another GPU's shard (0 unless sharded).  Synchronous. */
 glb_status glb_last_extract_counts(glb_ctx* ctx, uint64_t* out3);
+/* Device u64[3] (hits, misses, peer hits) that every extract rewrites on the ctx stream:
+ * copy it device->host after an extract (stream-ordered) to read that extract's counts
+ * without a synchronisation.  Peer hits are valid only for a sharded cache. */
+glb_status glb_extract_counts_device_ptr(glb_ctx* ctx, void** out);
 
 /* Hit-rate statistics over the recorded accesses (GLB_COUNT_ACCESS) for the
  * current cache: total accesses, accesses served by the cache (H = hits/total),

@@ -39,6 +39,7 @@ EXPORTS = [
     "glb_set_relabel_mode", "glb_relabel_mode", "glb_policy_hotness", "glb_footprint_similarity",
     "glb_load_edge_weights", "glb_build_cache_sharded", "glb_cache_device_ptr",
     "glb_cache_ipc_handle", "glb_attach_peer_cache", "glb_last_extract_counts",
+    "glb_sample_async", "glb_extract_counts_device_ptr",
 ]
 MAX_SHARDS = 16
 IPC_HANDLE_BYTES = 64
@@ -131,6 +132,8 @@ def lib(auto_build: bool = True):
         "glb_cache_ipc_handle": ([vp, vp], i32),
         "glb_attach_peer_cache": ([vp, u32, vp, vp], i32),
         "glb_last_extract_counts": ([vp, ctypes.POINTER(u64)], i32),
+        "glb_sample_async": ([vp, vp, u32, u64, u32, u32], i32),
+        "glb_extract_counts_device_ptr": ([vp, ctypes.POINTER(vp)], i32),
         "glb_footprint_similarity": ([vp, vp, vp, dbl, ctypes.POINTER(u64), ctypes.POINTER(u64),
                                       ctypes.POINTER(dbl)], i32),
     }
@@ -322,6 +325,24 @@ class Context:
     def sample_batch(self, epoch: int, batch: int):
         """Asynchronous: sample batch ``batch`` of epoch ``epoch`` (device-resident shuffle)."""
         self._ck(self._lib.glb_sample_batch(self._h, epoch, batch))
+
+    def sample_async(self, seeds, seed=0, epoch=0, batch=0):
+        """Asynchronous sample of caller seeds with the ctx sampler: a pinned CPU int32 tensor
+        (H2D copy on the ctx stream; keep it unchanged until the stream has consumed it) or
+        a CUDA int32 tensor.  Read the blocks with sample_result() (synchronises)."""
+        import torch
+        assert isinstance(seeds, torch.Tensor) and seeds.dtype == torch.int32
+        assert seeds.is_contiguous() and (seeds.is_cuda or seeds.is_pinned())
+        self._ck(self._lib.glb_sample_async(self._h, seeds.data_ptr(), seeds.numel(), seed,
+                                            epoch, batch))
+
+    def extract_counts_tensor(self):
+        """Zero-copy int64 CUDA view [3] = (hits, misses, peer hits) of the last extract,
+        rewritten on the ctx stream by every extract (copy it out stream-ordered)."""
+        import torch
+        p = ctypes.c_void_p()
+        self._ck(self._lib.glb_extract_counts_device_ptr(self._h, ctypes.byref(p)))
+        return torch.as_tensor(_CAI(p.value, (3,), "<i8", self), device=self.device)
 
     def sample_result(self) -> Blocks:
         b = _Blocks()

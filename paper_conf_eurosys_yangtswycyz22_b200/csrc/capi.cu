@@ -589,6 +589,31 @@ glb_status glb_sample(glb_ctx* c, const uint32_t* seeds, uint32_t n0, const uint
   return glb_sample_result(c, out);
 }
 
+glb_status glb_sample_async(glb_ctx* c, const uint32_t* seeds, uint32_t n0, uint64_t seed,
+                            uint32_t epoch, uint32_t batch) {
+  ENTER(c);
+  if (!c->V || !c->sampler_set) return set_err(c, GLB_ESTATE, "sample before load_graph/set_sampler");
+  if (n0 && !seeds) return set_err(c, GLB_EINVAL, "null seeds");
+  if (n0 > c->sb.cap_batch) return set_err(c, GLB_ENOMEM, "batch %u > max_batch %u", n0, c->sb.cap_batch);
+  const uint32_t* sd = seeds;
+  cudaPointerAttributes at;
+  const bool on_dev = n0 && cudaPointerGetAttributes(&at, seeds) == cudaSuccess &&
+                      at.type == cudaMemoryTypeDevice;
+  (void)cudaGetLastError();
+  if (!on_dev) {  // stream-ordered H2D (asynchronous when the host buffer is pinned)
+    if (n0) CK(cudaMemcpyAsync(c->sb.seeds, seeds, sizeof(uint32_t) * n0, cudaMemcpyHostToDevice, c->stream));
+    sd = c->sb.seeds;
+  }
+  return enqueue_sample(c, sd, n0, c->kind, c->fanouts, c->L, seed, epoch, batch);
+}
+
+glb_status glb_extract_counts_device_ptr(glb_ctx* c, void** out) {
+  ENTER(c);
+  if (!out) return set_err(c, GLB_EINVAL, "null out");
+  *out = c->xcount;
+  return GLB_OK;
+}
+
 glb_status glb_sample_batch(glb_ctx* c, uint32_t epoch, uint32_t b) {
   ENTER(c);
   if (!c->V || !c->sampler_set || !c->train_set) return set_err(c, GLB_ESTATE, "sample_batch needs graph, sampler, train set");

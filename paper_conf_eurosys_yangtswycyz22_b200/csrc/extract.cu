@@ -72,8 +72,48 @@ __global__ void __launch_bounds__(kThreads)
   }
 }
 
+// Feature-row loads.  GLB_GATHER_LD 0: __ldg; 1: ld.global.cs (evict-first in L1/L2);
+// 2: ld.global.nc.L1::no_allocate with an L2 evict_first policy -- the gather streams
+// hundreds of MB through L2 per batch, and evict-first keeps the next batch's relabel
+// table / CSR offsets resident.
+#ifndef GLB_GATHER_LD
+#define GLB_GATHER_LD 0
+#endif
+__device__ __forceinline__ uint64_t l2_evict_first_policy() {
+  uint64_t pol = 0;
+#if GLB_GATHER_LD == 2
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+#endif
+  return pol;
+}
 template <typename T>
-__device__ __forceinline__ T ld_row(const T* p) { return __ldg(p); }
+__device__ __forceinline__ T ld_row(const T* p, uint64_t pol);
+template <>
+__device__ __forceinline__ float4 ld_row<float4>(const float4* p, uint64_t pol) {
+#if GLB_GATHER_LD == 2
+  float4 v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pol));
+  return v;
+#elif GLB_GATHER_LD == 1
+  return __ldcs(p);
+#else
+  return __ldg(p);
+#endif
+}
+template <>
+__device__ __forceinline__ float ld_row<float>(const float* p, uint64_t pol) {
+#if GLB_GATHER_LD == 2
+  float v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;"
+               : "=f"(v) : "l"(p), "l"(pol));
+  return v;
+#elif GLB_GATHER_LD == 1
+  return __ldcs(p);
+#else
+  return __ldg(p);
+#endif
+}
 template <typename T>
 __device__ __forceinline__ void st_row(T* p, T v) { __stcs(p, v); }
 
@@ -112,6 +152,7 @@ __global__ void __launch_bounds__(kThreads, 4)
   const uint32_t t = threadIdx.x;
   const uint64_t nch = (nh + R - 1) / R, ncm = (nm + R - 1) / R;  // hit / miss chunks
   const float inv_u = 1.0f / (float)U;
+  const uint64_t pol = l2_evict_first_policy();
   // chunk id g: g < nch -> hit chunk g; else miss chunk g - nch
   auto claim = [&]() -> uint64_t {
     if (t == 0) {
@@ -170,7 +211,7 @@ __global__ void __launch_bounds__(kThreads, 4)
           uint32_t row = (uint32_t)(((float)v + 0.5f) * inv_u);  // exact for v < 2^20
           const uint32_t col = v - row * U;
           const RowEnt en = ent[buf][row];
-          x[q] = ld_row(en.src + col);
+          x[q] = ld_row(en.src + col, pol);
           dst[q] = en.dst + col;
         }
       }

@@ -30,12 +30,30 @@ extern "C" glb_status glb_trace_dump(void* host, size_t bytes) {
   return cudaMemcpyFromSymbol(host, g_trace, bytes) == cudaSuccess ? GLB_OK : GLB_ECUDA;
 }
 __device__ __forceinline__ unsigned long long gtime() {
-  return (unsigned long long)clock64();  // SM cycles (relative deltas within a tile)
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));  // ns, comparable across SMs
+  return t;
 }
+// [hop][0] = first block start, [hop][1] = last block end of k_khop (ns)
+__device__ unsigned long long g_ktrace[GLB_MAX_HOPS][2];
+extern "C" glb_status glb_trace_reset() {
+  unsigned long long h[GLB_MAX_HOPS][2];
+  for (int i = 0; i < GLB_MAX_HOPS; ++i) { h[i][0] = ~0ull; h[i][1] = 0; }
+  static unsigned long long z[GLB_MAX_HOPS][4096][8];
+  if (cudaMemcpyToSymbol(g_trace, z, sizeof(z)) != cudaSuccess) return GLB_ECUDA;
+  return cudaMemcpyToSymbol(g_ktrace, h, sizeof(h)) == cudaSuccess ? GLB_OK : GLB_ECUDA;
+}
+extern "C" glb_status glb_ktrace_dump(void* host) {
+  return cudaMemcpyFromSymbol(host, g_ktrace, sizeof(g_ktrace)) == cudaSuccess ? GLB_OK : GLB_ECUDA;
+}
+#define KTRACE_BEGIN(h) do { if (threadIdx.x == 0) atomicMin(&::g_ktrace[h][0], gtime()); } while (0)
+#define KTRACE_END(h) do { __syncthreads(); if (threadIdx.x == 0) atomicMax(&::g_ktrace[h][1], gtime()); } while (0)
 #define TRACE(h, t, ev) \
   do { if (threadIdx.x == 0 && (t) < 4096) ::g_trace[h][t][ev] = gtime(); } while (0)
 #else
 #define TRACE(h, t, ev) do {} while (0)
+#define KTRACE_BEGIN(h) do {} while (0)
+#define KTRACE_END(h) do {} while (0)
 #endif
 
 namespace glb {
@@ -227,6 +245,7 @@ __global__ void __launch_bounds__(kThreads)
            const uint32_t* __restrict__ indices, const uint32_t* __restrict__ uniq,
            uint32_t* __restrict__ picks, uint32_t* __restrict__ pidx, uint32_t* fix_ind) {
   pdl_enter();
+  KTRACE_BEGIN(hop);
   if (fix_ind) fixup_block(st->nnz[hop - 1], T.e, fix_ind);  // deferred lids of block hop-1
   const uint32_t gen = T.gen;
   const uint32_t n_l = st->n[hop];
@@ -294,6 +313,7 @@ __global__ void __launch_bounds__(kThreads)
       if (HASH) pidx[(size_t)d * k + s] = idx;
     }
   }
+  KTRACE_END(hop);
 }
 
 // ---------------------------------------------------------------- weighted k-hop (NEXT-1)
@@ -527,6 +547,10 @@ __global__ void __launch_bounds__(kThreads)
 constexpr unsigned long long kFlagAgg = 1ull << 62;
 constexpr unsigned long long kFlagInc = 2ull << 62;
 constexpr unsigned long long kValMask = (1ull << 62) - 1;
+#ifndef GLB_LOOKBACK
+#define GLB_LOOKBACK 8
+#endif
+constexpr int kLookback = GLB_LOOKBACK;  // look-back window = 32 * kLookback tiles
 
 __device__ __forceinline__ unsigned long long pack_status(unsigned long long flag,
                                                           unsigned long long pair) {
@@ -685,23 +709,52 @@ __global__ void __launch_bounds__(kThreads, 3)
         if (lane == 0) atomicExch(status + 0, pack_status(kFlagInc, agg));
       } else {
         if (lane == 0) atomicExch(status + tile, pack_status(kFlagAgg, agg));
+        // Look-back over a window of 32*kLookback predecessors at once (entry o = q*32 +
+        // lane is tile idx - o): all its status words are loaded together and re-polled
+        // until published, so an inclusive prefix propagates kLookback*32 tiles per L2
+        // round trip instead of 32 (the chain dominated small hops).
         long long idx = (long long)tile - 1;
         for (;;) {
-          const long long jx = idx - lane;
-          unsigned long long wv = kFlagInc;
-          if (jx >= 0) {
-            do {
-              wv = *((volatile unsigned long long*)(status + jx));
-            } while ((wv >> 62) == 0);
+          unsigned long long wv[kLookback];
+#pragma unroll
+          for (int q = 0; q < kLookback; ++q) {
+            const long long jx = idx - (q * 32 + lane);
+            wv[q] = jx >= 0 ? (unsigned long long)*((volatile unsigned long long*)(status + jx))
+                            : (unsigned long long)kFlagInc;
           }
-          const uint32_t incm = __ballot_sync(kFull, (wv >> 62) >= 2);
-          if (incm) {
-            const int firsti = __ffs(incm) - 1;
-            excl += warp_sum64(lane <= firsti ? unpack_pair(wv) : 0ull);
+          for (;;) {
+            bool pending = false;
+#pragma unroll
+            for (int q = 0; q < kLookback; ++q) pending |= (wv[q] >> 62) == 0;
+            if (!__any_sync(kFull, pending)) break;
+#pragma unroll
+            for (int q = 0; q < kLookback; ++q)
+              if ((wv[q] >> 62) == 0)
+                wv[q] = *((volatile unsigned long long*)(status + idx - (q * 32 + lane)));
+          }
+          int qmin = -1;
+          uint32_t incm = 0;
+#pragma unroll
+          for (int q = 0; q < kLookback; ++q) {
+            const uint32_t b = __ballot_sync(kFull, (wv[q] >> 62) >= 2);
+            if (qmin < 0 && b) {
+              qmin = q;
+              incm = b;
+            }
+          }
+          unsigned long long part = 0;
+          if (qmin >= 0) {  // nearest inclusive prefix: entry (qmin, first lane of incm)
+            const int lmin = __ffs(incm) - 1;
+#pragma unroll
+            for (int q = 0; q < kLookback; ++q)
+              if (q < qmin || (q == qmin && lane <= lmin)) part += unpack_pair(wv[q]);
+            excl += warp_sum64(part);
             break;
           }
-          excl += warp_sum64(unpack_pair(wv));
-          idx -= 32;
+#pragma unroll
+          for (int q = 0; q < kLookback; ++q) part += unpack_pair(wv[q]);
+          excl += warp_sum64(part);
+          idx -= 32 * kLookback;
         }
         if (lane == 0) atomicExch(status + tile, pack_status(kFlagInc, excl + agg));
       }

@@ -397,3 +397,39 @@ def test_weighted_khop_parity(fanouts, mode):
     ctx.presample(1)
     exp = go.presample("weighted", g.train, 64, fanouts, g.seed, 1, weights=w)
     assert np.array_equal(ctx.get_counts(glb.COUNT_PRESAMPLE), exp)
+
+
+def test_sample_async_pinned_seeds_and_device_counts(tiny):
+    """glb_sample_async (pinned host or device seeds, no host sync) gives the oracle's
+    sample; glb_extract_counts_device_ptr holds each extract's (hits, misses) in stream
+    order (the e2e bench path)."""
+    g, go = tiny
+    sh = g.shape
+    ctx = make_ctx(g, fanouts=sh.fanouts)
+    ctx.set_count_mode(glb.COUNT_PRESAMPLE)
+    ctx.presample(1)
+    ctx.set_count_mode(glb.COUNT_NONE)
+    ctx.build_cache(0.2)
+    slot = ctx.cache_slots()
+    cnt = ctx.extract_counts_tensor()
+    host = torch.zeros((3, 3), dtype=torch.int64).pin_memory()
+    outs = []
+    batches = oracle.epoch_batches(g.train, sh.batch, g.seed, 4)
+    for j, b in enumerate([0, 5, len(batches) - 1]):
+        seeds = torch.from_numpy(batches[b].view(np.int32).copy())
+        seeds = seeds.pin_memory() if j != 1 else seeds.cuda()
+        ctx.sample_async(seeds, seed=g.seed, epoch=4, batch=b)
+        s = ctx.sample_result()
+        exp = go.sample_khop(batches[b], sh.fanouts, g.seed, 4, b)
+        assert_same_sample(s, exp)
+        out = torch.empty((s.sizes[-1], sh.D), device="cuda")
+        ctx.extract_sample(out)
+        host[j].copy_(cnt, non_blocking=True)
+        outs.append((exp.uniq, out))
+    torch.cuda.synchronize()
+    for j, (uniq, out) in enumerate(outs):
+        hits = int((slot[uniq] >= 0).sum())
+        assert host[j].tolist() == [hits, len(uniq) - hits, 0]
+        assert np.array_equal(out.cpu().numpy().view(np.uint32), go.extract(uniq).view(np.uint32))
+    with pytest.raises(AssertionError):
+        ctx.sample_async(torch.from_numpy(batches[0].view(np.int32).copy()))  # pageable
