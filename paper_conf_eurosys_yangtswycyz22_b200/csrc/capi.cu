@@ -717,9 +717,20 @@ static glb_status build_cache_impl(glb_ctx* c, uint64_t C, const uint32_t* hotne
   c->shard_rank = rank;
   c->shard_world = world;
   const uint64_t Cl = C > rank ? (C - rank + world - 1) / world : 0;  // rows i = j*world + rank
+  // cache row stride: D floats, padded to GLB_CACHE_ALIGN bytes for 16-byte-vector rows
+#ifndef GLB_CACHE_ALIGN
+#define GLB_CACHE_ALIGN 0
+#endif
+  c->cache_stride = c->D;
+#if GLB_CACHE_ALIGN
+  if (c->D % 4 == 0) {
+    const uint32_t a = GLB_CACHE_ALIGN / 4;
+    c->cache_stride = (c->D + a - 1) / a * a;
+  }
+#endif
   c->C_local = Cl;
   if (c->features_mapped && (Cl || world > 1)) {
-    CK(dalloc(&c->cache, Cl * (uint64_t)c->D));  // >= 1 element: a shard always has a base
+    CK(dalloc(&c->cache, Cl * (uint64_t)c->cache_stride));  // >= 1 element: a shard always has a base
     const uint32_t* rows = order;
     if (world > 1) {
       uint32_t* sub = tmp + 4 * V;

@@ -152,3 +152,45 @@ def test_header_payload_roundtrip():
     assert torch.equal(uniq, b.uniq) and all(torch.equal(a, c) for a, c in zip(ip, b.indptr))
     assert all(torch.equal(a, c) for a, c in zip(ix, b.indices))
     assert all(torch.equal(a, c) for a, c in zip(ws, b.weights))
+
+
+class _ShardCtx:
+    """Stand-in ctx for parallel.build_sharded_cache: records the build and the attaches."""
+
+    def __init__(self, rank):
+        self.rank = rank
+        self.built = None
+        self.attached = {}
+
+    def build_cache_sharded(self, alpha, rank, world):
+        self.built = (alpha, rank, world)
+
+    def cache_ipc_handle(self):
+        return bytes([self.rank]) * 64  # a 64-byte opaque blob, unique per rank
+
+    def attach_peer_cache(self, peer, ipc_handle=None, dev_ptr=None):
+        assert dev_ptr is None and len(ipc_handle) == 64
+        self.attached[peer] = ipc_handle
+
+
+def _shard_worker(rank, world, port, out):
+    _init(rank, world, port)
+    c = _ShardCtx(rank)
+    par.build_sharded_cache(c, 0.125, rank, world)
+    ok = c.built == (0.125, rank, world) and sorted(c.attached) == [p for p in range(world)
+                                                                     if p != rank]
+    ok = ok and all(h == bytes([p]) * 64 for p, h in c.attached.items())
+    t = torch.tensor([1 if ok else 0])
+    dist.all_reduce(t)
+    if rank == 0:
+        torch.save(t, out)
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_sharded_cache_handle_exchange(tmp_path, world):
+    """NEXT-3: every rank builds its shard and maps every other rank's shard from the
+    all-gathered IPC handles (gloo, CPU; the CUDA side is tests/test_gpu_sharded.py)."""
+    out = str(tmp_path / "ok.pt")
+    mp.spawn(_shard_worker, args=(world, free_port(), out), nprocs=world, join=True)
+    assert int(torch.load(out)[0]) == world
