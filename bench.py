@@ -47,7 +47,10 @@ def parse():
     p.add_argument("--no-sweep", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
-    p.add_argument("--measure-epochs", type=int, default=2)
+    p.add_argument("--measure-epochs", type=int, default=10,
+                   help="epochs whose accesses define H and the Optimal H* (L148 fn4)")
+    p.add_argument("--k-sweep", default="1,2,3",
+                   help="PreSC#K values for the Fig 11(a) analog (empty: skip)")
     p.add_argument("--mode", default="dp", choices=["dp", "factored"],
                    help="factored: Ns sampler + Nt trainer ranks (PAPER.md §5.2-5.3)")
     p.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
@@ -59,7 +62,9 @@ def parse():
     p.add_argument("--cache", default="replicated", choices=["replicated", "sharded"],
                    help="sharded: each rank caches alpha*V distinct rows, peers read them over "
                         "NVLink (NEXT-3; glb_build_cache_sharded)")
-    p.add_argument("--pipeline", type=int, default=1, choices=[1, 2],
+    p.add_argument("--time-every", type=int, default=8,
+                   help="CUDA events around every n-th extract launch of the timed region")
+    p.add_argument("--pipeline", type=int, default=2, choices=[1, 2],
                    help="2: extract of batch b overlaps sampling of batch b+1 (two streams)")
     return p.parse_args()
 
@@ -417,7 +422,7 @@ def main():
     launches0 = ctx.launches
     barrier()
     torch.cuda.synchronize()
-    ctx.set_timing(True)
+    ctx.set_timing(args.time_every)  # events around every time_every-th extract launch
     clocks.start()
     t_start = torch.cuda.Event(enable_timing=True)
     t_end = torch.cuda.Event(enable_timing=True)
@@ -463,8 +468,36 @@ def main():
     # algorithmic HBM bytes of the extract launch: per row read (hit: cache row from
     # HBM) + write of the out row + the 8-byte (dst, src) work-list entry.
     hbm_bytes = [h * (2 * 4 * D + 8) + m * (4 * D + 8) for h, m in zip(hits, misses)]
-    ach_gbs = statistics.mean(bb / (t * 1e-3) for bb, t in zip(hbm_bytes, x_ms)) / 1e9
+    timed_bytes = hbm_bytes[:: args.time_every][: len(x_ms)]  # the sampled launches
+    ach_gbs = statistics.mean(bb / (t * 1e-3) for bb, t in zip(timed_bytes, x_ms)) / 1e9
     peak, peak_src = read_peaks()
+    # ---- the same extract launches without the overlapping sampler (pipeline depth 1):
+    # k_gather's own efficiency, CUDA events on its stream, same batches as the replay
+    iso = None
+    if args.pipeline == 2:
+        ctx.set_pipeline(1)
+        iso_steps = steps[: min(len(steps), 100)]
+        torch.cuda.synchronize()
+        ctx.set_timing(True)
+        i0 = torch.cuda.Event(enable_timing=True)
+        i1 = torch.cuda.Event(enable_timing=True)
+        i0.record(stream)
+        sd = 0
+        for i in iso_steps:
+            e, b = batch_of(i)
+            ctx.sample_batch(e, b)
+            ctx.extract_sample(out)
+            sd += n_seeds(b)
+        i1.record(stream)
+        torch.cuda.synchronize()
+        xi = ctx.extract_times()
+        ctx.set_timing(False)
+        ctx.set_pipeline(2)
+        ims = i0.elapsed_time(i1)
+        a_iso = statistics.mean(bb / (t * 1e-3) for bb, t in zip(hbm_bytes, xi)) / 1e9
+        iso = {"pipeline_depth": 1, "steps": len(iso_steps), "achieved": a_iso,
+               "frac": a_iso / peak, "extract_ms_per_step": statistics.mean(xi),
+               "ms_per_step": ims / len(iso_steps), "seeds_per_s": sd / (ims / 1e3)}
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
@@ -541,6 +574,7 @@ def main():
     # ---- hit rate vs Optimal (accesses recorded over measured epochs, untimed)
     result_hit = None
     sweep = []
+    k_sweep = []
     similarity = None
     peer_share = None
     if args.cache == "sharded":
@@ -557,20 +591,29 @@ def main():
                     t.copy_(c)
             return t
 
-        # per-epoch access footprints of the measured epochs (Table 2 / Optimal, L148 fn4)
+        # per-epoch access footprints of the measured epochs: Table 2 similarity of the
+        # first two, and their sum over all measured epochs for H and Optimal H* ("all
+        # sample footprints are recorded ... after training", L148 fn4)
         per_epoch = []
-        for e in range(sh.K, sh.K + args.measure_epochs):
+        acc_sum = None
+        # measured epochs start after every presample epoch of the K sweep (no overlap)
+        m0 = max([sh.K] + [int(x) for x in args.k_sweep.split(",") if x])
+        for e in range(m0, m0 + args.measure_epochs):
             ctx.reset_counts(glb.COUNT_ACCESS)
             ctx.set_count_mode(glb.COUNT_ACCESS)
             for b in range(rank, nb, world):
                 ctx.sample_batch(e, b)
             ctx.set_count_mode(glb.COUNT_NONE)
             ctx.sync()
-            per_epoch.append(reduce_counts(ctx.counts_tensor(glb.COUNT_ACCESS)).clone())
-        ctx.counts_tensor(glb.COUNT_ACCESS).copy_(sum(per_epoch))
+            f = reduce_counts(ctx.counts_tensor(glb.COUNT_ACCESS))
+            acc_sum = f.clone() if acc_sum is None else acc_sum.add_(f)
+            if len(per_epoch) < 2:
+                per_epoch.append(f.clone())
+        ctx.counts_tensor(glb.COUNT_ACCESS).copy_(acc_sum)
+        del acc_sum
         if len(per_epoch) >= 2:
             v, num, den = ctx.footprint_similarity(per_epoch[0], per_epoch[1], 0.1)
-            similarity = {"epochs": [sh.K, sh.K + 1], "top_frac": 0.1, "value": v,
+            similarity = {"epochs": [m0, m0 + 1], "top_frac": 0.1, "value": v,
                           "numerator": num, "denominator": den, "source": "Table 2 (L329)"}
         for a in sorted(set(sh.alphas) | {args.alpha}):
             policies = {}
@@ -606,6 +649,22 @@ def main():
             if a == args.alpha:
                 result_hit = sweep[-1]
 
+        # PreSC#K for K in --k-sweep at the shape's paper alpha (Fig 11(a) analog, L335:
+        # "K <= 2 already produce a decent hotness estimation"): presample epochs 0..K-1,
+        # hit rate over the same measured epochs (m0 .. m0+measure_epochs-1, after them)
+        a_k = next((a for a in sh.alphas if 0.0 < a < 1.0), None)
+        if args.k_sweep and a_k is not None:
+            for K in [int(x) for x in args.k_sweep.split(",") if x]:
+                ctx.reset_counts(glb.COUNT_PRESAMPLE)
+                ctx.presample(K, rank, world)
+                reduce_counts(ctx.counts_tensor(glb.COUNT_PRESAMPLE))
+                ctx.build_cache(a_k)
+                hs = ctx.hit_stats()
+                H = hs["hits"] / hs["total"] if hs["total"] else 0.0
+                Hs = hs["optimal_hits"] / hs["total"] if hs["total"] else 0.0
+                k_sweep.append({"K": K, "alpha": a_k, "hit_rate": H, "optimal_hit_rate": Hs,
+                                "presc_vs_optimal_pct": 100.0 * H / Hs if Hs else None})
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         cpu = cpu_baseline(g, sh, args.cpu_seconds)
@@ -633,7 +692,11 @@ def main():
                          "peak_source": peak_src,
                          "extract_ms_per_step": statistics.mean(x_ms),
                          "extract_share_of_step": statistics.mean(x_ms) / (elapsed_max / args.steps),
-                         "algorithmic_bytes_per_launch": statistics.mean(hbm_bytes)},
+                         "algorithmic_bytes_per_launch": statistics.mean(hbm_bytes),
+                         "timed_launches": f"every {args.time_every}th extract of the timed "
+                                           f"region ({len(x_ms)} launches)",
+                         "measured_with": f"pipeline depth {args.pipeline} (the timed region)",
+                         "isolated": iso},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_val, "unit": "seeds/s", "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": d2h, "steps": len(e2e_steps),
@@ -647,6 +710,8 @@ def main():
             "clocks": clk,
             "hit_rate": result_hit,
             "alpha_sweep": sweep,
+            "presc_k_sweep": k_sweep,
+            "measured_epochs": [m0, m0 + args.measure_epochs - 1] if not args.no_sweep else None,
             "footprint_similarity": similarity,
             "units": {"mean_n_L": statistics.mean(nL), "mean_hits": statistics.mean(hits),
                       "mean_misses": statistics.mean(misses)},

@@ -257,10 +257,12 @@ glb_status glb_extract_sample(glb_ctx* ctx, void* out, glb_extract_stats* stats)
  * work on the main stream.  Synchronous. */
 glb_status glb_set_pipeline(glb_ctx* ctx, int depth);
 glb_status glb_extract_stream(glb_ctx* ctx, void** cuda_stream_out);
-/* Timing of the extract kernel itself (CUDA events around each glb_extract_sample launch,
- * on the stream it runs on).  glb_extract_times synchronises, returns the durations in
- * call order (up to max) and resets the record. */
-glb_status glb_set_timing(glb_ctx* ctx, int enable);
+/* Timing of the extract kernel itself: CUDA events around every `period`-th
+ * glb_extract_sample launch (period 1 = each; 0 = off), on the stream it runs on -- events
+ * between the launches of a pipelined step cost overlap, so a bench samples them.
+ * glb_extract_times synchronises, returns the durations in call order (up to max) and
+ * resets the record; glb_set_timing restarts the call count (the first call is timed). */
+glb_status glb_set_timing(glb_ctx* ctx, int period);
 glb_status glb_extract_times(glb_ctx* ctx, float* out_ms, uint64_t max, uint64_t* n);
 
 /* launch counter: number of kernels this ctx launched so far (bench evidence) */

@@ -493,8 +493,9 @@ class Context:
             return torch.cuda.default_stream(self.device)
         return torch.cuda.ExternalStream(p.value, device=self.device)
 
-    def set_timing(self, enable: bool):
-        self._ck(self._lib.glb_set_timing(self._h, int(enable)))
+    def set_timing(self, period):
+        """Time every ``period``-th extract kernel with CUDA events (True = each, 0 = off)."""
+        self._ck(self._lib.glb_set_timing(self._h, int(period)))
 
     def extract_times(self, max_n: int = 1 << 16) -> list:
         """Durations (ms) of the extract kernels recorded since set_timing(True)."""

@@ -220,10 +220,13 @@ glb_status glb_create(int device, glb_ctx** out) {
   glb_ctx* c = new (std::nothrow) glb_ctx();
   if (!c) return set_err(nullptr, GLB_ENOMEM, "host alloc");
   c->device = device;
+  int prio_low = 0, prio_high = 0;
   if ((e = cudaSetDevice(device)) != cudaSuccess ||
       (e = cudaDeviceGetAttribute(&c->num_sms, cudaDevAttrMultiProcessorCount, device)) != cudaSuccess ||
       (e = cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking)) != cudaSuccess ||
-      (e = cudaStreamCreateWithFlags(&c->xstream, cudaStreamNonBlocking)) != cudaSuccess ||
+      (e = cudaDeviceGetStreamPriorityRange(&prio_low, &prio_high)) != cudaSuccess ||
+      // the extract stream (pipeline depth 2) yields SMs to the latency-bound sampler
+      (e = cudaStreamCreateWithPriority(&c->xstream, cudaStreamNonBlocking, prio_low)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_sampled[0], cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_sampled[1], cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_extracted[0], cudaEventDisableTiming)) != cudaSuccess ||
@@ -248,6 +251,8 @@ glb_status glb_create(int device, glb_ctx** out) {
   c->stream = c->own_stream;
   c->st = c->sts[0];
   if (const char* g = getenv("GLB_GATHER_BPS")) c->gather_bps = atoi(g) > 0 ? atoi(g) : 4;
+  c->gather_bps_pipe = getenv("GLB_GATHER_BPS") ? c->gather_bps : 2;
+  if (const char* g = getenv("GLB_GATHER_BPS_PIPE")) c->gather_bps_pipe = atoi(g) > 0 ? atoi(g) : 2;
   if (const char* g = getenv("GLB_L2_PIN")) c->l2_pin = atoi(g) != 0;
   *out = c;
   return GLB_OK;
@@ -717,20 +722,9 @@ static glb_status build_cache_impl(glb_ctx* c, uint64_t C, const uint32_t* hotne
   c->shard_rank = rank;
   c->shard_world = world;
   const uint64_t Cl = C > rank ? (C - rank + world - 1) / world : 0;  // rows i = j*world + rank
-  // cache row stride: D floats, padded to GLB_CACHE_ALIGN bytes for 16-byte-vector rows
-#ifndef GLB_CACHE_ALIGN
-#define GLB_CACHE_ALIGN 0
-#endif
-  c->cache_stride = c->D;
-#if GLB_CACHE_ALIGN
-  if (c->D % 4 == 0) {
-    const uint32_t a = GLB_CACHE_ALIGN / 4;
-    c->cache_stride = (c->D + a - 1) / a * a;
-  }
-#endif
   c->C_local = Cl;
   if (c->features_mapped && (Cl || world > 1)) {
-    CK(dalloc(&c->cache, Cl * (uint64_t)c->cache_stride));  // >= 1 element: a shard always has a base
+    CK(dalloc(&c->cache, Cl * (uint64_t)c->D));  // >= 1 element: a shard always has a base
     const uint32_t* rows = order;
     if (world > 1) {
       uint32_t* sub = tmp + 4 * V;
@@ -978,7 +972,7 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
     c->stream = c->xstream;
   }
   cudaEvent_t t0 = nullptr, t1 = nullptr;
-  if (c->timing) {
+  if (c->timing && (c->timing_calls++ % (uint64_t)c->timing) == 0) {
     if (c->tev_used + 2 > c->tev.size()) {
       for (int i = 0; i < 2; ++i) {
         cudaEvent_t ev;
@@ -1041,10 +1035,12 @@ glb_status glb_extract_stream(glb_ctx* c, void** out) {
   return GLB_OK;
 }
 
-glb_status glb_set_timing(glb_ctx* c, int enable) {
+glb_status glb_set_timing(glb_ctx* c, int enable /* period */) {
   ENTER(c);
   CK(sync_all(c));
-  c->timing = enable != 0;
+  if (enable < 0) return set_err(c, GLB_EINVAL, "timing period < 0");
+  c->timing = enable;
+  c->timing_calls = 0;
   c->tev_used = 0;
   return GLB_OK;
 }

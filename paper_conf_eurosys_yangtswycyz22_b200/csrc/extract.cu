@@ -132,8 +132,7 @@ __global__ void __launch_bounds__(kThreads, 4)
              const uint2* __restrict__ hit_list, const uint2* __restrict__ miss_list,
              const uint32_t* __restrict__ fill_src, const uint32_t* __restrict__ dev_counts,
              uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t R,
-             unsigned long long* xcount, unsigned int* work, ShardTab tab, uint32_t Uh,
-             uint32_t Uo) {
+             unsigned long long* xcount, unsigned int* work, ShardTab tab) {
   pdl_enter();
   // staged work entry: source row address and destination element offset, resolved once
   // per row so the per-vector loop is one LDS.128 + two adds
@@ -183,12 +182,12 @@ __global__ void __launch_bounds__(kThreads, 4)
       re.src = src_miss + (uint64_t)h.y * U;
     } else if (SHARD) {
       const uint32_t w = h.y % tab.W;
-      re.src = (const T*)tab.base[w] + (uint64_t)(h.y / tab.W) * Uh;
+      re.src = (const T*)tab.base[w] + (uint64_t)(h.y / tab.W) * U;
       npeer += (w != tab.rank) && (g * R + t < nh);
     } else {
-      re.src = src_hit + (uint64_t)h.y * Uh;
+      re.src = src_hit + (uint64_t)h.y * U;
     }
-    re.dst = (unsigned long long)h.x * Uo;
+    re.dst = (unsigned long long)h.x * U;
     return re;
   };
   uint64_t g = claim();
@@ -330,14 +329,10 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   const uint32_t D = c->D;
   const bool vec = (D % 4) == 0;
   const uint32_t U = vec ? D / 4 : D;
-  // row strides (in T units): the HBM cache may pad its rows (glb_ctx::cache_stride)
-  const uint32_t cs = c->cache_stride ? c->cache_stride : D;
-  const uint32_t Uh = vec ? cs / 4 : cs;
-  const uint32_t Uo = out == c->cache ? Uh : U;
   uint32_t R = kChunkUnits / U;
   if (R > (uint32_t)kThreads) R = kThreads;
   if (R < 1) R = 1;
-  const int grid = c->num_sms * c->gather_bps;
+  const int grid = c->num_sms * (c->stream == c->xstream ? c->gather_bps_pipe : c->gather_bps);
   // chunk counters of the launching stream (this ctx's gathers are serial on it; each
   // launch leaves them zeroed for the next)
   unsigned int* work = c->stream == c->xstream ? c->work + 4 : c->work;
@@ -353,19 +348,19 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   if (vec && shard)
     e = launch_pdl(k_gather<float4, true>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work, tab, Uh, Uo);
+                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work, tab);
   else if (vec)
     e = launch_pdl(k_gather<float4, false>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work, tab, Uh, Uo);
+                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work, tab);
   else if (shard)
     e = launch_pdl(k_gather<float, true>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   c->xcount, work, tab, Uh, Uo);
+                   c->xcount, work, tab);
   else
     e = launch_pdl(k_gather<float, false>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   c->xcount, work, tab, Uh, Uo);
+                   c->xcount, work, tab);
   count_launch(c);
   return e;
 }

@@ -158,8 +158,7 @@ struct glb_ctx {
 
   // cache (D3, D4, D5)
   int32_t* slot = nullptr;     // i32[V]
-  float* cache = nullptr;      // f32[C][cache_stride]
-  uint32_t cache_stride = 0;   // floats per cache row (D, or D padded to GLB_CACHE_ALIGN bytes)
+  float* cache = nullptr;      // f32[C][D]
   uint64_t C = 0;
   // NEXT-3 peer-sharded cache: global rank i < C is owned by shard i % W at row i / W;
   // shard_base[r] = device pointer (valid in this process) of shard r's rows.
@@ -187,10 +186,13 @@ struct glb_ctx {
   cudaEvent_t ev_sampled[2] = {nullptr, nullptr};
   cudaEvent_t ev_extracted[2] = {nullptr, nullptr};
   int gather_bps = 4;            // gather blocks per SM
+  int gather_bps_pipe = 2;       // ... on the extract stream at pipeline depth 2: leaves SM
+                                 // slots to the sampler running concurrently on the main stream
   unsigned int* work = nullptr;  // device [8]: gather chunk counters (main, extract stream)
   unsigned int* miss_bins = nullptr;  // [miss_bins_cap] host-page histogram of misses
   uint32_t miss_bins_cap = 0;
-  bool timing = false;           // record per-extract kernel events
+  int timing = 0;                // record events around every timing-th extract (0: off)
+  uint64_t timing_calls = 0;
   std::vector<cudaEvent_t> tev;  // pairs (start, end) of recorded extracts
   size_t tev_used = 0;
 
