@@ -85,6 +85,7 @@ void use_slot(glb_ctx* c, int s) {
 cudaError_t sync_all(glb_ctx* c) {
   cudaError_t e = cudaStreamSynchronize(c->stream);
   if (e == cudaSuccess && c->xstream) e = cudaStreamSynchronize(c->xstream);
+  if (e == cudaSuccess && c->sstream) e = cudaStreamSynchronize(c->sstream);
   return e;
 }
 
@@ -195,9 +196,52 @@ void set_l2_window(glb_ctx* c, void* base, size_t bytes) {
   c->pin.hit_ratio = r > 1.0 ? 1.0f : (float)r;
 }
 
+// a1: the permutation of `epoch` into dst, on c->stream (Philox keys + stable radix sort;
+// reading Q9/§8(c).2).  Uses the shuffle scratch: callers order it after any other user.
+cudaError_t compute_perm(glb_ctx* c, uint32_t epoch, uint32_t* dst) {
+  const uint64_t n = c->n_train;
+  unsigned long long* kout = nullptr;
+  uint32_t* vout = nullptr;
+  cudaError_t e = launch_shuffle_keys(c, epoch, c->shuf_keys, c->shuf_vals);
+  if (e == cudaSuccess)
+    e = radix_sort_pairs_u64(c, c->shuf_keys, c->shuf_vals, c->shuf_keys + n, c->shuf_vals + n, n,
+                             64, &kout, &vout);
+  if (e == cudaSuccess) e = launch_permute(c, c->train, vout, n, dst);
+  return e;
+}
+
+// Make `epoch`'s permutation current (prefetched, or computed now on the main stream),
+// then prefetch epoch + 1 into the other buffer on the side stream.
 glb_status ensure_perm(glb_ctx* c, uint32_t epoch) {
-  if (c->perm_epoch == (int)epoch) return GLB_OK;
-  return glb_shuffle(c, epoch);
+  int& cur = c->perm_cur;
+  if (c->perm_b_epoch[cur] != (int)epoch) {
+    const int o = cur ^ 1;
+    if (c->perm_b_epoch[o] == (int)epoch) {  // prefetched: order the main stream after it
+      CK(cudaStreamWaitEvent(c->stream, c->ev_perm[o], 0));
+    } else {  // compute now, after any side-stream shuffle (shared scratch)
+      CK(cudaStreamWaitEvent(c->stream, c->ev_perm[o], 0));
+      CK(cudaStreamWaitEvent(c->stream, c->ev_perm[cur], 0));
+      CK(compute_perm(c, epoch, c->perm_b[o]));
+      c->perm_b_epoch[o] = (int)epoch;
+    }
+    cur = o;
+    c->perm = c->perm_b[cur];
+  }
+  c->perm_epoch = (int)epoch;
+  const int o = cur ^ 1;
+  if (c->perm_prefetch && epoch < 0xFFFFu && c->perm_b_epoch[o] != (int)epoch + 1) {
+    // buffer o may still be read by batches enqueued on the main stream: wait for them
+    CK(cudaEventRecord(c->ev_mark, c->stream));
+    CK(cudaStreamWaitEvent(c->sstream, c->ev_mark, 0));
+    cudaStream_t main = c->stream;
+    c->stream = c->sstream;
+    const cudaError_t e = compute_perm(c, epoch + 1, c->perm_b[o]);
+    c->stream = main;
+    if (e != cudaSuccess) return cuda_fail(c, e, "prefetch shuffle");
+    CK(cudaEventRecord(c->ev_perm[o], c->sstream));
+    c->perm_b_epoch[o] = (int)epoch + 1;
+  }
+  return GLB_OK;
 }
 
 }  // namespace
@@ -227,6 +271,10 @@ glb_status glb_create(int device, glb_ctx** out) {
       (e = cudaDeviceGetStreamPriorityRange(&prio_low, &prio_high)) != cudaSuccess ||
       // the extract stream (pipeline depth 2) yields SMs to the latency-bound sampler
       (e = cudaStreamCreateWithPriority(&c->xstream, cudaStreamNonBlocking, prio_low)) != cudaSuccess ||
+      (e = cudaStreamCreateWithPriority(&c->sstream, cudaStreamNonBlocking, prio_low)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_perm[0], cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_perm[1], cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_mark, cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_sampled[0], cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_sampled[1], cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_extracted[0], cudaEventDisableTiming)) != cudaSuccess ||
@@ -254,6 +302,7 @@ glb_status glb_create(int device, glb_ctx** out) {
   c->gather_bps_pipe = getenv("GLB_GATHER_BPS") ? c->gather_bps : 2;
   if (const char* g = getenv("GLB_GATHER_BPS_PIPE")) c->gather_bps_pipe = atoi(g) > 0 ? atoi(g) : 2;
   if (const char* g = getenv("GLB_L2_PIN")) c->l2_pin = atoi(g) != 0;
+  if (const char* g = getenv("GLB_PERM_PREFETCH")) c->perm_prefetch = atoi(g) != 0;
   *out = c;
   return GLB_OK;
 }
@@ -263,11 +312,17 @@ glb_status glb_destroy(glb_ctx* c) {
   cudaSetDevice(c->device);
   if (c->stream) cudaStreamSynchronize(c->stream);
   if (c->xstream) cudaStreamSynchronize(c->xstream);
+  if (c->sstream) cudaStreamSynchronize(c->sstream);
   free_sample_bufs(c);
   free_graph(c);
   dfree(c->xb.hit_list); dfree(c->xb.miss_list); dfree(c->xb.miss_sorted);
   dfree(c->miss_bins);
-  dfree(c->train); dfree(c->perm); dfree(c->shuf_keys); dfree(c->shuf_vals);
+  dfree(c->train); dfree(c->perm_b[0]); dfree(c->perm_b[1]); dfree(c->shuf_keys); dfree(c->shuf_vals);
+  c->perm = nullptr;
+  if (c->ev_perm[0]) cudaEventDestroy(c->ev_perm[0]);
+  if (c->ev_perm[1]) cudaEventDestroy(c->ev_perm[1]);
+  if (c->ev_mark) cudaEventDestroy(c->ev_mark);
+  if (c->sstream) cudaStreamDestroy(c->sstream);
   dfree(c->sts[0]); dfree(c->sts[1]); dfree(c->st_x); dfree(c->scratch); dfree(c->xcount);
   dfree(c->work);
   for (int i = 0; i < 2; ++i) {
@@ -491,10 +546,15 @@ glb_status glb_set_train_set(glb_ctx* c, const uint32_t* train, uint64_t n, uint
   if (B == 0 || (n && !train) || n >= 0xFFFFFFFFull) return set_err(c, GLB_EINVAL, "bad train set");
   for (uint64_t i = 0; i < n; ++i)
     if (train[i] >= c->V) return set_err(c, GLB_EINVAL, "train id %u >= V", train[i]);
-  CK(cudaStreamSynchronize(c->stream));
-  dfree(c->train); dfree(c->perm); dfree(c->shuf_keys); dfree(c->shuf_vals);
+  CK(sync_all(c));
+  dfree(c->train); dfree(c->perm_b[0]); dfree(c->perm_b[1]); dfree(c->shuf_keys); dfree(c->shuf_vals);
+  c->perm = nullptr;
   CK(dalloc(&c->train, n));
-  CK(dalloc(&c->perm, n));
+  CK(dalloc(&c->perm_b[0], n));
+  CK(dalloc(&c->perm_b[1], n));
+  c->perm_b_epoch[0] = c->perm_b_epoch[1] = -1;
+  c->perm_cur = 0;
+  c->perm = c->perm_b[0];
   CK(dalloc(&c->shuf_keys, 2 * n));
   CK(dalloc(&c->shuf_vals, 2 * n));
   if (n) CK(cudaMemcpy(c->train, train, sizeof(uint32_t) * n, cudaMemcpyHostToDevice));
@@ -517,15 +577,7 @@ glb_status glb_shuffle(glb_ctx* c, uint32_t epoch) {
   ENTER(c);
   if (!c->train_set) return set_err(c, GLB_ESTATE, "shuffle before set_train_set");
   if (epoch > 0xFFFFu) return set_err(c, GLB_ERANGE, "epoch %u >= 2^16", epoch);
-  const uint64_t n = c->n_train;
-  unsigned long long* kout = nullptr;
-  uint32_t* vout = nullptr;
-  CK(launch_shuffle_keys(c, epoch, c->shuf_keys, c->shuf_vals));
-  CK(radix_sort_pairs_u64(c, c->shuf_keys, c->shuf_vals, c->shuf_keys + n, c->shuf_vals + n, n, 64,
-                          &kout, &vout));
-  CK(launch_permute(c, c->train, vout, n, c->perm));
-  c->perm_epoch = (int)epoch;
-  return GLB_OK;
+  return ensure_perm(c, epoch);
 }
 
 glb_status glb_get_permutation(glb_ctx* c, uint32_t* host_out) {
@@ -685,6 +737,7 @@ glb_status glb_get_counts(glb_ctx* c, int which, uint32_t* host_out) {
 // of maxc - h over gid order.  tmp: device u32[4V]; returns the order (inside tmp).
 static glb_status rank_vertices(glb_ctx* c, const uint32_t* hot, uint32_t* tmp, uint32_t** order_out) {
   const uint64_t V = c->V;
+  CK(sync_all(c));  // the radix-sort scratch is shared with the side-stream shuffle prefetch
   uint32_t *k0 = tmp, *v0 = tmp + V, *k1 = tmp + 2 * V, *v1 = tmp + 3 * V;
   uint32_t* dmax = (uint32_t*)c->scratch;
   CK(cudaMemsetAsync(dmax, 0, sizeof(uint32_t), c->stream));

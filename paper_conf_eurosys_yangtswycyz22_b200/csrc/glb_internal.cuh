@@ -198,7 +198,16 @@ struct glb_ctx {
 
   // training set (D9)
   uint32_t* train = nullptr;
-  uint32_t* perm = nullptr;
+  uint32_t* perm = nullptr;       // current epoch permutation (= perm_b[perm_cur])
+  // a1 prefetch: the next epoch's permutation is computed on a low-priority side stream
+  // while the current epoch's batches run, so no shuffle sits on the step's critical path
+  uint32_t* perm_b[2] = {nullptr, nullptr};
+  int perm_b_epoch[2] = {-1, -1};
+  int perm_cur = 0;
+  bool perm_prefetch = true;      // GLB_PERM_PREFETCH=0 disables
+  cudaStream_t sstream = nullptr;
+  cudaEvent_t ev_perm[2] = {nullptr, nullptr};
+  cudaEvent_t ev_mark = nullptr;
   uint64_t n_train = 0;
   uint32_t batch_size = 0;
   uint64_t seed = 0;
