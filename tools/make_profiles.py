@@ -28,12 +28,13 @@ def main(tag):
     buf = io.StringIO()
     with contextlib.redirect_stdout(buf):
         print(f"# ncu launch list of `python bench.py --steps 10 --warmup 3 --no-sweep "
-              f"--no-cpu-baseline` (PR, alpha=1), --cache-control none --clock-control none;")
+              f"--no-cpu-baseline` (PR, alpha=1, default pipeline depth), --cache-control none --clock-control none;")
         print("# per-launch times are serialised by ncu: compare SHARES with the bench, not absolutes")
         print("## all launches (includes load/presample/build_cache/shuffle setup)")
         L.main(os.path.join(src, f"launches_{tag}.csv"))
-        print("## last 56 launches (= steady-state steps: seed, 2x(khop, compact), fixup, gather)")
-        L.main(os.path.join(src, f"launches_{tag}.csv"), 56)
+        print("## last 70 launches (= the last 10 steps, the bench's e2e loop: seed, 2x(khop, compact), "
+              "fixup, gather)")
+        L.main(os.path.join(src, f"launches_{tag}.csv"), 70)
     open(os.path.join(dst, f"{tag}_launch_summary.txt"), "w").write(buf.getvalue())
     traffic = {}
     for k in ["k_gather", "k_compact", "k_khop", "k_seed_init", "k_fixup"]:
