@@ -53,6 +53,11 @@ def parse():
                    help="PreSC#K values for the Fig 11(a) analog (empty: skip)")
     p.add_argument("--mode", default="dp", choices=["dp", "factored"],
                    help="factored: Ns sampler + Nt trainer ranks (PAPER.md §5.2-5.3)")
+    p.add_argument("--handoff", default="peer", choices=["peer", "sendrecv"],
+                   help="factored mode: peer = samples pushed into the trainer's HBM ring by one "
+                        "copy kernel (glb_handoff_*, NVLink/IPC); sendrecv = torch.distributed "
+                        "send/recv of a packed payload")
+    p.add_argument("--handoff-slots", type=int, default=4)
     p.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                    help="gloo: CPU-staged send/recv (lets N ranks share one GPU for testing)")
     p.add_argument("--relabel", default="auto", choices=["auto", "dense", "hash"],
@@ -263,11 +268,29 @@ def run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_c
         ctx.extract(uniq.contiguous(), out=out[:sizes[-1]])
         seeds["n"] += sizes[0]
 
+    peer = args.handoff == "peer" and world > 1
+    if peer:
+        ho = par.PeerHandoff(ctx, roles, rank, slots=args.handoff_slots)
+        ntrain = len(g.train)
+
+        def sample_peer(gidx):  # asynchronous: no sizes read back on the sampler
+            ctx.sample_batch(sh.K + gidx // nb, gidx % nb)
+
+        def extract_peer(gidx):  # the pushed sample is the ctx's current one
+            b = gidx % nb
+            ctx.extract_sample(out)
+            seeds["n"] += min(sh.batch, ntrain - b * sh.batch)
+
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     t0 = time.perf_counter()
-    if world == 1:
+    if peer:
+        if roles.is_sampler(rank):
+            par.run_sampler_peer(sample_peer, ho, total, store, tag)
+        else:
+            par.run_trainer_peer(extract_peer, ho, total, store, tag)
+    elif world == 1:
         for gidx in range(total):
             e, blk = sample_fn(gidx)
             extract_fn(gidx, e, blk.sizes, blk.nnz, (blk.uniq,))
@@ -305,7 +328,9 @@ def run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_c
                 "config": {"workload": workload_name(sh, args.alpha), "mode": "factored",
                            "samplers": ns, "trainers": world - ns,
                            "Ts_ms": 1e3 * float(prof[0]), "Tt_ms": 1e3 * float(prof[1]),
-                           "backend": args.backend, "parallelism": f"factored{ns}s{world - ns}t"},
+                           "backend": args.backend, "parallelism": f"factored{ns}s{world - ns}t",
+                           "handoff": (f"peer ({args.handoff_slots}-slot HBM ring per trainer, "
+                                       "glb_handoff_*)") if peer else "sendrecv"},
                 "timing": "host wall clock around the sampler/trainer loops (max over ranks)",
                 "preprocess_s": {"presample": t_pre, "build_cache": t_cache}}
         print(json.dumps(line), flush=True)

@@ -265,6 +265,54 @@ glb_status glb_extract_stream(glb_ctx* ctx, void** cuda_stream_out);
 glb_status glb_set_timing(glb_ctx* ctx, int period);
 glb_status glb_extract_times(glb_ctx* ctx, float* out_ms, uint64_t max, uint64_t* n);
 
+/* ------------------------------------------ a8: factored Sampler -> Trainer handoff (peer memory)
+ * GNNLab's Samplers put each mini-batch's samples into a global queue from which a Trainer
+ * takes them and extracts their features (Fig 9 L217-L246, L250-L252 §5.2; Table 5 "C").
+ * Here the queue slots live in the TRAINER's HBM: a ring of `slots` receive slots, each sized
+ * for the largest sample of the trainer's sampler config (glb_set_sampler; samplers must use
+ * the same kind / hops and no larger capacities).  A sampler's GPU writes a finished sample
+ * (sizes, uniq, every block's indptr / indices / weights) into a slot with ONE copy kernel --
+ * over NVLink when the ranks are on different GPUs, through CUDA IPC when they are different
+ * processes -- and the trainer marks and extracts it locally.  Ordering is device-side through
+ * interprocess CUDA events (no host sync on either side); the caller's control plane decides
+ * which batch goes to which (trainer, slot) and must order:
+ *   a sampler's glb_handoff_send(t, s) for a slot's k-th use after the trainer's
+ *     glb_handoff_release(s) of its (k-1)-th use was CALLED (host order), and
+ *   the trainer's glb_handoff_recv(p, s) after sampler p's glb_handoff_send(t, s) was CALLED.
+ * Blobs are GLB_HANDOFF_BLOB_BYTES opaque bytes to exchange between processes (e.g. all-gathered
+ * over torch.distributed); a peer in the same process is recognised and used directly.
+ * Ids (trainer, sampler) are caller-chosen in [0, GLB_HANDOFF_MAX_PEERS), e.g. ranks.
+ * glb_set_sampler and glb_destroy drop the ring and every attachment. */
+#define GLB_HANDOFF_MAX_SLOTS 8
+#define GLB_HANDOFF_MAX_PEERS 16
+#define GLB_HANDOFF_BLOB_BYTES 2048
+/* trainer: allocate the ring (device) and its "consumed" events; blob_out receives the ring's
+ * IPC handle, layout and event handles.  Synchronous.  Errors: EINVAL (slots not in
+ * [1, GLB_HANDOFF_MAX_SLOTS]), ESTATE (no sampler config), ENOMEM. */
+glb_status glb_handoff_create(glb_ctx* ctx, uint32_t slots, void* blob_out);
+/* sampler: map trainer `trainer`'s ring from its blob and create this sampler's "ready"
+ * events; blob_out receives their handles for glb_handoff_connect.  Synchronous.  Errors:
+ * EINVAL (bad blob; ring smaller than this sampler's capacity or other hop count / kind). */
+glb_status glb_handoff_attach(glb_ctx* ctx, uint32_t trainer, const void* trainer_blob,
+                              void* blob_out);
+/* trainer: open sampler `sampler`'s ready events from the blob glb_handoff_attach returned. */
+glb_status glb_handoff_connect(glb_ctx* ctx, uint32_t sampler, const void* sampler_blob);
+/* sampler: push the current sample (the last glb_sample*) into slot `slot` of trainer
+ * `trainer` after the trainer's last release of that slot; `tag` (e.g. the global batch id)
+ * travels in the slot header.  Asynchronous on the ctx stream.  Errors: ESTATE (not attached,
+ * no sample), EINVAL (slot out of range, hop count mismatch). */
+glb_status glb_handoff_send(glb_ctx* ctx, uint32_t trainer, uint32_t slot, uint64_t tag);
+/* trainer: make slot `slot` (filled by sampler `sampler`) the ctx's current sample: wait for
+ * the push, mark it against THIS ctx's cache (a4: slot map -> hit / miss lists, cache_slot),
+ * so glb_sample_result / glb_extract_sample read it in place.  Asynchronous. */
+glb_status glb_handoff_recv(glb_ctx* ctx, uint32_t sampler, uint32_t slot);
+/* trainer: the tag of the current received sample (synchronous read). */
+glb_status glb_handoff_tag(glb_ctx* ctx, uint64_t* out);
+/* trainer: the slot may be overwritten once everything enqueued so far on the ctx stream
+ * (and, at pipeline depth 2, its extract stream) has run; if it held the current sample,
+ * the ctx has no current sample afterwards.  Asynchronous. */
+glb_status glb_handoff_release(glb_ctx* ctx, uint32_t slot);
+
 /* launch counter: number of kernels this ctx launched so far (bench evidence) */
 uint64_t glb_kernel_launches(const glb_ctx* ctx);
 

@@ -40,9 +40,14 @@ EXPORTS = [
     "glb_load_edge_weights", "glb_build_cache_sharded", "glb_cache_device_ptr",
     "glb_cache_ipc_handle", "glb_attach_peer_cache", "glb_last_extract_counts",
     "glb_sample_async", "glb_extract_counts_device_ptr",
+    "glb_handoff_create", "glb_handoff_attach", "glb_handoff_connect", "glb_handoff_send",
+    "glb_handoff_recv", "glb_handoff_tag", "glb_handoff_release",
 ]
 MAX_SHARDS = 16
 IPC_HANDLE_BYTES = 64
+HANDOFF_MAX_SLOTS = 8
+HANDOFF_MAX_PEERS = 16
+HANDOFF_BLOB_BYTES = 2048
 
 
 class GlbError(RuntimeError):
@@ -134,6 +139,13 @@ def lib(auto_build: bool = True):
         "glb_last_extract_counts": ([vp, ctypes.POINTER(u64)], i32),
         "glb_sample_async": ([vp, vp, u32, u64, u32, u32], i32),
         "glb_extract_counts_device_ptr": ([vp, ctypes.POINTER(vp)], i32),
+        "glb_handoff_create": ([vp, u32, vp], i32),
+        "glb_handoff_attach": ([vp, u32, vp, vp], i32),
+        "glb_handoff_connect": ([vp, u32, vp], i32),
+        "glb_handoff_send": ([vp, u32, u32, u64], i32),
+        "glb_handoff_recv": ([vp, u32, u32], i32),
+        "glb_handoff_tag": ([vp, ctypes.POINTER(u64)], i32),
+        "glb_handoff_release": ([vp, u32], i32),
         "glb_footprint_similarity": ([vp, vp, vp, dbl, ctypes.POINTER(u64), ctypes.POINTER(u64),
                                       ctypes.POINTER(dbl)], i32),
     }
@@ -452,6 +464,41 @@ class Context:
         self._ck(self._lib.glb_hit_stats_get(self._h, ctypes.byref(s)))
         return {"total": s.total, "hits": s.hits, "optimal_hits": s.optimal_hits,
                 "cache_rows": s.cache_rows}
+
+    # ------------------------------------- a8: factored Sampler -> Trainer handoff
+    def handoff_create(self, slots: int) -> bytes:
+        """Trainer: allocate a ring of ``slots`` receive slots in this GPU's HBM; returns the
+        blob samplers attach with (include/glb.h glb_handoff_create)."""
+        buf = ctypes.create_string_buffer(HANDOFF_BLOB_BYTES)
+        self._ck(self._lib.glb_handoff_create(self._h, slots, buf))
+        return buf.raw
+
+    def handoff_attach(self, trainer: int, trainer_blob: bytes) -> bytes:
+        """Sampler: map trainer ``trainer``'s ring; returns the blob for handoff_connect."""
+        tb = ctypes.create_string_buffer(trainer_blob, HANDOFF_BLOB_BYTES)
+        buf = ctypes.create_string_buffer(HANDOFF_BLOB_BYTES)
+        self._ck(self._lib.glb_handoff_attach(self._h, trainer, tb, buf))
+        return buf.raw
+
+    def handoff_connect(self, sampler: int, sampler_blob: bytes):
+        sb = ctypes.create_string_buffer(sampler_blob, HANDOFF_BLOB_BYTES)
+        self._ck(self._lib.glb_handoff_connect(self._h, sampler, sb))
+
+    def handoff_send(self, trainer: int, slot: int, tag: int):
+        """Sampler: push the current sample into (trainer, slot); asynchronous."""
+        self._ck(self._lib.glb_handoff_send(self._h, trainer, slot, tag))
+
+    def handoff_recv(self, sampler: int, slot: int):
+        """Trainer: the sample in ``slot`` (pushed by ``sampler``) becomes the current one."""
+        self._ck(self._lib.glb_handoff_recv(self._h, sampler, slot))
+
+    def handoff_tag(self) -> int:
+        t = ctypes.c_uint64()
+        self._ck(self._lib.glb_handoff_tag(self._h, ctypes.byref(t)))
+        return t.value
+
+    def handoff_release(self, slot: int):
+        self._ck(self._lib.glb_handoff_release(self._h, slot))
 
     # ------------------------------------------------------------------ extract
     def extract(self, vertices, out=None, stats: bool = False):

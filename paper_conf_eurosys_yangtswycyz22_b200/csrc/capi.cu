@@ -313,6 +313,7 @@ glb_status glb_destroy(glb_ctx* c) {
   if (c->stream) cudaStreamSynchronize(c->stream);
   if (c->xstream) cudaStreamSynchronize(c->xstream);
   if (c->sstream) cudaStreamSynchronize(c->sstream);
+  handoff_free(c);
   free_sample_bufs(c);
   free_graph(c);
   dfree(c->xb.hit_list); dfree(c->xb.miss_list); dfree(c->xb.miss_sorted);
@@ -459,6 +460,7 @@ glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32
     return set_err(c, GLB_EINVAL, "unknown sampler kind %d", kind);
   }
   CK(sync_all(c));
+  handoff_free(c);  // the ring is sized from the sampler config
   free_sample_bufs(c);
   SampleBufs b;
   b.cap_batch = max_batch;
@@ -604,7 +606,7 @@ glb_status glb_sample_result(glb_ctx* c, glb_blocks* out) {
   if (!out) return GLB_OK;
   memset(out, 0, sizeof(*out));
   out->num_hops = c->last_L;
-  out->num_seeds = c->last_n0;
+  out->num_seeds = h.n[0];
   out->uniq = c->sb.uniq;
   out->cache_slot = c->sb.lidslot;
   for (uint32_t l = 0; l <= c->last_L; ++l) out->sizes[l] = h.n[l];

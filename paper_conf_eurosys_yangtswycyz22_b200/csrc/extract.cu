@@ -40,9 +40,10 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
 }
 
 __global__ void __launch_bounds__(kThreads)
-    k_mark(const uint32_t* __restrict__ vertices, uint64_t n, uint64_t V,
+    k_mark(const uint32_t* __restrict__ vertices, uint64_t n, const uint32_t* n_dev, uint64_t V,
            const int32_t* __restrict__ slot, DevState* st, uint2* __restrict__ hit_list,
-           uint2* __restrict__ miss_list) {
+           uint2* __restrict__ miss_list, int32_t* __restrict__ lidslot) {
+  if (n_dev) n = *n_dev;  // count produced on the device (e.g. a received sample's n_L)
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   for (uint64_t i0 = (uint64_t)blockIdx.x * blockDim.x + (threadIdx.x & ~31u); i0 < n; i0 += stride) {
     const uint64_t i = i0 + (threadIdx.x & 31);
@@ -67,6 +68,7 @@ __global__ void __launch_bounds__(kThreads)
     }
     bh = __shfl_sync(kFull, bh, 0);
     bm = __shfl_sync(kFull, bm, 0);
+    if (lidslot && act) lidslot[i] = s;
     if (hit) hit_list[bh + __popc(mh & lanemask_lt())] = make_uint2((uint32_t)i, (uint32_t)s);
     if (miss) miss_list[bm + __popc(mm & lanemask_lt())] = make_uint2((uint32_t)i, u);
   }
@@ -314,11 +316,16 @@ cudaError_t launch_sort_misses(glb_ctx* c, const uint2* miss, const uint32_t* nm
 }
 
 cudaError_t launch_mark(glb_ctx* c, const uint32_t* vertices, uint64_t n) {
+  return launch_mark_to(c, vertices, n, nullptr, c->st_x, c->xb.hit_list, c->xb.miss_list, nullptr);
+}
+
+cudaError_t launch_mark_to(glb_ctx* c, const uint32_t* vertices, uint64_t n, const uint32_t* n_dev,
+                           DevState* st, uint2* hit_list, uint2* miss_list, int32_t* lidslot) {
   int grid = (int)((n + kThreads - 1) / kThreads);
   if (grid < 1) grid = 1;
   if (grid > c->num_sms * 8) grid = c->num_sms * 8;
-  k_mark<<<grid, kThreads, 0, c->stream>>>(vertices, n, c->V, c->slot, c->st_x, c->xb.hit_list,
-                                           c->xb.miss_list);
+  k_mark<<<grid, kThreads, 0, c->stream>>>(vertices, n, n_dev, c->V, c->slot, st, hit_list,
+                                           miss_list, lidslot);
   count_launch(c);
   return cudaGetLastError();
 }

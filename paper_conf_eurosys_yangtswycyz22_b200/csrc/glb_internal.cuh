@@ -124,6 +124,41 @@ struct ExtractBufs {
   uint2* miss_sorted = nullptr;
 };
 
+// a8 factored handoff (handoff.cu).  A trainer owns a ring of receive slots in its HBM;
+// each slot holds a pushed sample: [header: DevState + tag | uniq | indptr_l | indices_l |
+// weights_l], every array at a 256-byte aligned offset fixed by the trainer's sampler
+// capacities (HandoffLayout, shipped to samplers in the trainer's blob).
+constexpr int kHandoffMaxSlots = 8;   // GLB_HANDOFF_MAX_SLOTS
+constexpr int kHandoffMaxPeers = 16;  // GLB_HANDOFF_MAX_PEERS
+struct HandoffLayout {
+  uint64_t slot_bytes, off_tag, off_uniq, cap_uniq;
+  uint64_t off_indptr[GLB_MAX_HOPS], off_indices[GLB_MAX_HOPS], off_weights[GLB_MAX_HOPS];
+  uint64_t cap_indptr[GLB_MAX_HOPS], cap_nnz[GLB_MAX_HOPS];
+  uint32_t L, weighted;
+};
+struct HandoffRecv {  // trainer side
+  uint32_t slots = 0;
+  HandoffLayout lay = {};
+  uint8_t* ring = nullptr;  // device [slots * slot_bytes], IPC-exported
+  int32_t* lidslot[kHandoffMaxSlots] = {};  // local per-slot marks (trainer's cache)
+  uint2* hit[kHandoffMaxSlots] = {};
+  uint2* miss[kHandoffMaxSlots] = {};
+  uint2* miss_sorted[kHandoffMaxSlots] = {};
+  cudaEvent_t consumed[kHandoffMaxSlots] = {};            // own, interprocess
+  cudaEvent_t ready[kHandoffMaxPeers][kHandoffMaxSlots] = {};  // samplers' (opened)
+  bool ready_opened[kHandoffMaxPeers] = {};              // opened via IPC (destroy on free)
+  int cur = -1;                                          // slot of the current sample
+};
+struct HandoffSend {  // sampler side, one per attached trainer
+  uint32_t slots = 0;
+  HandoffLayout lay = {};
+  uint8_t* ring = nullptr;  // trainer's ring, mapped (IPC) or borrowed (same process)
+  bool ring_ipc = false;
+  cudaEvent_t consumed[kHandoffMaxSlots] = {};  // trainer's (opened, or borrowed)
+  bool consumed_opened = false;
+  cudaEvent_t ready[kHandoffMaxSlots] = {};     // own, interprocess
+};
+
 }  // namespace glb
 
 struct glb_ctx {
@@ -233,6 +268,10 @@ struct glb_ctx {
   unsigned long long* xcount = nullptr;      // device [3] hits/misses/peer hits of the last extract
   unsigned long long* h_xcount = nullptr;    // pinned mirror
 
+  // a8 factored handoff (handoff.cu)
+  glb::HandoffRecv* ho_recv = nullptr;
+  glb::HandoffSend* ho_send[glb::kHandoffMaxPeers] = {};
+
   // radix sort scratch
   void* sort_tmp = nullptr;
   size_t sort_tmp_bytes = 0;
@@ -292,6 +331,11 @@ cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, 
 cudaError_t launch_fixup(glb_ctx* c, uint32_t hop);
 cudaError_t launch_table_reset(glb_ctx* c);
 cudaError_t launch_mark(glb_ctx* c, const uint32_t* vertices, uint64_t n);
+// mark into caller-chosen lists; n_dev (nullable) overrides n with a device count; lidslot
+// (nullable) receives slot[vertices[i]] per entry
+cudaError_t launch_mark_to(glb_ctx* c, const uint32_t* vertices, uint64_t n, const uint32_t* n_dev,
+                           DevState* st, uint2* hit_list, uint2* miss_list, int32_t* lidslot);
+void handoff_free(glb_ctx* c);  // handoff.cu: drop the a8 ring / peer mappings
 // Gather rows: hits src_hit[list.y] -> out[list.x], misses src_miss[list.y] -> out[list.x];
 // fill_src (non-null) replaces miss_list with (r, fill_src[r]) (identity destination).
 cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const float* src_miss,

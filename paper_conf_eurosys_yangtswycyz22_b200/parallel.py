@@ -208,3 +208,75 @@ def run_trainer(extract_fn, roles: Roles, rank: int, total: int, store, tag: str
         extract_fn(g, epoch, sizes, nnz, unpack_payload(buf, sizes, nnz, weighted))
         n += 1
     return n
+
+
+# ----------------------------------------------------- factored, peer-memory handoff (a8)
+class PeerHandoff:
+    """The factored handoff over peer memory (include/glb.h glb_handoff_*): every trainer
+    owns a ring of ``slots`` receive slots in its HBM; a sampler's GPU pushes a finished
+    sample into one with a single copy kernel (NVLink between GPUs, CUDA IPC between
+    processes) and the trainer extracts it in place -- the B200 replacement of the
+    send/recv above (no payload packing, no host staging, no host sync on the sampler).
+
+    Batch g goes to trainer ``roles.trainer_rank(g)``, slot ``(g // Nt) % slots``, so batch
+    g reuses the slot of batch g - Nt*slots.  The control plane is the process group's
+    store (the paper's global queue, L217): ``{tag}/src/{g}`` = the sampler that pushed g
+    (set after its push was enqueued), ``{tag}/rel/{g}`` = g's slot was released (set after
+    the trainer's release was enqueued).  Device-side order comes from the library's
+    interprocess events; the store only orders the host calls that enqueue them."""
+
+    def __init__(self, ctx, roles: Roles, rank: int, slots: int = 4, group=None):
+        self.ctx, self.roles, self.rank, self.slots = ctx, roles, rank, slots
+        world = roles.world
+        tblob = ctx.handoff_create(slots) if not roles.is_sampler(rank) else None
+        tblobs = [None] * world
+        dist.all_gather_object(tblobs, tblob, group=group)
+        sblobs = {}
+        if roles.is_sampler(rank):
+            for t in range(roles.n_samplers, world):
+                sblobs[t] = ctx.handoff_attach(t, tblobs[t])
+        allsb = [None] * world
+        dist.all_gather_object(allsb, sblobs, group=group)
+        if not roles.is_sampler(rank):
+            for s in range(roles.n_samplers):
+                ctx.handoff_connect(s, allsb[s][rank])
+        dist.barrier(group=group)
+
+    def slot_of(self, g: int) -> int:
+        return (g // self.roles.n_trainers) % self.slots
+
+
+def run_sampler_peer(sample_fn, ho: PeerHandoff, total: int, store, tag: str):
+    """Sampler executor over peer memory: pull batch g from the global scheduler (L250),
+    wait (host) until its slot's previous batch was released, sample, push.  sample_fn(g)
+    leaves batch g as the ctx's current sample.  Returns #batches."""
+    sched = GlobalScheduler(store, f"{tag}/next")
+    reuse = ho.roles.n_trainers * ho.slots
+    done = 0
+    while True:
+        g = sched.next()
+        if g >= total:
+            break
+        if g >= reuse:
+            store.get(f"{tag}/rel/{g - reuse}")  # blocks until the slot was released
+        sample_fn(g)
+        ho.ctx.handoff_send(ho.roles.trainer_rank(g), ho.slot_of(g), g)
+        store.set(f"{tag}/src/{g}", str(ho.rank))
+        done += 1
+    return done
+
+
+def run_trainer_peer(extract_fn, ho: PeerHandoff, total: int, store, tag: str):
+    """Trainer executor over peer memory: for each batch it owns, find its sampler in the
+    global queue, make the pushed sample current (mark against this GPU's cache), let
+    extract_fn(g) extract / consume it, release the slot.  Returns #batches."""
+    n = 0
+    for g in ho.roles.trainer_batches(ho.rank, total):
+        src = int(store.get(f"{tag}/src/{g}"))
+        s = ho.slot_of(g)
+        ho.ctx.handoff_recv(src, s)
+        extract_fn(g)
+        ho.ctx.handoff_release(s)
+        store.set(f"{tag}/rel/{g}", "1")
+        n += 1
+    return n

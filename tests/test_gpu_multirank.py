@@ -62,14 +62,17 @@ def test_dp_presample_two_ranks_equals_oracle(tmp_path):
     assert np.array_equal(np.load(out).view(np.uint32), full)
 
 
-@pytest.mark.parametrize("mode,cache", [("dp", "replicated"), ("factored", "replicated"),
-                                        ("dp", "sharded")])
-def test_bench_two_ranks(mode, cache):
+@pytest.mark.parametrize("mode,cache,handoff", [("dp", "replicated", "peer"),
+                                                ("factored", "replicated", "peer"),
+                                                ("factored", "replicated", "sendrecv"),
+                                                ("dp", "sharded", "peer")])
+def test_bench_two_ranks(mode, cache, handoff):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
            "--master-addr", "127.0.0.1", "--master-port", str(free_port()), "bench.py",
            "--gpus", "2", "--steps", "16", "--warmup", "3", "--config", "tiny",
            "--backend", "gloo", "--mode", mode, "--no-sweep", "--no-cpu-baseline",
-           "--cache", cache, "--alpha", "0.3" if cache == "sharded" else "1.0"]
+           "--cache", cache, "--alpha", "0.3" if cache == "sharded" else "1.0",
+           "--handoff", handoff]
     r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stderr[-3000:]
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
@@ -78,6 +81,7 @@ def test_bench_two_ranks(mode, cache):
     assert d["n_gpus"] == 2 and d["value"] > 0
     if mode == "factored":
         assert d["config"]["samplers"] + d["config"]["trainers"] == 2
+        assert d["config"]["handoff"].startswith(handoff)
     if cache == "sharded":  # two shards of floor(0.3 V) rows: 60% of the vertices cached
         assert d["cache"]["layout"] == "sharded"
         assert d["cache"]["rows_cached"] == 2 * int(0.3 * 10000)

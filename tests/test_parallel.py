@@ -194,3 +194,80 @@ def test_sharded_cache_handle_exchange(tmp_path, world):
     out = str(tmp_path / "ok.pt")
     mp.spawn(_shard_worker, args=(world, free_port(), out), nprocs=world, join=True)
     assert int(torch.load(out)[0]) == world
+
+
+# ---------------------------------------------------- factored over peer memory (a8)
+class _RingCtx:
+    """Stand-in for the library's handoff calls: a trainer's ring is a directory of slot
+    files; send writes (tag, payload) into the slot file immediately, so a sampler that
+    overwrote a slot before its release would be caught by the trainer's tag check."""
+
+    def __init__(self, rank, ringdir):
+        self.rank, self.dir, self.cur = rank, ringdir, None
+        self.sample = None
+
+    def handoff_create(self, slots):
+        return f"ring{self.rank}:{slots}".encode()
+
+    def handoff_attach(self, trainer, blob):
+        assert blob.decode().startswith(f"ring{trainer}:")
+        return f"ready{self.rank}->{trainer}".encode()
+
+    def handoff_connect(self, sampler, blob):
+        assert blob.decode() == f"ready{sampler}->{self.rank}"
+
+    def handoff_send(self, trainer, slot, tag):
+        np.save(os.path.join(self.dir, f"t{trainer}s{slot}.npy"),
+                np.array([tag, self.rank] + list(self.sample), dtype=np.int64))
+
+    def handoff_recv(self, sampler, slot):
+        a = np.load(os.path.join(self.dir, f"t{self.rank}s{slot}.npy"))
+        assert int(a[1]) == sampler
+        self.cur = (int(a[0]), a[2:])
+
+    def handoff_release(self, slot):
+        self.cur = None
+
+
+def _peer_worker(rank, world, port, ns, slots, total, outdir):
+    import time
+    _init(rank, world, port)
+    roles = par.Roles(ns, world)
+    ctx = _RingCtx(rank, outdir)
+    ho = par.PeerHandoff(ctx, roles, rank, slots=slots)
+    store = dist.distributed_c10d._get_default_store()
+    rng = np.random.default_rng(rank)
+    if roles.is_sampler(rank):
+        def sample_fn(gidx):
+            ctx.sample = [gidx * 7 + i for i in range(3)]
+        n = par.run_sampler_peer(sample_fn, ho, total, store, "p")
+        np.save(os.path.join(outdir, f"s{rank}.npy"), np.array([n]))
+    else:
+        got = []
+
+        def extract_fn(gidx):
+            time.sleep(float(rng.uniform(0, 0.01)))  # let samplers run ahead
+            tag, payload = ctx.cur
+            assert tag == gidx, (tag, gidx)
+            assert payload.tolist() == [gidx * 7 + i for i in range(3)]
+            got.append(gidx)
+
+        par.run_trainer_peer(extract_fn, ho, total, store, "p")
+        np.save(os.path.join(outdir, f"t{rank}.npy"), np.array(got))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,ns,slots", [(2, 1, 1), (3, 2, 2), (4, 1, 3), (4, 3, 1)])
+def test_factored_peer_handoff_protocol(tmp_path, world, ns, slots):
+    """Slot g reuse waits for g - Nt*slots's release; every batch reaches its trainer once
+    and intact, whatever the interleaving of samplers."""
+    total = 30
+    mp.spawn(_peer_worker, args=(world, free_port(), ns, slots, total, str(tmp_path)),
+             nprocs=world, join=True)
+    trained = sorted(int(x) for r in range(ns, world) for x in np.load(tmp_path / f"t{r}.npy"))
+    assert trained == list(range(total))
+    assert sum(int(np.load(tmp_path / f"s{r}.npy")[0]) for r in range(ns)) == total
+    roles = par.Roles(ns, world)
+    for r in range(ns, world):  # each trainer got exactly its batches, in order
+        assert np.load(tmp_path / f"t{r}.npy").tolist() == roles.trainer_batches(r, total)
