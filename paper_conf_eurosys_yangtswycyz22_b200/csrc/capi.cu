@@ -302,6 +302,8 @@ glb_status glb_create(int device, glb_ctx** out) {
   c->gather_bps_pipe = getenv("GLB_GATHER_BPS") ? c->gather_bps : 2;
   if (const char* g = getenv("GLB_GATHER_BPS_PIPE")) c->gather_bps_pipe = atoi(g) > 0 ? atoi(g) : 2;
   if (const char* g = getenv("GLB_L2_PIN")) c->l2_pin = atoi(g) != 0;
+  if (const char* g = getenv("GLB_CACHE_ALIGN")) c->cache_align = (uint32_t)atoi(g);
+  if (const char* g = getenv("GLB_GATHER_ST")) c->gather_st_wb = atoi(g) != 0;
   if (const char* g = getenv("GLB_PERM_PREFETCH")) c->perm_prefetch = atoi(g) != 0;
   *out = c;
   return GLB_OK;
@@ -779,7 +781,13 @@ static glb_status build_cache_impl(glb_ctx* c, uint64_t C, const uint32_t* hotne
   const uint64_t Cl = C > rank ? (C - rank + world - 1) / world : 0;  // rows i = j*world + rank
   c->C_local = Cl;
   if (c->features_mapped && (Cl || world > 1)) {
-    CK(dalloc(&c->cache, Cl * (uint64_t)c->D));  // >= 1 element: a shard always has a base
+    // cache rows: D floats, padded to cache_align bytes when rows are 16-byte vectors
+    c->cache_stride = c->D;
+    if (c->cache_align >= 16 && c->D % 4 == 0) {
+      const uint32_t a = c->cache_align / 4;
+      c->cache_stride = (c->D + a - 1) / a * a;
+    }
+    CK(dalloc(&c->cache, Cl * (uint64_t)c->cache_stride));  // >= 1 element: a shard always has a base
     const uint32_t* rows = order;
     if (world > 1) {
       uint32_t* sub = tmp + 4 * V;

@@ -133,8 +133,10 @@ __global__ void __launch_bounds__(kThreads, 4)
     k_gather(T* __restrict__ out, const T* __restrict__ src_hit, const T* __restrict__ src_miss,
              const uint2* __restrict__ hit_list, const uint2* __restrict__ miss_list,
              const uint32_t* __restrict__ fill_src, const uint32_t* __restrict__ dev_counts,
-             uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t R,
-             unsigned long long* xcount, unsigned int* work, ShardTab tab) {
+             uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t R, uint32_t Sh, uint32_t So,
+             int st_wb, unsigned long long* xcount, unsigned int* work, ShardTab tab) {
+  // U: T-units per row moved; Sh: row stride of src_hit (the HBM cache may pad its rows);
+  // So: row stride of out; host rows (src_miss) are dense (stride U)
   pdl_enter();
   // staged work entry: source row address and destination element offset, resolved once
   // per row so the per-vector loop is one LDS.128 + two adds
@@ -184,12 +186,12 @@ __global__ void __launch_bounds__(kThreads, 4)
       re.src = src_miss + (uint64_t)h.y * U;
     } else if (SHARD) {
       const uint32_t w = h.y % tab.W;
-      re.src = (const T*)tab.base[w] + (uint64_t)(h.y / tab.W) * U;
+      re.src = (const T*)tab.base[w] + (uint64_t)(h.y / tab.W) * Sh;
       npeer += (w != tab.rank) && (g * R + t < nh);
     } else {
-      re.src = src_hit + (uint64_t)h.y * U;
+      re.src = src_hit + (uint64_t)h.y * Sh;
     }
-    re.dst = (unsigned long long)h.x * U;
+    re.dst = (unsigned long long)h.x * So;
     return re;
   };
   uint64_t g = claim();
@@ -220,7 +222,10 @@ __global__ void __launch_bounds__(kThreads, 4)
 #pragma unroll
       for (int q = 0; q < kVecPerThread; ++q) {
         const uint32_t v = base + q * kThreads + t;
-        if (v < total) st_row(out + dst[q], x[q]);
+        if (v < total) {
+          if (st_wb) out[dst[q]] = x[q];
+          else st_row(out + dst[q], x[q]);
+        }
       }
     }
     buf ^= 1;
@@ -340,6 +345,11 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   if (R > (uint32_t)kThreads) R = kThreads;
   if (R < 1) R = 1;
   const int grid = c->num_sms * (c->stream == c->xstream ? c->gather_bps_pipe : c->gather_bps);
+  // row strides in T units: the HBM cache's rows may be padded (glb_ctx::cache_stride)
+  const uint32_t cs = c->cache_stride ? c->cache_stride : D;
+  const uint32_t Sh = vec ? cs / 4 : cs;
+  const uint32_t So = out == c->cache ? Sh : U;
+  const int wb = c->gather_st_wb;
   // chunk counters of the launching stream (this ctx's gathers are serial on it; each
   // launch leaves them zeroed for the next)
   unsigned int* work = c->stream == c->xstream ? c->work + 4 : c->work;
@@ -355,19 +365,19 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   if (vec && shard)
     e = launch_pdl(k_gather<float4, true>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work, tab);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, c->xcount, work, tab);
   else if (vec)
     e = launch_pdl(k_gather<float4, false>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, c->xcount, work, tab);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, c->xcount, work, tab);
   else if (shard)
     e = launch_pdl(k_gather<float, true>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   c->xcount, work, tab);
+                   Sh, So, wb, c->xcount, work, tab);
   else
     e = launch_pdl(k_gather<float, false>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   c->xcount, work, tab);
+                   Sh, So, wb, c->xcount, work, tab);
   count_launch(c);
   return e;
 }

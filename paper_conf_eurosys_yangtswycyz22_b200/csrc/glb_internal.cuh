@@ -193,7 +193,10 @@ struct glb_ctx {
 
   // cache (D3, D4, D5)
   int32_t* slot = nullptr;     // i32[V]
-  float* cache = nullptr;      // f32[C][D]
+  float* cache = nullptr;      // f32[C][cache_stride]
+  uint32_t cache_stride = 0;   // floats per cache row: D, or D padded to cache_align bytes
+  uint32_t cache_align = 0;    // GLB_CACHE_ALIGN (bytes; 0 = dense rows)
+  int gather_st_wb = 0;        // GLB_GATHER_ST=1: write-back stores instead of streaming
   uint64_t C = 0;
   // NEXT-3 peer-sharded cache: global rank i < C is owned by shard i % W at row i / W;
   // shard_base[r] = device pointer (valid in this process) of shard r's rows.
