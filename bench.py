@@ -58,6 +58,8 @@ def parse():
                         "copy kernel (glb_handoff_*, NVLink/IPC); sendrecv = torch.distributed "
                         "send/recv of a packed payload")
     p.add_argument("--handoff-slots", type=int, default=4)
+    p.add_argument("--no-switching", action="store_true",
+                   help="factored/peer: disable dynamic executor switching (PAPER.md L267-L277)")
     p.add_argument("--backend", default="nccl", choices=["nccl", "gloo"],
                    help="gloo: CPU-staged send/recv (lets N ranks share one GPU for testing)")
     p.add_argument("--relabel", default="auto", choices=["auto", "dense", "hash"],
@@ -287,7 +289,11 @@ def run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_c
     t0 = time.perf_counter()
     if peer:
         if roles.is_sampler(rank):
-            par.run_sampler_peer(sample_peer, ho, total, store, tag)
+            # dynamic switching: a sampler that would wait for a busy slot extracts the batch
+            # itself (standby Trainer, same cache here: T_t' = T_t) when the profit is > 0
+            par.run_sampler_peer(sample_peer, ho, total, store, tag,
+                                 standby_fn=None if args.no_switching else extract_peer,
+                                 t_train=float(prof[1]), t_standby=float(prof[1]))
         else:
             par.run_trainer_peer(extract_peer, ho, total, store, tag)
     elif world == 1:
@@ -310,16 +316,17 @@ def run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_c
         par.run_trainer(extract_fn, roles, rank, total, store, tag, comm_dev)
     torch.cuda.synchronize()
     el = time.perf_counter() - t0
-    red = torch.tensor([el, float(seeds["n"])], dtype=torch.float64)
+    red = torch.tensor([el, float(seeds["n"]), float(ho.standby if peer else 0)],
+                       dtype=torch.float64)
     if world > 1:
         r2 = red.to(comm_dev)
         t_max = r2[:1].clone()
         dist.all_reduce(t_max, op=dist.ReduceOp.MAX)
         n_sum = r2[1:].clone()
         dist.all_reduce(n_sum)
-        el, n_all = float(t_max.cpu()), float(n_sum.cpu())
+        el, n_all, n_standby = float(t_max.cpu()), float(n_sum[0].cpu()), int(n_sum[1].cpu())
     else:
-        n_all = float(seeds["n"])
+        n_all, n_standby = float(seeds["n"]), 0
     if rank == 0:
         line = {"metric": METRIC, "value": n_all / el, "unit": "seeds/s", "n_gpus": world,
                 "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * el / args.steps,
@@ -330,7 +337,9 @@ def run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_c
                            "Ts_ms": 1e3 * float(prof[0]), "Tt_ms": 1e3 * float(prof[1]),
                            "backend": args.backend, "parallelism": f"factored{ns}s{world - ns}t",
                            "handoff": (f"peer ({args.handoff_slots}-slot HBM ring per trainer, "
-                                       "glb_handoff_*)") if peer else "sendrecv"},
+                                       "glb_handoff_*)") if peer else "sendrecv",
+                           "standby_batches": n_standby,
+                           "switching": peer and not args.no_switching},
                 "timing": "host wall clock around the sampler/trainer loops (max over ranks)",
                 "preprocess_s": {"presample": t_pre, "build_cache": t_cache}}
         print(json.dumps(line), flush=True)

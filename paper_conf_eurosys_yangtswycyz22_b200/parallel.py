@@ -227,6 +227,7 @@ class PeerHandoff:
 
     def __init__(self, ctx, roles: Roles, rank: int, slots: int = 4, group=None):
         self.ctx, self.roles, self.rank, self.slots = ctx, roles, rank, slots
+        self.standby = 0  # batches this rank extracted as a standby Trainer (switching)
         world = roles.world
         tblob = ctx.handoff_create(slots) if not roles.is_sampler(rank) else None
         tblobs = [None] * world
@@ -246,10 +247,28 @@ class PeerHandoff:
         return (g // self.roles.n_trainers) % self.slots
 
 
-def run_sampler_peer(sample_fn, ho: PeerHandoff, total: int, store, tag: str):
+def switch_profit(m_r: int, t_t: float, n_t: int, t_standby: float) -> float:
+    """Dynamic executor switching's profit metric (§5.3):
+    P = M_r * T_t / N_t - T_t' if N_t > 0, +inf if N_t == 0 -- whether a standby Trainer
+    (on a Sampler's GPU, time T_t' per batch) finishes one task before the N_t normal
+    Trainers (T_t per batch) drain the M_r tasks remaining in the global queue."""
+    if n_t <= 0:
+        return math.inf
+    return m_r * t_t / n_t - t_standby
+
+
+def run_sampler_peer(sample_fn, ho: PeerHandoff, total: int, store, tag: str,
+                     standby_fn=None, t_train: float = 0.0, t_standby: float = 0.0):
     """Sampler executor over peer memory: pull batch g from the global scheduler (L250),
-    wait (host) until its slot's previous batch was released, sample, push.  sample_fn(g)
-    leaves batch g as the ctx's current sample.  Returns #batches."""
+    sample it (sample_fn(g) leaves it as the ctx's current sample), and push it into its
+    trainer's slot once that slot's previous batch was released.
+
+    Dynamic executor switching (L267-L277): when the slot is still busy -- the Trainers
+    are behind and this Sampler would idle -- and a ``standby_fn`` is given, the GPU
+    switches to a standby Trainer for this batch if the profit metric is positive
+    (switch_profit with M_r = batches pushed but not yet extracted): standby_fn(g)
+    extracts the batch locally and the global queue records it as done ("-1"), so its
+    trainer skips it.  Returns #batches sampled; ho.standby counts the switched ones."""
     sched = GlobalScheduler(store, f"{tag}/next")
     reuse = ho.roles.n_trainers * ho.slots
     done = 0
@@ -257,26 +276,40 @@ def run_sampler_peer(sample_fn, ho: PeerHandoff, total: int, store, tag: str):
         g = sched.next()
         if g >= total:
             break
-        if g >= reuse:
-            store.get(f"{tag}/rel/{g - reuse}")  # blocks until the slot was released
         sample_fn(g)
-        ho.ctx.handoff_send(ho.roles.trainer_rank(g), ho.slot_of(g), g)
-        store.set(f"{tag}/src/{g}", str(ho.rank))
         done += 1
+        if g >= reuse:
+            rel = f"{tag}/rel/{g - reuse}"
+            if standby_fn is not None and not store.check([rel]):
+                m_r = int(store.add(f"{tag}/pushed", 0)) - int(store.add(f"{tag}/trained", 0))
+                if switch_profit(m_r, t_train, ho.roles.n_trainers, t_standby) > 0:
+                    standby_fn(g)
+                    ho.standby += 1
+                    store.set(f"{tag}/src/{g}", "-1")
+                    continue
+            store.get(rel)  # blocks until the slot was released
+        ho.ctx.handoff_send(ho.roles.trainer_rank(g), ho.slot_of(g), g)
+        store.add(f"{tag}/pushed", 1)
+        store.set(f"{tag}/src/{g}", str(ho.rank))
     return done
 
 
 def run_trainer_peer(extract_fn, ho: PeerHandoff, total: int, store, tag: str):
     """Trainer executor over peer memory: for each batch it owns, find its sampler in the
     global queue, make the pushed sample current (mark against this GPU's cache), let
-    extract_fn(g) extract / consume it, release the slot.  Returns #batches."""
+    extract_fn(g) extract / consume it, release the slot.  A batch a standby Trainer took
+    (queue entry "-1") is skipped; its slot was never written.  Returns #batches."""
     n = 0
     for g in ho.roles.trainer_batches(ho.rank, total):
         src = int(store.get(f"{tag}/src/{g}"))
+        if src < 0:
+            store.set(f"{tag}/rel/{g}", "1")
+            continue
         s = ho.slot_of(g)
         ho.ctx.handoff_recv(src, s)
         extract_fn(g)
         ho.ctx.handoff_release(s)
+        store.add(f"{tag}/trained", 1)
         store.set(f"{tag}/rel/{g}", "1")
         n += 1
     return n

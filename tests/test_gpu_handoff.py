@@ -148,7 +148,7 @@ def free_port():
     return p
 
 
-def _worker(rank, world, port, outdir, ns, total):
+def _worker(rank, world, port, outdir, ns, total, switching=False):
     import torch.distributed as dist
 
     from paper_conf_eurosys_yangtswycyz22_b200 import parallel as par
@@ -158,45 +158,57 @@ def _worker(rank, world, port, outdir, ns, total):
     g = synth.make_graph("tiny")
     sh = g.shape
     roles = par.Roles(ns, world)
-    ctx = make(g, "khop", sh.fanouts, None if roles.is_sampler(rank) else 0.2)
+    # samplers hold no cache, unless they may switch to standby trainers (same cache here)
+    ctx = make(g, "khop", sh.fanouts, 0.2 if switching or not roles.is_sampler(rank) else None)
     ctx.set_pipeline(2)
     ho = par.PeerHandoff(ctx, roles, rank, slots=2)
     store = dist.distributed_c10d._get_default_store()
     nb = ctx.num_batches
+    res = {}
+
+    def extract_fn(gi, tag=None):
+        s = ctx.sample_result()
+        out = torch.empty((s.sizes[-1], sh.D), dtype=torch.float32, device="cuda:0")
+        st = ctx.extract_sample(out, stats=True)
+        res[gi] = (ctx.handoff_tag() if tag is None else tag, u32(s.uniq).copy(),
+                   [u32(x).copy() for x in s.indptr], [u32(x).copy() for x in s.indices],
+                   out.cpu().numpy().view(np.uint32).copy(), st["hits"])
+        if switching and tag is None:
+            import time
+            time.sleep(0.01)  # slow trainers: samplers would idle (the switching case, L265)
+
     if roles.is_sampler(rank):
         def sample_fn(gi):
             ctx.sample_batch(1 + gi // nb, gi % nb)
-        par.run_sampler_peer(sample_fn, ho, total, store, "h")
+        standby = (lambda gi: extract_fn(gi, tag=gi)) if switching else None
+        par.run_sampler_peer(sample_fn, ho, total, store, "h", standby_fn=standby,
+                             t_train=0.01, t_standby=0.001)
+        assert ho.standby == len(res)
     else:
-        res = {}
-
-        def extract_fn(gi):
-            s = ctx.sample_result()
-            out = torch.empty((s.sizes[-1], sh.D), dtype=torch.float32, device="cuda:0")
-            st = ctx.extract_sample(out, stats=True)
-            res[gi] = (ctx.handoff_tag(), u32(s.uniq).copy(),
-                       [u32(x).copy() for x in s.indptr], [u32(x).copy() for x in s.indices],
-                       out.cpu().numpy().view(np.uint32).copy(), st["hits"])
         par.run_trainer_peer(extract_fn, ho, total, store, "h")
-        np.save(os.path.join(outdir, f"r{rank}.npy"), np.array([res], dtype=object),
-                allow_pickle=True)
+    np.save(os.path.join(outdir, f"r{rank}.npy"), np.array([res], dtype=object), allow_pickle=True)
     torch.cuda.synchronize()
     dist.barrier()
     ctx.close()
     dist.destroy_process_group()
 
 
-@pytest.mark.parametrize("world,ns", [(2, 1), (3, 2), (3, 1)])
-def test_handoff_two_processes_ipc_bit_exact(tiny, tmp_path, world, ns):
+@pytest.mark.parametrize("world,ns,switching", [(2, 1, False), (3, 2, False), (3, 1, False),
+                                                (2, 1, True), (3, 1, True)])
+def test_handoff_two_processes_ipc_bit_exact(tiny, tmp_path, world, ns, switching):
+    """...and with dynamic executor switching: batches a sampler
+    extracted as a standby trainer are bit-exact too, and every batch is extracted once."""
     import torch.multiprocessing as mp
     g, go, counts = tiny
     sh = g.shape
     total = 21  # crosses an epoch boundary (16 batches per epoch), reuses every slot
-    mp.spawn(_worker, args=(world, free_port(), str(tmp_path), ns, total), nprocs=world, join=True)
+    mp.spawn(_worker, args=(world, free_port(), str(tmp_path), ns, total, switching),
+             nprocs=world, join=True)
     slot_map = oracle.cache_slots(counts, 0.2)
     nb = (len(g.train) + sh.batch - 1) // sh.batch
     seen = set()
-    for r in range(ns, world):
+    n_standby = 0
+    for r in range(world):
         res = np.load(os.path.join(tmp_path, f"r{r}.npy"), allow_pickle=True)[0]
         for gi, (tag, uniq, indptr, indices, feats, hits) in res.items():
             e, b = 1 + gi // nb, gi % nb
@@ -209,5 +221,8 @@ def test_handoff_two_processes_ipc_bit_exact(tiny, tmp_path, world, ns):
                 assert np.array_equal(indices[l], exp.indices[l])
             assert np.array_equal(feats, go.extract(exp.uniq).view(np.uint32).reshape(-1, sh.D))
             assert hits == int((slot_map[exp.uniq] >= 0).sum())
+            assert gi not in seen
             seen.add(gi)
+            n_standby += r < ns
     assert seen == set(range(total))
+    assert (n_standby > 0) == switching

@@ -271,3 +271,68 @@ def test_factored_peer_handoff_protocol(tmp_path, world, ns, slots):
     roles = par.Roles(ns, world)
     for r in range(ns, world):  # each trainer got exactly its batches, in order
         assert np.load(tmp_path / f"t{r}.npy").tolist() == roles.trainer_batches(r, total)
+
+
+def test_switch_profit_formula():
+    # P = M_r * T_t / N_t - T_t'; +inf without trainers
+    assert par.switch_profit(10, 2.0, 4, 3.0) == 2.0
+    assert par.switch_profit(1, 2.0, 4, 3.0) < 0
+    assert par.switch_profit(0, 2.0, 0, 3.0) == float("inf")
+
+
+def _switch_worker(rank, world, port, ns, slots, total, t_standby, outdir):
+    import time
+    _init(rank, world, port)
+    roles = par.Roles(ns, world)
+    ctx = _RingCtx(rank, outdir)
+    ho = par.PeerHandoff(ctx, roles, rank, slots=slots)
+    store = dist.distributed_c10d._get_default_store()
+    if roles.is_sampler(rank):
+        local = []
+
+        def sample_fn(gidx):
+            ctx.sample = [gidx * 7 + i for i in range(3)]
+
+        def standby_fn(gidx):
+            assert ctx.sample == [gidx * 7 + i for i in range(3)]
+            local.append(gidx)
+
+        n = par.run_sampler_peer(sample_fn, ho, total, store, "w", standby_fn=standby_fn,
+                                 t_train=0.02, t_standby=t_standby)
+        assert ho.standby == len(local)
+        np.save(os.path.join(outdir, f"s{rank}.npy"), np.array([n]))
+        np.save(os.path.join(outdir, f"l{rank}.npy"), np.array(local, dtype=np.int64))
+    else:
+        got = []
+
+        def extract_fn(gidx):
+            time.sleep(0.02)  # trainers 10x+ slower than samplers: the switching case (L265)
+            tag, payload = ctx.cur
+            assert tag == gidx and payload.tolist() == [gidx * 7 + i for i in range(3)]
+            got.append(gidx)
+
+        par.run_trainer_peer(extract_fn, ho, total, store, "w")
+        np.save(os.path.join(outdir, f"t{rank}.npy"), np.array(got, dtype=np.int64))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world,ns,t_standby,expect_switch", [(2, 1, 0.02, True), (3, 1, 0.02, True),
+                                                               (3, 2, 0.02, True),
+                                                               (2, 1, 1e9, False)])
+def test_dynamic_switching_protocol(tmp_path, world, ns, t_standby, expect_switch):
+    """Samplers that would idle behind slow trainers switch to standby trainers when the
+    profit metric is positive; every batch is extracted exactly once, either by its
+    trainer (in order) or by a standby."""
+    total, slots = 24, 2  # M_r <= Nt*slots: one slot per trainer never makes P > 0
+    mp.spawn(_switch_worker, args=(world, free_port(), ns, slots, total, t_standby, str(tmp_path)),
+             nprocs=world, join=True)
+    local = sorted(int(x) for r in range(ns) for x in np.load(tmp_path / f"l{r}.npy"))
+    trained = sorted(int(x) for r in range(ns, world) for x in np.load(tmp_path / f"t{r}.npy"))
+    assert sorted(local + trained) == list(range(total))
+    assert (len(local) > 0) == expect_switch
+    roles = par.Roles(ns, world)
+    for r in range(ns, world):
+        mine = [g for g in roles.trainer_batches(r, total) if g not in set(local)]
+        assert np.load(tmp_path / f"t{r}.npy").tolist() == mine
+    assert sum(int(np.load(tmp_path / f"s{r}.npy")[0]) for r in range(ns)) == total
