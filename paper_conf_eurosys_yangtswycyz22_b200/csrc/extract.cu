@@ -25,7 +25,10 @@ namespace glb {
 namespace {
 
 constexpr unsigned kFull = 0xFFFFFFFFu;
-constexpr int kVecPerThread = 8;
+#ifndef GLB_GATHER_VEC  // 16-byte vectors in flight per thread (A/B builds: -DGLB_GATHER_VEC=4)
+#define GLB_GATHER_VEC 8
+#endif
+constexpr int kVecPerThread = GLB_GATHER_VEC;
 constexpr int kChunkUnits = kThreads * kVecPerThread;  // vectors per chunk
 
 struct ShardTab {
@@ -134,7 +137,8 @@ __global__ void __launch_bounds__(kThreads, 4)
              const uint2* __restrict__ hit_list, const uint2* __restrict__ miss_list,
              const uint32_t* __restrict__ fill_src, const uint32_t* __restrict__ dev_counts,
              uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t R, uint32_t Sh, uint32_t So,
-             int st_wb, unsigned long long* xcount, unsigned int* work, ShardTab tab) {
+             int st_wb, int misses_only, unsigned long long* xcount, unsigned int* work,
+             ShardTab tab) {
   // U: T-units per row moved; Sh: row stride of src_hit (the HBM cache may pad its rows);
   // So: row stride of out; host rows (src_miss) are dense (stride U)
   pdl_enter();
@@ -147,12 +151,13 @@ __global__ void __launch_bounds__(kThreads, 4)
   __shared__ RowEnt ent[2][kThreads];
   __shared__ unsigned int s_next;
   uint32_t npeer = 0;
-  const uint64_t nh = dev_counts ? dev_counts[0] : nh_host;
+  const uint64_t nh_all = dev_counts ? dev_counts[0] : nh_host;
   const uint64_t nm = dev_counts ? dev_counts[1] : nm_host;
   if (xcount && blockIdx.x == 0 && threadIdx.x == 0) {
-    xcount[0] = nh;
+    xcount[0] = nh_all;
     xcount[1] = nm;
   }
+  const uint64_t nh = misses_only ? 0 : nh_all;  // hits gathered by k_gather_bulk instead
   const uint32_t t = threadIdx.x;
   const uint64_t nch = (nh + R - 1) / R, ncm = (nm + R - 1) / R;  // hit / miss chunks
   const float inv_u = 1.0f / (float)U;
@@ -300,6 +305,111 @@ __global__ void k_miss_scatter(const uint2* __restrict__ miss, const uint32_t* _
   }
 }
 
+// ---- a7 hits through the TMA bulk-copy engine (cp.async.bulk, no tensor map):
+// k_gather moves every 16-byte vector through registers, so it needs many resident
+// threads (and registers) per SM -- exactly what the latency-bound sampler of the next
+// batch, running concurrently at pipeline depth 2, needs too.  Here each lane of a
+// one- or two-warp block owns a ring of P row slots in shared memory and streams its
+// rows through it: bulk load global -> smem (completion on a per-slot mbarrier with the
+// row's byte count), then bulk store smem -> out (bulk_group).  The copy engine keeps
+// 32*NW*(P-1) rows in flight per SM with a handful of registers; the SM's warps stay
+// free for the sampler.  Rows are 16-byte multiples (D % 4 == 0), all addresses
+// 16-byte aligned.  Lane gl takes hit rows gl, gl + NL, ... (static; rows are uniform).
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
+}
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n"
+      "WAIT_%=:\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+      "@!p bra WAIT_%=;\n}" ::"r"(bar), "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+      ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void bulk_store(void* dst, uint32_t src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+               ::"l"(dst), "r"(src), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+
+template <bool SHARD>
+__global__ void __launch_bounds__(64)
+    k_gather_bulk(uint8_t* __restrict__ out, const uint8_t* __restrict__ src_hit,
+                  const uint2* __restrict__ hit_list, const uint32_t* __restrict__ dev_counts,
+                  uint64_t nh_host, uint32_t row_bytes, uint64_t src_stride, uint32_t P,
+                  unsigned long long* xcount, ShardTab tab) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  pdl_enter();
+  const uint32_t lanes = blockDim.x;  // lanes of this block
+  const uint32_t lane = threadIdx.x;
+  // layout: [P][lanes] mbarriers (8 B), [P][lanes] destination rows (4 B), then the
+  // [P][lanes] row slots (128-byte aligned)
+  const uint32_t bar0 = smem_u32(smem);
+  uint32_t* dstrow = reinterpret_cast<uint32_t*>(smem + (uint64_t)P * lanes * 8);
+  const uint32_t slot0 = smem_u32(smem + (((uint64_t)P * lanes * 12 + 127) & ~127ull));
+  auto bar = [&](uint32_t s) { return bar0 + (s * lanes + lane) * 8u; };
+  auto slot = [&](uint32_t s) { return slot0 + (s * lanes + lane) * row_bytes; };
+  for (uint32_t s = 0; s < P; ++s) mbar_init(bar(s), 1);
+  asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  const uint64_t nh = dev_counts ? dev_counts[0] : nh_host;
+  if (xcount && blockIdx.x == 0 && lane == 0) {
+    xcount[0] = nh;
+    xcount[1] = dev_counts ? dev_counts[1] : 0;  // rewritten by the miss gather if it runs
+  }
+  const uint64_t NL = (uint64_t)gridDim.x * lanes;
+  const uint64_t gl = (uint64_t)blockIdx.x * lanes + lane;
+  const uint64_t nk = gl < nh ? (nh - gl + NL - 1) / NL : 0;  // rows of this lane
+  uint32_t npeer = 0;
+  auto src_of = [&](uint2 h) -> const uint8_t* {
+    if (SHARD) {
+      const uint32_t w = h.y % tab.W;
+      npeer += w != tab.rank;
+      return (const uint8_t*)tab.base[w] + (uint64_t)(h.y / tab.W) * src_stride;
+    }
+    return src_hit + (uint64_t)h.y * src_stride;
+  };
+  auto issue = [&](uint64_t k) {  // load row k of this lane into slot k % P
+    const uint2 h = __ldg(hit_list + gl + k * NL);
+    const uint32_t s = (uint32_t)(k % P);
+    dstrow[s * lanes + lane] = h.x;
+    mbar_expect_tx(bar(s), row_bytes);
+    bulk_load(slot(s), src_of(h), row_bytes, bar(s));
+  };
+  const uint64_t pro = nk < P ? nk : P;
+#pragma unroll 1
+  for (uint64_t k = 0; k < pro; ++k) issue(k);
+#pragma unroll 1
+  for (uint64_t k = 0; k < nk; ++k) {
+    const uint32_t s = (uint32_t)(k % P);
+    mbar_wait(bar(s), (uint32_t)((k / P) & 1));
+    bulk_store(out + (uint64_t)dstrow[s * lanes + lane] * row_bytes, slot(s), row_bytes);
+    // refill the slot of the previous row (P >= 2) once its store has read it; the store
+    // just issued may stay in flight
+    if (k >= 1 && k - 1 + P < nk) {
+      asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+      issue(k - 1 + P);
+    }
+  }
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");  // stores complete before exit
+  if (SHARD) {
+    const uint32_t wsum = __reduce_add_sync(kFull, npeer);
+    if ((lane & 31) == 0 && wsum && xcount) atomicAdd(&xcount[2], (unsigned long long)wsum);
+  }
+}
+
 }  // namespace
 
 cudaError_t launch_sort_misses(glb_ctx* c, const uint2* miss, const uint32_t* nmiss_dev,
@@ -350,6 +460,44 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   const uint32_t Sh = vec ? cs / 4 : cs;
   const uint32_t So = out == c->cache ? Sh : U;
   const int wb = c->gather_st_wb;
+  int mo = 0;
+  // hits through the bulk-copy engine (sample / generic extracts, rows of 16-byte vectors)
+  if (c->gather_bulk && vec && hit_list && !fill_src && out != c->cache) {
+    const uint32_t lanes = 64, row_bytes = 4 * D;
+    uint32_t P = (uint32_t)((uint64_t)c->gather_bulk_smem / ((uint64_t)lanes * row_bytes));
+    if (P > 16) P = 16;
+    if (P >= 2) {
+      const size_t smem = (((size_t)P * lanes * 12 + 127) & ~(size_t)127) + (size_t)P * lanes * row_bytes;
+      const bool shard = c->shard_world > 1 && src_hit == c->cache;
+      ShardTab tab = {};
+      tab.W = c->shard_world;
+      tab.rank = c->shard_rank;
+      for (uint32_t w = 0; w < c->shard_world; ++w) tab.base[w] = c->shard_base[w];
+      cudaError_t e;
+      if (shard && (e = cudaMemsetAsync(c->xcount + 2, 0, sizeof(unsigned long long), c->stream)) != cudaSuccess)
+        return e;
+      auto kern = shard ? k_gather_bulk<true> : k_gather_bulk<false>;
+      if ((e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) != cudaSuccess)
+        return e;
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3(c->num_sms);
+      cfg.blockDim = dim3(lanes);
+      cfg.dynamicSmemBytes = smem;
+      cfg.stream = c->stream;
+      cudaLaunchAttribute attr[1];
+      attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+      attr[0].val.programmaticStreamSerializationAllowed = 1;
+      cfg.attrs = attr;
+      cfg.numAttrs = 1;
+      const uint64_t stride = 4ull * (c->cache_stride ? c->cache_stride : D);
+      e = cudaLaunchKernelEx(&cfg, kern, (uint8_t*)out, (const uint8_t*)src_hit, hit_list,
+                             dev_counts, (uint64_t)nhit_host, row_bytes, stride, P, c->xcount, tab);
+      count_launch(c);
+      if (e != cudaSuccess) return e;
+      if (c->C >= c->V) return cudaSuccess;  // every vertex cached: no misses to gather
+      mo = 1;  // the misses follow on the LSU path (host memory over PCIe)
+    }
+  }
   // chunk counters of the launching stream (this ctx's gathers are serial on it; each
   // launch leaves them zeroed for the next)
   unsigned int* work = c->stream == c->xstream ? c->work + 4 : c->work;
@@ -360,24 +508,24 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   tab.rank = c->shard_rank;
   for (uint32_t w = 0; w < c->shard_world; ++w) tab.base[w] = c->shard_base[w];
   cudaError_t e;
-  if (shard && (e = cudaMemsetAsync(c->xcount + 2, 0, sizeof(unsigned long long), c->stream)) != cudaSuccess)
+  if (shard && !mo && (e = cudaMemsetAsync(c->xcount + 2, 0, sizeof(unsigned long long), c->stream)) != cudaSuccess)
     return e;
   if (vec && shard)
     e = launch_pdl(k_gather<float4, true>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, c->xcount, work, tab);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo, c->xcount, work, tab);
   else if (vec)
     e = launch_pdl(k_gather<float4, false>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, c->xcount, work, tab);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo, c->xcount, work, tab);
   else if (shard)
     e = launch_pdl(k_gather<float, true>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   Sh, So, wb, c->xcount, work, tab);
+                   Sh, So, wb, mo, c->xcount, work, tab);
   else
     e = launch_pdl(k_gather<float, false>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   Sh, So, wb, c->xcount, work, tab);
+                   Sh, So, wb, mo, c->xcount, work, tab);
   count_launch(c);
   return e;
 }

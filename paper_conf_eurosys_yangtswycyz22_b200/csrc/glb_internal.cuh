@@ -197,6 +197,9 @@ struct glb_ctx {
   uint32_t cache_stride = 0;   // floats per cache row: D, or D padded to cache_align bytes
   uint32_t cache_align = 0;    // GLB_CACHE_ALIGN (bytes; 0 = dense rows)
   int gather_st_wb = 0;        // GLB_GATHER_ST=1: write-back stores instead of streaming
+  int gather_bulk = 0;         // GLB_GATHER_BULK=1: hits through cp.async.bulk (k_gather_bulk);
+                               // measured 2x slower than the LSU gather
+  uint32_t gather_bulk_smem = 96 * 1024;  // row-slot bytes per bulk block (GLB_GATHER_BULK_SMEM)
   uint64_t C = 0;
   // NEXT-3 peer-sharded cache: global rank i < C is owned by shard i % W at row i / W;
   // shard_base[r] = device pointer (valid in this process) of shard r's rows.

@@ -224,12 +224,16 @@ def test_presample_cache_and_hit_stats(tiny, mode):
         assert hs["hits"] <= hs["optimal_hits"]
 
 
-@pytest.mark.parametrize("mode", MODES)
+@pytest.mark.parametrize("mode", MODES + ["bulk"])
 @pytest.mark.parametrize("alpha", [0.0, 0.1, 0.5, 1.0])
-def test_extract_sample_bytes(tiny, alpha, mode):
+def test_extract_sample_bytes(tiny, alpha, mode, monkeypatch):
+    """mode 'bulk': hits through the cp.async.bulk gather (GLB_GATHER_BULK=1, off by
+    default), misses through the LSU gather."""
     g, go = tiny
     sh = g.shape
-    ctx = make_ctx(g, fanouts=sh.fanouts, mode=mode)
+    if mode == "bulk":
+        monkeypatch.setenv("GLB_GATHER_BULK", "1")
+    ctx = make_ctx(g, fanouts=sh.fanouts, mode="auto" if mode == "bulk" else mode)
     ctx.presample(1)
     ctx.build_cache(alpha)
     slot = ctx.cache_slots()
