@@ -49,7 +49,54 @@ def oracle_counts_parallel(g, sh, epochs):
         return sum(ex.map(run, shards)).astype(np.uint32)
 
 
-def check_config(name, Ks=None):
+def make_sampler_ctx(g, sh, features=True):
+    ctx = glb.Context(0)
+    ctx.load_graph(g.indptr, g.indices, g.features if features else None)
+    if sh.sampler == "khop":
+        ctx.set_sampler("khop", fanouts=sh.fanouts, max_batch=sh.batch)
+    else:
+        ctx.set_sampler("rwalk", layers=len(sh.fanouts), walks=synth.RW_WALKS,
+                        walk_len=synth.RW_LEN, topk=sh.fanouts[0], max_batch=sh.batch)
+    ctx.set_train_set(g.train, sh.batch, g.seed)
+    return ctx
+
+
+def check_handoff(g, sh, go, trainer, slot_map, e):
+    """a8 at full size (config 5's factored split): a topology-only sampler ctx pushes
+    batches into the trainer ctx's HBM ring (glb_handoff_*); the trainer marks them against
+    its cache and extracts.  Bit-exact samples, sampled rows and hit counts."""
+    sampler = make_sampler_ctx(g, sh, features=False)  # samplers hold no features / cache
+    trainer.handoff_connect(0, sampler.handoff_attach(1, trainer.handoff_create(2)))
+    ob = oracle.epoch_batches(g.train, sh.batch, g.seed, e)
+    nb = len(ob)
+    rng = np.random.default_rng(1)
+    ub = sh.batch
+    for k in sh.fanouts:
+        ub = min(ub * (1 + k), sh.V)
+    out = torch.empty((ub, sh.D), dtype=torch.float32, device="cuda")
+    for i, b in enumerate([0, 1, int(rng.integers(2, nb - 1)), nb - 1]):
+        sampler.sample_batch(e, b)
+        sampler.handoff_send(1, i % 2, b)
+        trainer.handoff_recv(0, i % 2)
+        s = trainer.sample_result()
+        os_ = oracle_sample(go, sh, ob[b], g.seed, e, b)
+        assert s.sizes == os_.sizes, b
+        assert np.array_equal(u32(s.uniq), os_.uniq)
+        for l in range(len(sh.fanouts)):
+            assert np.array_equal(u32(s.indptr[l]), os_.indptr[l]), (b, l)
+            assert np.array_equal(u32(s.indices[l]), os_.indices[l]), (b, l)
+        assert np.array_equal(s.cache_slot.cpu().numpy(), slot_map[os_.uniq])
+        st = trainer.extract_sample(out, stats=True)
+        idx = rng.integers(0, s.sizes[-1], 2048)
+        got = out[torch.from_numpy(idx).cuda()].cpu().numpy()
+        assert np.array_equal(got.view(np.uint32), g.features[os_.uniq[idx]].view(np.uint32))
+        assert st["hits"] == int((slot_map[os_.uniq] >= 0).sum())
+        assert trainer.handoff_tag() == b
+        trainer.handoff_release(i % 2)
+    sampler.close()
+
+
+def check_config(name, Ks=None, handoff=False):
     sh = synth.SHAPES[name]
     g = synth.make_graph(sh)
     go = oracle.GraphOracle(g.indptr, g.indices, g.features)
@@ -94,6 +141,8 @@ def check_config(name, Ks=None):
         assert np.array_equal(got.view(np.uint32), g.features[os_.uniq[idx]].view(np.uint32))
         slot = ctx.cache_slots()
         assert st["hits"] == int((slot[os_.uniq] >= 0).sum())
+    if handoff:
+        check_handoff(g, sh, go, ctx, oracle.cache_slots(counts, sh.alphas[-1]), e)
     ctx.close()
 
 
@@ -106,4 +155,5 @@ def test_pa_fullsize_presc_k123():
 
 
 def test_uk_fullsize():
-    check_config("UK")
+    """configs[4]: also the factored sampler -> trainer handoff at full size."""
+    check_config("UK", handoff=True)
