@@ -228,58 +228,59 @@ def cpu_baseline(g, sh, budget_s):
     return par
 
 
-def _oracle_worker(args):
-    """One process of the all-cores oracle run: batches p, p+P, ... of the epoch until
-    its time budget is spent (at least one)."""
-    p, P, budget = args
-    go, g, sh, bs = _ORACLE_SHARED
-    t_tot, seeds, nb = 0.0, 0, 0
-    for b in range(p, len(bs), P):
-        if nb and t_tot >= budget:
-            break
-        t0 = time.perf_counter()
-        s = go.sample(sh.sampler, bs[b], sh.fanouts, g.seed, sh.K, b, g.weights)
-        go.extract(s.uniq)
-        t_tot += time.perf_counter() - t0
-        seeds += len(bs[b])
-        nb += 1
-    return seeds, t_tot, nb
-
-
-_ORACLE_SHARED = None
-
-
 def cpu_baseline_parallel(go, g, sh, bs, budget_s):
-    """SURVEY §8(d) timing (ii): the same oracle, process-parallel over disjoint batches on
-    the host's cores (fork: the graph is shared copy-on-write; each process owns its
-    batches).  P = usable cores, capped at the epoch's batch count and at 64 processes
-    (each extract allocates n_L x D floats).  value = all seeds / the slowest process."""
-    import multiprocessing as mp
-    global _ORACLE_SHARED
+    """SURVEY §8(d) timing (ii): the same oracle on all usable host cores, over disjoint
+    batches of epochs K, K+1, ... -- one thread per core, each with its own GraphOracle
+    (lid scratch) over the shared graph; the oracle's sample and extract are C calls made
+    through ctypes, which release the GIL, so the threads run in parallel.  The thread
+    count is capped by the memory one batch needs (lid scratch + extract output) against
+    half the available host RAM.  value = all seeds / the slowest thread's busy time."""
+    import concurrent.futures as cf
+
+    import oracle
     try:
         ncpu = len(os.sched_getaffinity(0))
     except AttributeError:
         ncpu = os.cpu_count() or 1
-    P = max(1, min(ncpu, len(bs), 64))
+    ub = sh.batch
+    for k in sh.fanouts:
+        ub = min(ub * (1 + (k if sh.sampler != "rwalk" else k)), sh.V)
+    per_thread = 4 * sh.V + 6 * ub * 4 + ub * sh.D * 4
+    try:
+        import psutil
+        avail = psutil.virtual_memory().available
+    except Exception:
+        avail = 8 << 30
+    P = max(1, min(ncpu, int(avail * 0.5 // max(per_thread, 1)), 64))
     if P < 2:
         return None
-    _ORACLE_SHARED = (go, g, sh, bs)
-    try:
-        with mp.get_context("fork").Pool(P) as pool:
-            res = pool.map(_oracle_worker, [(p, P, budget_s) for p in range(P)])
-    except Exception as e:  # report the single-threaded number only
-        print(f"[bench] all-cores oracle run failed: {e}", file=sys.stderr)
-        return None
-    finally:
-        _ORACLE_SHARED = None
+    epochs = [bs] + [oracle.epoch_batches(g.train, sh.batch, g.seed, sh.K + i) for i in (1, 2, 3)]
+    jobs = [(sh.K + i, b, s) for i, ep in enumerate(epochs) for b, s in enumerate(ep)]
+
+    def run(p):
+        o = oracle.GraphOracle(g.indptr, g.indices, g.features)
+        t_tot, seeds, nb = 0.0, 0, 0
+        for e, b, sd in jobs[p::P]:
+            if nb and t_tot >= budget_s:
+                break
+            t0 = time.perf_counter()
+            smp = o.sample(sh.sampler, sd, sh.fanouts, g.seed, e, b, g.weights)
+            o.extract(smp.uniq)
+            t_tot += time.perf_counter() - t0
+            seeds += len(sd)
+            nb += 1
+        return seeds, t_tot, nb
+
+    with cf.ThreadPoolExecutor(P) as ex:
+        res = list(ex.map(run, range(P)))
     seeds = sum(r[0] for r in res)
     wall = max(r[1] for r in res)
     nb = sum(r[2] for r in res)
     return {"value": seeds / wall, "unit": "seeds/s", "cores": P, "kind": "oracle",
             "host_cpus": ncpu,
-            "sample": f"{nb} mini-batches of epoch {sh.K} over {P} processes (disjoint batches, "
-                      f"sample+relabel+extract, {seeds} seeds, slowest process {wall:.1f} s), "
-                      f"single-threaded C oracle per process"}
+            "sample": f"{nb} mini-batches of epochs {sh.K}.. over {P} threads (disjoint batches, "
+                      f"sample+relabel+extract, {seeds} seeds, slowest thread {wall:.1f} s), "
+                      f"single-threaded C oracle per thread (ctypes releases the GIL)"}
 
 
 # ------------------------------------------------------------------------------------------
