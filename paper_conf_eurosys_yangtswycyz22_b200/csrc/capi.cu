@@ -302,6 +302,7 @@ glb_status glb_create(int device, glb_ctx** out) {
   c->gather_bps_pipe = getenv("GLB_GATHER_BPS") ? c->gather_bps : 2;
   if (const char* g = getenv("GLB_GATHER_BPS_PIPE")) c->gather_bps_pipe = atoi(g) > 0 ? atoi(g) : 2;
   if (const char* g = getenv("GLB_L2_PIN")) c->l2_pin = atoi(g) != 0;
+  if (const char* g = getenv("GLB_SAMPLE_BPS")) c->sample_bps = atoi(g) > 0 ? atoi(g) : 8;
   if (const char* g = getenv("GLB_CACHE_ALIGN")) c->cache_align = (uint32_t)atoi(g);
   if (const char* g = getenv("GLB_GATHER_ST")) c->gather_st_wb = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_BULK")) c->gather_bulk = atoi(g) != 0;

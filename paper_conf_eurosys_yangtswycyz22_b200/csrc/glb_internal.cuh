@@ -226,6 +226,7 @@ struct glb_ctx {
   cudaStream_t xstream = nullptr;  // extract stream (pipeline depth 2)
   cudaEvent_t ev_sampled[2] = {nullptr, nullptr};
   cudaEvent_t ev_extracted[2] = {nullptr, nullptr};
+  int sample_bps = 8;            // sampler kernels' blocks per SM (GLB_SAMPLE_BPS)
   int gather_bps = 4;            // gather blocks per SM
   int gather_bps_pipe = 2;       // ... on the extract stream at pipeline depth 2: leaves SM
                                  // slots to the sampler running concurrently on the main stream

@@ -597,8 +597,11 @@ __device__ __forceinline__ unsigned long long warp_sum64(unsigned long long x) {
 //  monotone (later atomicMins never replace it) and a concurrent reader sees
 //  either value, both of which it resolves correctly.
 
+#ifndef GLB_COMPACT_MINB  // min resident compaction blocks per SM (register cap; A/B builds)
+#define GLB_COMPACT_MINB 3
+#endif
 template <bool W, bool HASH>
-__global__ void __launch_bounds__(kThreads, 3)
+__global__ void __launch_bounds__(kThreads, GLB_COMPACT_MINB)
     k_compact(uint32_t hop, uint32_t k, Table T, DevState* st,
               const uint32_t* __restrict__ picks, const uint32_t* __restrict__ pickw,
               const uint32_t* __restrict__ pidx,
@@ -863,7 +866,10 @@ __global__ void k_table_reset(VEntry* __restrict__ t, uint64_t n) {
   }
 }
 
-inline int grid_for(glb_ctx* c, int per_sm = 8) { return c->num_sms * per_sm; }
+// sampler grids: blocks per SM (GLB_SAMPLE_BPS; default 8 = a full SM of 256-thread blocks)
+inline int grid_for(glb_ctx* c, int per_sm = 0) {
+  return c->num_sms * (per_sm ? per_sm : c->sample_bps);
+}
 
 MarkArgs mark_args(glb_ctx* c, int count_mode) {
   MarkArgs m;
@@ -1001,7 +1007,7 @@ cudaError_t launch_fixup(glb_ctx* c, uint32_t hop) {
 
 cudaError_t launch_compact(glb_ctx* c, uint32_t hop, uint32_t k, bool weighted, int count_mode) {
   const SampleBufs& b = c->sb;
-  const int grid = grid_for(c, 3);
+  const int grid = grid_for(c, GLB_COMPACT_MINB);
   const uint32_t* pk = b.picks;
   const uint32_t* pw = b.pickw;
   const uint32_t* pi = b.pidx;
