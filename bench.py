@@ -779,6 +779,7 @@ def main():
             "cache": {"layout": args.cache, "rows_cached": ctx_cache_rows,
                       "peer_hit_share": peer_share},
             "relabel_table": ctx.relabel_mode,
+            "relabel_l2_window_bytes": ctx.relabel_l2_window,
             "host_wall_ms_timed_region": wall_ms,
             "host_enqueue_ms_timed_region": enqueue_ms,
             "roofline": {"kernel": "k_gather (extract a7)", "bound": "hbm", "achieved": ach_gbs,

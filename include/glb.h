@@ -98,6 +98,11 @@ glb_status glb_set_sampler(glb_ctx* ctx, int kind, const uint32_t* fanouts, uint
  * the mode in use (1 or 2). */
 glb_status glb_set_relabel_mode(glb_ctx* ctx, int mode);
 glb_status glb_relabel_mode(const glb_ctx* ctx, int* out);
+/* Bytes of the relabel table covered by a persisting-L2 access-policy window on the sampler's
+ * kernels (0 = none).  Set by glb_set_sampler: by default only when the whole table fits in
+ * a third of L2 (it then stays resident while the pipelined gather streams through L2);
+ * environment GLB_L2_PIN=0 / 1 forces it off / on. */
+glb_status glb_relabel_l2_window(const glb_ctx* ctx, uint64_t* bytes_out);
 
 /* Training set T (host u32[n], distinct, each < V) and mini-batch size B
  * (L305 §6.2: shuffle T each epoch and divide it; last batch partial).

@@ -41,7 +41,7 @@ EXPORTS = [
     "glb_cache_ipc_handle", "glb_attach_peer_cache", "glb_last_extract_counts",
     "glb_sample_async", "glb_extract_counts_device_ptr",
     "glb_handoff_create", "glb_handoff_attach", "glb_handoff_connect", "glb_handoff_send",
-    "glb_handoff_recv", "glb_handoff_tag", "glb_handoff_release",
+    "glb_handoff_recv", "glb_handoff_tag", "glb_handoff_release", "glb_relabel_l2_window",
 ]
 MAX_SHARDS = 16
 IPC_HANDLE_BYTES = 64
@@ -130,6 +130,7 @@ def lib(auto_build: bool = True):
         "glb_extract_times": ([vp, vp, u64, ctypes.POINTER(u64)], i32),
         "glb_set_relabel_mode": ([vp, i32], i32),
         "glb_relabel_mode": ([vp, ctypes.POINTER(i32)], i32),
+        "glb_relabel_l2_window": ([vp, ctypes.POINTER(u64)], i32),
         "glb_policy_hotness": ([vp, i32, u64, vp], i32),
         "glb_load_edge_weights": ([vp, vp], i32),
         "glb_build_cache_sharded": ([vp, dbl, vp, u32, u32], i32),
@@ -280,6 +281,13 @@ class Context:
         m = ctypes.c_int()
         self._ck(self._lib.glb_relabel_mode(self._h, ctypes.byref(m)))
         return {1: "dense", 2: "hash"}[m.value]
+
+    @property
+    def relabel_l2_window(self) -> int:
+        """Bytes of the relabel table pinned in L2 for the sampler's kernels (0 = none)."""
+        b = ctypes.c_uint64()
+        self._ck(self._lib.glb_relabel_l2_window(self._h, ctypes.byref(b)))
+        return b.value
 
     def set_train_set(self, train: np.ndarray, batch_size: int, seed: int):
         t = np.ascontiguousarray(train, dtype=np.uint32)

@@ -108,6 +108,11 @@ void free_graph(glb_ctx* c) {
   c->hslot = nullptr;
   c->hmask = 0;
   c->hash_mode = false;
+  if (c->pin.bytes) {  // release this ctx's persisting-L2 set-aside
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
+    cudaCtxResetPersistingL2Cache();
+    (void)cudaGetLastError();
+  }
   c->pin = L2Window();
   dfree(c->slot); dfree(c->cache); dfree(c->counts); dfree(c->access);
   if (c->registered && c->h_features) cudaHostUnregister((void*)c->h_features);
@@ -178,13 +183,26 @@ glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, in
 }
 
 // Persisting-L2 set-aside + window over the relabel table (skipped if unsupported).
+// Auto (GLB_L2_PIN unset): only when the whole table fits in a third of L2 and in the
+// persisting set-aside.  Measured at pipeline depth 2 (profiles/r01_ab_experiments.txt):
+// PR's 39 MB dense table pinned keeps the sampler's relabel accesses in L2 while the
+// previous batch's gather streams ~850 MB through it, 234 -> 206 us/step; tables that
+// need most of the set-aside (PR's 80 MB hash table, UK/TW/PA) starve the gather's L2
+// share and run 1.3-2.9x slower, so they are never pinned automatically.
 void set_l2_window(glb_ctx* c, void* base, size_t bytes) {
+  if (c->pin.bytes) {  // drop an earlier set-aside of this ctx
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, 0);
+    cudaCtxResetPersistingL2Cache();
+    (void)cudaGetLastError();
+  }
   c->pin = L2Window();
-  if (!c->l2_pin || !base || !bytes) return;
-  int max_persist = 0, max_window = 0;
+  if (c->l2_pin == 0 || !base || !bytes) return;
+  int max_persist = 0, max_window = 0, l2 = 0;
   cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, c->device);
   cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, c->device);
+  cudaDeviceGetAttribute(&l2, cudaDevAttrL2CacheSize, c->device);
   if (max_persist <= 0 || max_window <= 0) return;
+  if (c->l2_pin < 0 && (bytes > (size_t)l2 / 3 || bytes > (size_t)max_persist)) return;
   const size_t setaside = bytes < (size_t)max_persist ? bytes : (size_t)max_persist;
   if (cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, setaside) != cudaSuccess) {
     (void)cudaGetLastError();
@@ -301,7 +319,7 @@ glb_status glb_create(int device, glb_ctx** out) {
   if (const char* g = getenv("GLB_GATHER_BPS")) c->gather_bps = atoi(g) > 0 ? atoi(g) : 4;
   c->gather_bps_pipe = getenv("GLB_GATHER_BPS") ? c->gather_bps : 2;
   if (const char* g = getenv("GLB_GATHER_BPS_PIPE")) c->gather_bps_pipe = atoi(g) > 0 ? atoi(g) : 2;
-  if (const char* g = getenv("GLB_L2_PIN")) c->l2_pin = atoi(g) != 0;
+  if (const char* g = getenv("GLB_L2_PIN")) c->l2_pin = atoi(g) != 0 ? 1 : 0;
   if (const char* g = getenv("GLB_SAMPLE_BPS")) c->sample_bps = atoi(g) > 0 ? atoi(g) : 8;
   if (const char* g = getenv("GLB_CACHE_ALIGN")) c->cache_align = (uint32_t)atoi(g);
   if (const char* g = getenv("GLB_GATHER_ST")) c->gather_st_wb = atoi(g) != 0;
@@ -1077,6 +1095,12 @@ glb_status glb_set_relabel_mode(glb_ctx* c, int mode) {
   ENTER(c);
   if (mode < 0 || mode > 2) return set_err(c, GLB_EINVAL, "relabel mode must be 0 (auto), 1 (dense) or 2 (hash)");
   c->relabel_mode = mode;
+  return GLB_OK;
+}
+
+glb_status glb_relabel_l2_window(const glb_ctx* c, uint64_t* out) {
+  if (!c || !out) return GLB_EINVAL;
+  *out = c->pin.bytes;
   return GLB_OK;
 }
 

@@ -188,7 +188,7 @@ struct glb_ctx {
   bool hash_mode = false;
   int relabel_mode = 0;         // 0 auto, 1 dense, 2 hash (glb_set_relabel_mode)
   glb::L2Window pin;            // persisting-L2 window over the relabel table
-  bool l2_pin = false;          // GLB_L2_PIN=1 enables (measured slower: DESIGN.md)
+  int l2_pin = -1;              // -1 auto (small tables only), GLB_L2_PIN=0 off / 1 on
   uint32_t gen = 0;
 
   // cache (D3, D4, D5)
