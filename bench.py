@@ -620,8 +620,10 @@ def main():
     # ---- e2e through the public API with host buffers: every step copies its seeds from
     # pinned host memory (glb_sample_async, H2D on the ctx stream) and reads its result --
     # the extract's (hits, misses) -- back into pinned host memory (stream-ordered D2H);
-    # the host consumes step j-1's result while step j runs (a trainer's pattern).  Wall
-    # clock from the first call to the last result on the host.
+    # the host consumes the result of step j-D while step j runs (D = the pipeline depth:
+    # with depth 2 the extract of j-1 and the sampling of j are both in flight, so the host
+    # reads j-2 and keeps the next step enqueued ahead of the device).  Wall clock from the
+    # first call to the last result on the host.
     e2e_steps = steps[: max(1, min(len(steps), 200))]
     host_seeds = {}
     for i in e2e_steps:
@@ -636,6 +638,8 @@ def main():
                                      .view(np.int32).copy()).pin_memory()
     cnt_dev = ctx.extract_counts_tensor()
     cnt_host = torch.zeros((len(e2e_steps), 3), dtype=torch.int64).pin_memory()
+
+    lag = max(1, args.pipeline)
 
     def e2e_run(sync_api):
         evs = []
@@ -656,13 +660,13 @@ def main():
                     ev = torch.cuda.Event()
                     ev.record(xs)
                 evs.append(ev)
-                if j:
-                    evs[j - 1].synchronize()
-                    rows_seen += int(cnt_host[j - 1, 0] + cnt_host[j - 1, 1])
+                if j >= lag:
+                    evs[j - lag].synchronize()
+                    rows_seen += int(cnt_host[j - lag, 0] + cnt_host[j - lag, 1])
             seeds_done += n_seeds(b)
-        if evs:
-            evs[-1].synchronize()
-            rows_seen += int(cnt_host[-1, 0] + cnt_host[-1, 1])
+        for jj in range(max(0, len(evs) - lag), len(evs)):
+            evs[jj].synchronize()
+            rows_seen += int(cnt_host[jj, 0] + cnt_host[jj, 1])
         return time.perf_counter() - t0, seeds_done, rows_seen
 
     e2e_run(False)  # warm the pinned buffers / events
@@ -813,7 +817,8 @@ def main():
             "e2e": {"value": e2e_val, "unit": "seeds/s", "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": d2h, "steps": len(e2e_steps),
                     "api": "glb_sample_async(pinned host seeds) + glb_extract_sample + "
-                           "D2H of the step's counts (host reads step j-1 during step j)",
+                           "D2H of the step's counts (host reads step j-D during step j, "
+                           f"D = pipeline depth {lag})",
                     "rows_extracted": e2e_rows,
                     "sync_api_value": e2e_sync_val,
                     "sync_api": "glb_sample(host seeds; sizes D2H, sync) + glb_extract_sample "
