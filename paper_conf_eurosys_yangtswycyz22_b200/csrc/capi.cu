@@ -324,6 +324,7 @@ glb_status glb_create(int device, glb_ctx** out) {
   if (const char* g = getenv("GLB_CACHE_ALIGN")) c->cache_align = (uint32_t)atoi(g);
   if (const char* g = getenv("GLB_GATHER_ST")) c->gather_st_wb = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_BULK")) c->gather_bulk = atoi(g) != 0;
+  if (const char* g = getenv("GLB_MISS_BULK")) c->miss_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_BULK_SMEM")) c->gather_bulk_smem = (uint32_t)atoi(g);
   if (const char* g = getenv("GLB_PERM_PREFETCH")) c->perm_prefetch = atoi(g) != 0;
   *out = c;

@@ -152,12 +152,14 @@ __global__ void __launch_bounds__(kThreads, 4)
   __shared__ unsigned int s_next;
   uint32_t npeer = 0;
   const uint64_t nh_all = dev_counts ? dev_counts[0] : nh_host;
-  const uint64_t nm = dev_counts ? dev_counts[1] : nm_host;
+  const uint64_t nm_all = dev_counts ? dev_counts[1] : nm_host;
   if (xcount && blockIdx.x == 0 && threadIdx.x == 0) {
     xcount[0] = nh_all;
-    xcount[1] = nm;
+    xcount[1] = nm_all;
   }
-  const uint64_t nh = misses_only ? 0 : nh_all;  // hits gathered by k_gather_bulk instead
+  const uint64_t nm = (misses_only & 2) ? 0 : nm_all;
+  // skip bit 0: hits gathered by k_gather_bulk instead; bit 1: misses gathered by it
+  const uint64_t nh = (misses_only & 1) ? 0 : nh_all;
   const uint32_t t = threadIdx.x;
   const uint64_t nch = (nh + R - 1) / R, ncm = (nm + R - 1) / R;  // hit / miss chunks
   const float inv_u = 1.0f / (float)U;
@@ -349,7 +351,9 @@ __global__ void __launch_bounds__(64)
     k_gather_bulk(uint8_t* __restrict__ out, const uint8_t* __restrict__ src_hit,
                   const uint2* __restrict__ hit_list, const uint32_t* __restrict__ dev_counts,
                   uint64_t nh_host, uint32_t row_bytes, uint64_t src_stride, uint32_t P,
-                  unsigned long long* xcount, ShardTab tab) {
+                  unsigned long long* xcount, ShardTab tab, int which) {
+  // which 0: hit list (dst row, cache slot) from the HBM cache; 1: miss list (dst row, gid)
+  // from the mapped host matrix (src_hit = its device alias, dense rows)
   extern __shared__ __align__(128) uint8_t smem[];
   pdl_enter();
   const uint32_t lanes = blockDim.x;  // lanes of this block
@@ -364,10 +368,10 @@ __global__ void __launch_bounds__(64)
   for (uint32_t s = 0; s < P; ++s) mbar_init(bar(s), 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  const uint64_t nh = dev_counts ? dev_counts[0] : nh_host;
-  if (xcount && blockIdx.x == 0 && lane == 0) {
-    xcount[0] = nh;
-    xcount[1] = dev_counts ? dev_counts[1] : 0;  // rewritten by the miss gather if it runs
+  const uint64_t nh = dev_counts ? dev_counts[which] : nh_host;
+  if (xcount && blockIdx.x == 0 && lane == 0 && dev_counts) {
+    xcount[0] = dev_counts[0];
+    xcount[1] = dev_counts[1];
   }
   const uint64_t NL = (uint64_t)gridDim.x * lanes;
   const uint64_t gl = (uint64_t)blockIdx.x * lanes + lane;
@@ -491,11 +495,42 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
       cfg.numAttrs = 1;
       const uint64_t stride = 4ull * (c->cache_stride ? c->cache_stride : D);
       e = cudaLaunchKernelEx(&cfg, kern, (uint8_t*)out, (const uint8_t*)src_hit, hit_list,
-                             dev_counts, (uint64_t)nhit_host, row_bytes, stride, P, c->xcount, tab);
+                             dev_counts, (uint64_t)nhit_host, row_bytes, stride, P, c->xcount, tab, 0);
       count_launch(c);
       if (e != cudaSuccess) return e;
       if (c->C >= c->V) return cudaSuccess;  // every vertex cached: no misses to gather
       mo = 1;  // the misses follow on the LSU path (host memory over PCIe)
+    }
+  }
+  // misses through the bulk-copy engine (GLB_MISS_BULK=1): one cp.async.bulk per host row
+  if (c->miss_bulk && vec && hit_list && miss_list && !fill_src && out != c->cache &&
+      dev_counts && c->C < c->V) {
+    const uint32_t lanes = 32, row_bytes = 4 * D;
+    uint32_t P = (uint32_t)((uint64_t)c->gather_bulk_smem / ((uint64_t)lanes * row_bytes));
+    if (P > 16) P = 16;
+    if (P >= 2) {
+      const size_t smem = (((size_t)P * lanes * 12 + 127) & ~(size_t)127) + (size_t)P * lanes * row_bytes;
+      cudaError_t e;
+      if ((e = cudaFuncSetAttribute(k_gather_bulk<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem)) != cudaSuccess)
+        return e;
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3(c->num_sms);
+      cfg.blockDim = dim3(lanes);
+      cfg.dynamicSmemBytes = smem;
+      cfg.stream = c->stream;
+      cudaLaunchAttribute attr[1];
+      attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+      attr[0].val.programmaticStreamSerializationAllowed = 1;
+      cfg.attrs = attr;
+      cfg.numAttrs = 1;
+      ShardTab tab0 = {};
+      e = cudaLaunchKernelEx(&cfg, k_gather_bulk<false>, (uint8_t*)out, (const uint8_t*)src_miss,
+                             miss_list, dev_counts, (uint64_t)0, row_bytes, (uint64_t)row_bytes, P,
+                             c->xcount, tab0, 1);
+      count_launch(c);
+      if (e != cudaSuccess) return e;
+      if (mo) return cudaSuccess;  // hits were bulk-gathered too
+      mo = 2;                      // the LSU gather does the hits only
     }
   }
   // chunk counters of the launching stream (this ctx's gathers are serial on it; each

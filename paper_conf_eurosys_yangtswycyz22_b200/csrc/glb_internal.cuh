@@ -200,6 +200,7 @@ struct glb_ctx {
   int gather_bulk = 0;         // GLB_GATHER_BULK=1: hits through cp.async.bulk (k_gather_bulk);
                                // measured 2x slower than the LSU gather
   uint32_t gather_bulk_smem = 96 * 1024;  // row-slot bytes per bulk block (GLB_GATHER_BULK_SMEM)
+  int miss_bulk = 0;           // GLB_MISS_BULK=1: host misses through cp.async.bulk
   uint64_t C = 0;
   // NEXT-3 peer-sharded cache: global rank i < C is owned by shard i % W at row i / W;
   // shard_base[r] = device pointer (valid in this process) of shard r's rows.

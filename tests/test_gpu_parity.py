@@ -224,16 +224,18 @@ def test_presample_cache_and_hit_stats(tiny, mode):
         assert hs["hits"] <= hs["optimal_hits"]
 
 
-@pytest.mark.parametrize("mode", MODES + ["bulk"])
+@pytest.mark.parametrize("mode", MODES + ["bulk", "bulkmiss", "bulkboth"])
 @pytest.mark.parametrize("alpha", [0.0, 0.1, 0.5, 1.0])
 def test_extract_sample_bytes(tiny, alpha, mode, monkeypatch):
     """mode 'bulk': hits through the cp.async.bulk gather (GLB_GATHER_BULK=1, off by
     default), misses through the LSU gather."""
     g, go = tiny
     sh = g.shape
-    if mode == "bulk":
+    if mode in ("bulk", "bulkboth"):
         monkeypatch.setenv("GLB_GATHER_BULK", "1")
-    ctx = make_ctx(g, fanouts=sh.fanouts, mode="auto" if mode == "bulk" else mode)
+    if mode in ("bulkmiss", "bulkboth"):
+        monkeypatch.setenv("GLB_MISS_BULK", "1")
+    ctx = make_ctx(g, fanouts=sh.fanouts, mode=mode if mode in MODES else "auto")
     ctx.presample(1)
     ctx.build_cache(alpha)
     slot = ctx.cache_slots()
