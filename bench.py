@@ -64,7 +64,7 @@ def parse():
                    help="gloo: CPU-staged send/recv (lets N ranks share one GPU for testing)")
     p.add_argument("--relabel", default="auto", choices=["auto", "dense", "hash"],
                    help="relabel table (glb_set_relabel_mode)")
-    p.add_argument("--host-alloc", default="register", choices=["register", "cuda"],
+    p.add_argument("--host-alloc", default="register", choices=["register", "cuda", "thp"],
                    help="host feature memory: pageable + cudaHostRegister, or cudaHostAlloc")
     p.add_argument("--cache", default="replicated", choices=["replicated", "sharded"],
                    help="sharded: each rank caches alpha*V distinct rows, peers read them over "
@@ -451,6 +451,9 @@ def main():
     if args.host_alloc == "cuda":
         def alloc(nbytes):  # cudaHostAlloc'ed (pinned, mapped under UVA) via torch
             return torch.empty(nbytes, dtype=torch.uint8, pin_memory=True).numpy()
+    elif args.host_alloc == "thp":
+        def alloc(nbytes):  # 2 MB transparent huge pages (madvise), registered by load_graph
+            return synth.aligned_empty(nbytes, np.uint8, huge=True)
     g = synth.make_graph(sh, feature_alloc=alloc)
     t_gen = time.perf_counter() - t0
 

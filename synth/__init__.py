@@ -105,11 +105,21 @@ def seed_for(shape: Shape) -> int:
     return BASE_SEED + CONFIG_INDEX.get(shape.name, 9)
 
 
-def aligned_empty(n: int, dtype, align: int = 1 << 21) -> np.ndarray:
-    """Page-aligned host array (so it can be cudaHostRegister'ed whole)."""
+def aligned_empty(n: int, dtype, align: int = 1 << 21, huge: bool = False) -> np.ndarray:
+    """Page-aligned host array (so it can be cudaHostRegister'ed whole).  huge: anonymous
+    mmap advised MADV_HUGEPAGE (2 MB transparent huge pages where the kernel allows)."""
     dtype = np.dtype(dtype)
     nbytes = max(n * dtype.itemsize, 1)
-    raw = np.empty(nbytes + align, dtype=np.uint8)
+    if huge:
+        import mmap
+        m = mmap.mmap(-1, nbytes + align, flags=mmap.MAP_PRIVATE | mmap.MAP_ANONYMOUS)
+        try:
+            m.madvise(mmap.MADV_HUGEPAGE)
+        except (AttributeError, OSError):
+            pass
+        raw = np.frombuffer(m, dtype=np.uint8)
+    else:
+        raw = np.empty(nbytes + align, dtype=np.uint8)
     off = (-raw.ctypes.data) % align
     return raw[off:off + nbytes].view(dtype)[:n]
 
