@@ -368,6 +368,9 @@ __global__ void __launch_bounds__(64)
   for (uint32_t s = 0; s < P; ++s) mbar_init(bar(s), 1);
   asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  // the bulk-copy instructions take uniform operands: the compiler issues every lane's copy
+  // from one thread in turn, so another lane's barrier must be initialised first
+  __syncthreads();
   const uint64_t nh = dev_counts ? dev_counts[which] : nh_host;
   if (xcount && blockIdx.x == 0 && lane == 0 && dev_counts) {
     xcount[0] = dev_counts[0];
