@@ -53,6 +53,8 @@ def lib():
         L.synth_trainset.restype = i32
         L.synth_perm.argtypes = [u64, u64, u32, u64]
         L.synth_perm.restype = u64
+        L.synth_perm_fill.argtypes = [u64, u64, u32, vp]
+        L.synth_perm_fill.restype = None
         L.synth_edge_weights.argtypes = [u64, vp, u32, u64, vp, i32]
         L.synth_edge_weights.restype = i32
         _lib = L
@@ -212,3 +214,11 @@ def small_graph(V: int, E: int, gamma: float, D: int, n_train: int, seed: int,
     indptr, indices = gen_topology(V, E, gamma, gamma, seed, cap)
     return Graph(sh, seed, indptr, indices, gen_trainset(V, n_train, seed),
                  gen_features(V, D, seed))
+
+
+def rank_order(V: int, seed: int) -> np.ndarray:
+    """rank -> vertex map of the generator's degree ranks (rank 0 = the heaviest vertex;
+    in- and out-degree share it).  Tools only (e.g. hot-first renumbering experiments)."""
+    out = np.empty(V, np.uint32)
+    lib().synth_perm_fill(V, seed, 7, out.ctypes.data)
+    return out

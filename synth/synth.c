@@ -90,6 +90,12 @@ uint64_t synth_perm(uint64_t n, uint64_t seed, uint32_t tag, uint64_t x) {
   sy_perm p; sy_perm_init(&p, n, seed, tag); return sy_perm_apply(&p, x);
 }
 
+/* out[r] = perm(r) for r < n (the rank -> vertex map of the generator; tools only) */
+void synth_perm_fill(uint64_t n, uint64_t seed, uint32_t tag, uint32_t* out) {
+  sy_perm p; sy_perm_init(&p, n, seed, tag);
+  for (uint64_t r = 0; r < n; ++r) out[r] = (uint32_t)sy_perm_apply(&p, r);
+}
+
 /* ---- tiny parallel-for ---- */
 typedef void (*sy_body)(void* ctx, uint64_t lo, uint64_t hi);
 typedef struct { sy_body f; void* ctx; uint64_t n, chunk; uint64_t* next; pthread_mutex_t* mu; } sy_job;
