@@ -287,7 +287,9 @@ glb_status glb_extract_times(glb_ctx* ctx, float* out_ms, uint64_t max, uint64_t
  * Blobs are GLB_HANDOFF_BLOB_BYTES opaque bytes to exchange between processes (e.g. all-gathered
  * over torch.distributed); a peer in the same process is recognised and used directly.
  * Ids (trainer, sampler) are caller-chosen in [0, GLB_HANDOFF_MAX_PEERS), e.g. ranks.
- * glb_set_sampler and glb_destroy drop the ring and every attachment. */
+ * glb_set_sampler and glb_destroy drop the ring and every attachment; a ctx must not be
+ * destroyed (or re-configured) while a peer may still use its ring or events -- callers
+ * synchronise and barrier first. */
 #define GLB_HANDOFF_MAX_SLOTS 8
 #define GLB_HANDOFF_MAX_PEERS 16
 #define GLB_HANDOFF_BLOB_BYTES 2048
