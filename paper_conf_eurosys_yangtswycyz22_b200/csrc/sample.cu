@@ -439,8 +439,11 @@ __global__ void __launch_bounds__(kThreads)
 // PinSAGE (L209, L353): G >= walks lanes per frontier vertex, one walk per lane.
 // PinSAGE (L209, L353): G >= walks lanes per frontier vertex, one walk per lane;
 // LEN >= walk length (register arrays; 3 for PinSAGE).
+#ifndef GLB_RWALK_MINB  // min resident random-walk blocks per SM (register cap; A/B builds)
+#define GLB_RWALK_MINB 1
+#endif
 template <int G, int LEN, bool HASH>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads, GLB_RWALK_MINB)
     k_rwalk(uint32_t hop, uint32_t walks, uint32_t len, uint32_t topk, uint64_t seed,
             uint32_t epoch, uint32_t batch, Table T, const DevState* __restrict__ st,
             DevState* st_w, const uint64_t* __restrict__ indptr,
