@@ -2,18 +2,27 @@
 """Benchmark: GNNLab sample+extract hot path on B200 (BASELINE.json metric).
 
 One step = one mini-batch through the whole per-batch path: epoch shuffle
-(a1, at epoch boundaries), k-hop sampling (a2), dedup/relabel into blocks
+(a1, at epoch boundaries), sampling (a2 / a2'), dedup/relabel into blocks
 (a3), mark (a4) and feature extract (a7) from the PreSC cache (a5/a6 run
 once before the timed region, timed separately like Table 6, PAPER.md
-L468-474).  Workload: configs[1] (ogbn-products-shaped PR, GraphSAGE [25,10],
-batch 8000), synthetic (synth/), alpha = 1.0 (the paper's R% for GSG-PR,
-Table 5); the alpha sweep reports hit rate vs Optimal and seeds/s.
+L468-474).
+
+Default workload (the headline): BASELINE.json configs[3], the largest
+single-GPU configuration -- Papers100M-shaped synthetic graph (111 M vertices,
+1.6 B edges, feat 128), PinSAGE random walks (3 layers x 4 walks of length 3,
+top-5), batch 8000, PreSC#1, cache ratio alpha = 0.22 (the paper's R% for
+PSG-PA, Table 5): 78 % of the vertices stay in pinned host memory, so the
+extract is bound by the host link.  The line also carries
+`pr_alpha1` (configs[1], Products-shaped, alpha = 1: every row an HBM hit).
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
 
-Under torchrun each rank owns one GPU; batches shard round-robin (batch
-g = i*N + rank); the only collective is the all-reduce of PreSC counts
-(and the max-over-ranks timing).  Rank 0 prints ONE JSON line.
+--gpus N without a launcher re-executes itself under torch.distributed.run
+(one rank per GPU).  Under torchrun each rank owns one GPU; batches shard
+round-robin (batch g = i*N + rank); the only collective is the all-reduce of
+PreSC counts (and the max-over-ranks timing).  Host inputs are generated once
+per node and mapped by every local rank (synth/shm.py).  Rank 0 prints ONE
+JSON line.
 """
 from __future__ import annotations
 
@@ -21,7 +30,9 @@ import argparse
 import json
 import math
 import os
+import socket
 import statistics
+import subprocess
 import sys
 import time
 
@@ -33,19 +44,25 @@ sys.path.insert(0, ROOT)
 import synth  # noqa: E402
 
 METRIC = "sample+extract seeds/sec at 1/2/4/8 B200; cache hit rate vs optimal (%)"
+PCIE_GEN5_X16_GBS = 64.0  # nominal per direction (context only)
 
 
-def parse():
+def parse(argv=None):
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
-    p.add_argument("--steps", type=int, default=400)
+    p.add_argument("--steps", type=int, default=20)
     p.add_argument("--warmup", type=int, default=5)
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    p.add_argument("--config", default="PR", choices=list(synth.SHAPES))
-    p.add_argument("--alpha", type=float, default=1.0)
+    p.add_argument("--config", default="PA", choices=list(synth.SHAPES))
+    p.add_argument("--alpha", type=float, default=None,
+                   help="cache ratio (default: the shape's paper R%%, synth.SHAPES alphas[0])")
+    p.add_argument("--runs", type=int, default=3,
+                   help="timed regions of K steps each; value = their median (SURVEY §8(d))")
     p.add_argument("--sweep-steps", type=int, default=10)
     p.add_argument("--no-sweep", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-pr-alpha1", action="store_true",
+                   help="skip the extra PR alpha=1 (all-HBM-hit) measurement")
     p.add_argument("--cpu-seconds", type=float, default=15.0)
     p.add_argument("--measure-epochs", type=int, default=10,
                    help="epochs whose accesses define H and the Optimal H* (L148 fn4)")
@@ -53,6 +70,10 @@ def parse():
                    help="PreSC#K values for the Fig 11(a) analog (empty: skip)")
     p.add_argument("--mode", default="dp", choices=["dp", "factored"],
                    help="factored: Ns sampler + Nt trainer ranks (PAPER.md §5.2-5.3)")
+    p.add_argument("--ns", type=int, default=0,
+                   help="factored: force Ns sampler ranks (0: adaptive, Ns = ceil(N/(K+1)))")
+    p.add_argument("--ns-sweep", action="store_true",
+                   help="factored: also run every Ns in 1..N-1 (Fig 15 analog, L458-476)")
     p.add_argument("--handoff", default="peer", choices=["peer", "sendrecv"],
                    help="factored mode: peer = samples pushed into the trainer's HBM ring by one "
                         "copy kernel (glb_handoff_*, NVLink/IPC); sendrecv = torch.distributed "
@@ -66,6 +87,8 @@ def parse():
                    help="relabel table (glb_set_relabel_mode)")
     p.add_argument("--host-alloc", default="register", choices=["register", "cuda", "thp"],
                    help="host feature memory: pageable + cudaHostRegister, or cudaHostAlloc")
+    p.add_argument("--shared-inputs", default="auto", choices=["auto", "on", "off"],
+                   help="one copy of the host inputs per node, mapped by every local rank")
     p.add_argument("--cache", default="replicated", choices=["replicated", "sharded"],
                    help="sharded: each rank caches alpha*V distinct rows, peers read them over "
                         "NVLink (NEXT-3; glb_build_cache_sharded)")
@@ -73,14 +96,39 @@ def parse():
                    help="CUDA events around every n-th extract launch of the timed region")
     p.add_argument("--pipeline", type=int, default=2, choices=[1, 2],
                    help="2: extract of batch b overlaps sampling of batch b+1 (two streams)")
-    return p.parse_args()
+    a = p.parse_args(argv)
+    if a.alpha is None:
+        a.alpha = synth.SHAPES[a.config].alphas[0]
+    return a
 
 
 def dist_env():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    return world, rank, local
+    local_world = int(os.environ.get("LOCAL_WORLD_SIZE", str(world)))
+    return world, rank, local, local_world
+
+
+def free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def launch_ranks(n, argv, capture=False):
+    """Run this script under torch.distributed.run with n ranks on this node."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()),
+           os.path.abspath(__file__)] + list(argv)
+    if capture:
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        sys.stderr.write(r.stderr[-4000:])
+        lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+        return r.returncode, (json.loads(lines[-1]) if lines else None)
+    return subprocess.call(cmd), None
 
 
 def workload_name(sh, alpha):
@@ -97,6 +145,80 @@ def read_peaks():
         d = json.load(open(p))
         return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def host_info():
+    """CPU model (lscpu), usable cores, NUMA nodes of this host (SURVEY §8(d) protocol)."""
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for ln in out.splitlines():
+            if ln.startswith("Model name:"):
+                model = ln.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    if model is None:
+        try:
+            for ln in open("/proc/cpuinfo"):
+                if ln.startswith("model name"):
+                    model = ln.split(":", 1)[1].strip()
+                    break
+        except OSError:
+            pass
+    try:
+        ncpu = len(os.sched_getaffinity(0))
+    except AttributeError:
+        ncpu = os.cpu_count() or 1
+    import glob
+    nodes = len(glob.glob("/sys/devices/system/node/node[0-9]*")) or 1
+    return {"cpu_model": model, "nproc": ncpu, "numa_nodes": nodes}
+
+
+def gpu_info(index):
+    """Driver, ECC, clocks, PCIe link and NUMA affinity of the GPU (nvidia-smi -q fields)."""
+    try:
+        import pynvml as nv
+        nv.nvmlInit()
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+        phys = int(vis.split(",")[index]) if vis and vis.split(",")[0].isdigit() else index
+        h = nv.nvmlDeviceGetHandleByIndex(phys)
+        d = {"name": nv.nvmlDeviceGetName(h), "driver": nv.nvmlSystemGetDriverVersion()}
+        for k, f in (("ecc_mode", lambda: nv.nvmlDeviceGetCurrentEccMode(h)),
+                     ("sm_max_mhz", lambda: nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)),
+                     ("mem_max_mhz", lambda: nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_MEM)),
+                     ("pcie_gen", lambda: nv.nvmlDeviceGetCurrPcieLinkGeneration(h)),
+                     ("pcie_width", lambda: nv.nvmlDeviceGetCurrPcieLinkWidth(h)),
+                     ("numa_node", lambda: nv.nvmlDeviceGetNumaNodeId(h))):
+            try:
+                d[k] = f()
+            except Exception:
+                d[k] = None
+        return d
+    except Exception as e:  # noqa: BLE001
+        return {"error": str(e)[:120]}
+
+
+def hostlink_peak(dev):
+    """Measured host->device link peak for the roofline, in this run: DMA of 1 GiB pinned
+    host memory to HBM (copy engine), best of 5, CUDA events on the copying stream."""
+    import torch
+    n = 1 << 30
+    h = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+    h[::4096] = 1
+    d = torch.empty(n, dtype=torch.uint8, device=dev)
+    s = torch.cuda.current_stream(dev)
+    d.copy_(h, non_blocking=True)
+    best = 0.0
+    for _ in range(5):
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        d.copy_(h, non_blocking=True)
+        e1.record(s)
+        e1.synchronize()
+        best = max(best, n / (e0.elapsed_time(e1) * 1e-3) / 1e9)
+    del h, d
+    return best
 
 
 class Clocks:
@@ -163,7 +285,7 @@ def reference_arm(args):
     cores: the W warm-up and K timed mini-batches are spread over P threads (one
     GraphOracle scratch each; the oracle's C calls release the GIL), value = timed seeds /
     wall time of the timed batches."""
-    world, rank, _ = dist_env()
+    world, rank, _, _ = dist_env()
     if rank != 0:
         return
     import concurrent.futures as cf
@@ -199,12 +321,14 @@ def reference_arm(args):
         tot_s = sum(ex.map(run, jobs_t))
         tot_t = time.perf_counter() - t0
     v = tot_s / tot_t
+    hi = host_info()
     line = {
         "impl": "reference", "metric": METRIC, "value": v, "unit": "seeds/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot_t / args.steps,
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
         "data": "synthetic", "config": {"workload": workload_name(sh, args.alpha)},
         "cpu_baseline": {"value": v, "unit": "seeds/s", "cores": P, "kind": "oracle",
+                         "cpu_model": hi["cpu_model"], "nproc": hi["nproc"],
                          "sample": f"{args.steps} full mini-batches (sample+relabel+extract) over "
                                    f"{P} threads, single-threaded C oracle per thread"},
         "e2e": {"value": v, "unit": "seeds/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -244,13 +368,16 @@ def cpu_baseline(g, sh, budget_s):
         t_tot += time.perf_counter() - t0
         seeds += len(bs[nb])
         nb += 1
+    hi = host_info()
     single = {"value": seeds / t_tot, "unit": "seeds/s", "cores": 1, "kind": "oracle",
               "sample": f"{nb} mini-batches of epoch {sh.K} (sample+relabel+extract, "
                         f"{seeds} seeds, {t_tot:.1f} s), single-threaded C oracle"}
     par = cpu_baseline_parallel(go, g, sh, bs, max(2.0, budget_s * 2 / 3))
     if par is None:
+        single.update({"cpu_model": hi["cpu_model"], "nproc": hi["nproc"]})
         return single
     par["single_thread"] = single
+    par.update({"cpu_model": hi["cpu_model"], "nproc": hi["nproc"]})
     return par
 
 
@@ -303,8 +430,8 @@ def cpu_baseline_parallel(go, g, sh, bs, budget_s):
 # ------------------------------------------------------------------------------------------
 def run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_cache, par, glb):
     """Factored mode (§5.2-5.3): profile Ts/Tt, split ranks into Ns samplers
-    and Nt trainers (Ns = ceil(N/(K+1)), K = Tt/Ts, L262), then samplers pull batches
-    from the global scheduler and hand samples to trainers, which extract."""
+    and Nt trainers (Ns = ceil(N/(K+1)), K = Tt/Ts, L262; or --ns), then samplers pull
+    batches from the global scheduler and hand samples to trainers, which extract."""
     import torch
     import torch.distributed as dist
     cpu_comm = args.backend == "gloo"
@@ -327,11 +454,12 @@ def run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_c
         prof = prof.to(comm_dev)
         dist.all_reduce(prof)
         prof = prof.cpu() / world
-    ns = par.num_samplers(world, float(prof[0]), float(prof[1]))
+    ns_adaptive = par.num_samplers(world, float(prof[0]), float(prof[1]))
+    ns = min(max(args.ns, 1), world - 1) if (args.ns and world > 1) else ns_adaptive
     roles = par.Roles(ns, world)
     total = args.steps * world
     store = dist.distributed_c10d._get_default_store() if world > 1 else None
-    tag = "bench"
+    tag = f"bench{ns}"
     seeds = {"n": 0}
 
     def sample_fn(gidx):
@@ -410,7 +538,8 @@ def run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_c
                 "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
                 "data": "synthetic",
                 "config": {"workload": workload_name(sh, args.alpha), "mode": "factored",
-                           "samplers": ns, "trainers": world - ns,
+                           "samplers": ns, "trainers": world - ns, "ns_adaptive": ns_adaptive,
+                           "ns_forced": bool(args.ns),
                            "Ts_ms": 1e3 * float(prof[0]), "Tt_ms": 1e3 * float(prof[1]),
                            "backend": args.backend, "parallelism": f"factored{ns}s{world - ns}t",
                            "handoff": (f"peer ({args.handoff_slots}-slot HBM ring per trainer, "
@@ -424,60 +553,69 @@ def run_factored(args, ctx, g, sh, out, nb, world, rank, dev, stream, t_pre, t_c
         dist.destroy_process_group()
 
 
-def main():
-    args = parse()
-    if args.impl == "reference":
-        return reference_arm(args)
+# ------------------------------------------------------------------------------------------
+def sampling_bytes(sh, sizes, nnz):
+    """Algorithmic HBM bytes of sampling one batch: k-hop 32 B per frontier
+    vertex (indptr pair) + 72 B per sampled edge (index sector, padded write, relabel probe,
+    compaction); random walk 64 B per walk step (indptr + index sectors) + 40 B per kept
+    edge (relabel probe, compaction)."""
+    L = len(nnz)
+    if sh.sampler == "rwalk":
+        return sum(sizes[l] * synth.RW_WALKS * synth.RW_LEN * 64 + 40 * nnz[l] for l in range(L))
+    return sum(32 * sizes[l] + 72 * nnz[l] for l in range(L))
+
+
+def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, full,
+                 link_peak):
+    """One workload through the DP path: inputs, load, PreSC, cache, `args.runs` timed
+    regions of K steps, the untimed replay that counts each launch's units, the depth-1
+    isolated extract replay, e2e through the public API, and (full) the hit-rate sweeps
+    and the CPU oracle baseline.  Returns the fields of the JSON line."""
     import torch
     import torch.distributed as dist
 
     import paper_conf_eurosys_yangtswycyz22_b200 as glb
     from paper_conf_eurosys_yangtswycyz22_b200 import parallel as par
 
-    world, rank, local = dist_env()
-    local = local % torch.cuda.device_count()
-    if world > 1:
-        torch.cuda.set_device(local)
-        if args.backend == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        else:
-            dist.init_process_group("gloo")
-    dev = torch.device("cuda", local)
-    torch.cuda.set_device(dev)
-    sh = synth.SHAPES[args.config]
+    def barrier():
+        if world > 1:
+            dist.barrier()
 
     t0 = time.perf_counter()
-    alloc = None
-    if args.host_alloc == "cuda":
-        def alloc(nbytes):  # cudaHostAlloc'ed (pinned, mapped under UVA) via torch
-            return torch.empty(nbytes, dtype=torch.uint8, pin_memory=True).numpy()
-    elif args.host_alloc == "thp":
-        def alloc(nbytes):  # 2 MB transparent huge pages (madvise), registered by load_graph
-            return synth.aligned_empty(nbytes, np.uint8, huge=True)
-    g = synth.make_graph(sh, feature_alloc=alloc)
+    shared = None
+    use_shared = world > 1 and local_world > 1 and args.shared_inputs != "off"
+    if use_shared:
+        from synth import shm
+        store = dist.distributed_c10d._get_default_store()
+        shared = shm.make_graph_shared(sh, local, local_world, store)
+        g = shared.graph
+    else:
+        alloc = None
+        if args.host_alloc == "cuda":
+            def alloc(nbytes):  # cudaHostAlloc'ed (pinned, mapped under UVA) via torch
+                return torch.empty(nbytes, dtype=torch.uint8, pin_memory=True).numpy()
+        elif args.host_alloc == "thp":
+            def alloc(nbytes):  # 2 MB transparent huge pages (madvise), registered by load_graph
+                return synth.aligned_empty(nbytes, np.uint8, huge=True)
+        g = synth.make_graph(sh, feature_alloc=alloc)
+    barrier()
     t_gen = time.perf_counter() - t0
 
     ctx = glb.Context(local)
-    stream = torch.cuda.current_stream(dev)
     ctx.set_stream(stream)
     t0 = time.perf_counter()
     ctx.load_graph(g.indptr, g.indices, g.features)
     t_load = time.perf_counter() - t0
-    kind = sh.sampler
     ctx.set_relabel_mode(args.relabel)
     if g.weights is not None:
         ctx.load_edge_weights(g.weights)
-    if kind in ("khop", "weighted"):
-        ctx.set_sampler(kind, fanouts=sh.fanouts, max_batch=sh.batch)
+    if sh.sampler in ("khop", "weighted"):
+        ctx.set_sampler(sh.sampler, fanouts=sh.fanouts, max_batch=sh.batch)
     else:
         ctx.set_sampler("rwalk", layers=len(sh.fanouts), walks=synth.RW_WALKS,
                         walk_len=synth.RW_LEN, topk=sh.fanouts[0], max_batch=sh.batch)
     ctx.set_train_set(g.train, sh.batch, g.seed)
     nb = ctx.num_batches
-
-    def barrier():
-        if world > 1:
-            dist.barrier()
 
     # ---- preprocessing (Table 6 analog): PreSC#K and load_cache
     barrier()
@@ -496,9 +634,9 @@ def main():
     t_pre = time.perf_counter() - t0
     t0 = time.perf_counter()
     if args.cache == "sharded":
-        par.build_sharded_cache(ctx, args.alpha, rank, world)
+        par.build_sharded_cache(ctx, alpha, rank, world)
     else:
-        ctx.build_cache(args.alpha)
+        ctx.build_cache(alpha)
     torch.cuda.synchronize()
     t_cache = time.perf_counter() - t0
 
@@ -529,48 +667,54 @@ def main():
     ctx.sync()
     torch.cuda.synchronize()
 
-    # ---- timed region: device time, CUDA events on the launching streams (sampling on the
-    # main stream, extract on the extract stream; the last kernel of the region is an extract)
-    steps = list(range(args.warmup, args.warmup + args.steps))
+    # ---- timed regions: device time, CUDA events on the launching streams (sampling on the
+    # main stream, extract on the extract stream; the last kernel of a region is an extract).
+    # Run r times steps [W + r*K, W + (r+1)*K): different batches, same protocol.
+    K = args.steps
     clocks = Clocks(local)
     launches0 = ctx.launches
-    barrier()
-    torch.cuda.synchronize()
     ctx.set_timing(args.time_every)  # events around every time_every-th extract launch
     clocks.start()
-    t_start = torch.cuda.Event(enable_timing=True)
-    t_end = torch.cuda.Event(enable_timing=True)
-    t_start.record(stream)
-    wall0 = time.perf_counter()
-    seeds_done = 0
-    for i in steps:
-        e, b = batch_of(i)
-        ctx.sample_batch(e, b)
-        ctx.extract_sample(out)
-        seeds_done += n_seeds(b)
-    t_end.record(xs)
-    enqueue_ms = 1e3 * (time.perf_counter() - wall0)
-    torch.cuda.synchronize()
-    wall_ms = 1e3 * (time.perf_counter() - wall0)
-    barrier()
+    runs, run_ms, enq_ms, wall_ms = [], [], [], []
+    for r in range(args.runs):
+        steps = range(args.warmup + r * K, args.warmup + (r + 1) * K)
+        barrier()
+        torch.cuda.synchronize()
+        t_start = torch.cuda.Event(enable_timing=True)
+        t_end = torch.cuda.Event(enable_timing=True)
+        t_start.record(stream)
+        wall0 = time.perf_counter()
+        seeds_done = 0
+        for i in steps:
+            e, b = batch_of(i)
+            ctx.sample_batch(e, b)
+            ctx.extract_sample(out)
+            seeds_done += n_seeds(b)
+        t_end.record(xs)
+        enq_ms.append(1e3 * (time.perf_counter() - wall0))
+        torch.cuda.synchronize()
+        wall_ms.append(1e3 * (time.perf_counter() - wall0))
+        barrier()
+        el = torch.tensor([t_start.elapsed_time(t_end)], dtype=torch.float64, device=dev)
+        tot = torch.tensor([float(seeds_done)], dtype=torch.float64, device=dev)
+        if world > 1:
+            if args.backend == "gloo":
+                el, tot = el.cpu(), tot.cpu()
+            dist.all_reduce(el, op=dist.ReduceOp.MAX)
+            dist.all_reduce(tot)
+        run_ms.append(float(el.item()))
+        runs.append(float(tot.item()) / (float(el.item()) / 1e3))
     clk = clocks.stop()
-    launches = ctx.launches - launches0
+    launches = (ctx.launches - launches0) / args.runs
     x_ms = ctx.extract_times()
     ctx.set_timing(False)
-    elapsed_ms = t_start.elapsed_time(t_end)
-    el = torch.tensor([elapsed_ms], dtype=torch.float64, device=dev)
-    tot = torch.tensor([float(seeds_done)], dtype=torch.float64, device=dev)
-    if world > 1:
-        if args.backend == "gloo":
-            el, tot = el.cpu(), tot.cpu()
-        dist.all_reduce(el, op=dist.ReduceOp.MAX)
-        dist.all_reduce(tot)
-    elapsed_max = float(el.item())
-    value = float(tot.item()) / (elapsed_max / 1e3)
+    med = sorted(range(args.runs), key=lambda j: runs[j])[args.runs // 2]
+    value, elapsed_max = runs[med], run_ms[med]
+    timed_steps = list(range(args.warmup, args.warmup + args.runs * K))
 
     # ---- replay (untimed) to count the units each timed launch processed
-    nL, hits, misses = [], [], []
-    for i in steps:
+    nL, hits, misses, samp_b = [], [], [], []
+    for i in timed_steps:
         e, b = batch_of(i)
         ctx.sample_batch(e, b)
         s = ctx.sample_result()
@@ -578,19 +722,27 @@ def main():
         nL.append(s.sizes[-1])
         hits.append(st["hits"])
         misses.append(st["misses"])
+        samp_b.append(sampling_bytes(sh, s.sizes, s.nnz))
     D = sh.D
-    # algorithmic HBM bytes of the extract launch: per row read (hit: cache row from
-    # HBM) + write of the out row + the 8-byte (dst, src) work-list entry.
+    hbm_peak, hbm_src = read_peaks()
+    # algorithmic HBM bytes of the extract launch: per row read (hit: cache row from HBM) +
+    # write of the out row + the 8-byte (dst, src) work-list entry; host-link bytes: the
+    # miss rows read over PCIe
     hbm_bytes = [h * (2 * 4 * D + 8) + m * (4 * D + 8) for h, m in zip(hits, misses)]
-    timed_bytes = hbm_bytes[:: args.time_every][: len(x_ms)]  # the sampled launches
-    ach_gbs = statistics.mean(bb / (t * 1e-3) for bb, t in zip(timed_bytes, x_ms)) / 1e9
-    peak, peak_src = read_peaks()
-    # ---- the same extract launches without the overlapping sampler (pipeline depth 1):
-    # k_gather's own efficiency, CUDA events on its stream, same batches as the replay
+    link_bytes = [m * 4 * D for m in misses]
+    sel = list(range(0, len(timed_steps), args.time_every))[: len(x_ms)]  # the timed launches
+    ach_hbm = statistics.mean(hbm_bytes[j] / (t * 1e-3) for j, t in zip(sel, x_ms)) / 1e9
+    ach_link = statistics.mean(link_bytes[j] / (t * 1e-3) for j, t in zip(sel, x_ms)) / 1e9
+    x_mean = statistics.mean(x_ms)
+    # the extract's binding roof: hits (HBM) and misses (host link) overlap in one launch
+    bound_ms = statistics.mean(max(hbm_bytes[j] / hbm_peak, link_bytes[j] / link_peak) / 1e6
+                               for j in sel)
+    host_bound = statistics.mean(link_bytes) / link_peak > statistics.mean(hbm_bytes) / hbm_peak
+    # ---- the same extract launches without the overlapping sampler (pipeline depth 1)
     iso = None
     if args.pipeline == 2:
         ctx.set_pipeline(1)
-        iso_steps = steps[: min(len(steps), 100)]
+        iso_steps = timed_steps[: min(len(timed_steps), 100)]
         torch.cuda.synchronize()
         ctx.set_timing(True)
         i0 = torch.cuda.Event(enable_timing=True)
@@ -608,26 +760,58 @@ def main():
         ctx.set_timing(False)
         ctx.set_pipeline(2)
         ims = i0.elapsed_time(i1)
-        a_iso = statistics.mean(bb / (t * 1e-3) for bb, t in zip(hbm_bytes, xi)) / 1e9
-        iso = {"pipeline_depth": 1, "steps": len(iso_steps), "achieved": a_iso,
-               "frac": a_iso / peak, "extract_ms_per_step": statistics.mean(xi),
-               "ms_per_step": ims / len(iso_steps), "seeds_per_s": sd / (ims / 1e3)}
+        a_hbm = statistics.mean(bb / (t * 1e-3) for bb, t in zip(hbm_bytes, xi)) / 1e9
+        a_link = statistics.mean(bb / (t * 1e-3) for bb, t in zip(link_bytes, xi)) / 1e9
+        iso = {"pipeline_depth": 1, "steps": len(iso_steps),
+               "achieved": a_link if host_bound else a_hbm,
+               "frac": (a_link / link_peak) if host_bound else (a_hbm / hbm_peak),
+               "hbm_achieved": a_hbm, "hbm_frac": a_hbm / hbm_peak,
+               "extract_ms_per_step": statistics.mean(xi),
+               "ms_per_step": ims / len(iso_steps), "seeds_per_s": world * sd / (ims / 1e3)}
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         tj = json.load(open(tp))
-        key = f"{sh.name}:{args.alpha}"
-        if key in tj:
-            traffic = tj[key]
+        traffic = tj.get(f"{sh.name}:{alpha}")
+    hbm_obj = {"achieved": ach_hbm, "peak": hbm_peak, "unit": "GB/s", "frac": ach_hbm / hbm_peak,
+               "peak_source": hbm_src,
+               "algorithmic_bytes_per_launch": statistics.mean(hbm_bytes[j] for j in sel)}
+    link_obj = {"achieved": ach_link, "peak": link_peak, "unit": "GB/s",
+                "frac": ach_link / link_peak,
+                "peak_source": "DMA H2D of 1 GiB pinned host memory, best of 5, measured in "
+                               f"this run (PCIe Gen5 x16 nominal {PCIE_GEN5_X16_GBS:.0f} GB/s)",
+                "algorithmic_bytes_per_launch": statistics.mean(link_bytes[j] for j in sel)}
+    if host_bound:
+        roof = {"kernel": "k_gather (extract a7)", "bound": "host-link", **link_obj,
+                "traffic": traffic, "hbm": hbm_obj}
+    else:
+        roof = {"kernel": "k_gather (extract a7)", "bound": "hbm", **hbm_obj, "traffic": traffic,
+                "host_link": link_obj}
+    roof.update({
+        "extract_ms_per_step": x_mean,
+        "extract_share_of_step": x_mean / (elapsed_max / K),
+        "kernel_bound_ms": bound_ms, "frac_of_binding_bound": bound_ms / x_mean,
+        "timed_launches": f"every {args.time_every}th extract of the {args.runs} timed regions "
+                          f"({len(x_ms)} launches)",
+        "measured_with": f"pipeline depth {args.pipeline} (the timed region)",
+        "isolated": iso})
+    # the whole step's roof: sampling + extract HBM bytes against HBM, misses against the
+    # host link, the two overlapping (SURVEY §8(d) "End-to-end bound per batch")
+    step_bound = statistics.mean(max((samp_b[j] + hbm_bytes[j]) / hbm_peak,
+                                     link_bytes[j] / link_peak) / 1e6
+                                 for j in range(len(timed_steps)))
+    path = {"bound_ms_per_step": step_bound, "measured_ms_per_step": elapsed_max / K,
+            "frac": step_bound / (elapsed_max / K),
+            "sampling_bytes_per_step": statistics.mean(samp_b),
+            "extract_hbm_bytes_per_step": statistics.mean(hbm_bytes),
+            "host_link_bytes_per_step": statistics.mean(link_bytes)}
 
     # ---- e2e through the public API with host buffers: every step copies its seeds from
     # pinned host memory (glb_sample_async, H2D on the ctx stream) and reads its result --
-    # the extract's (hits, misses) -- back into pinned host memory (stream-ordered D2H);
-    # the host consumes the result of step j-D while step j runs (D = the pipeline depth:
-    # with depth 2 the extract of j-1 and the sampling of j are both in flight, so the host
-    # reads j-2 and keeps the next step enqueued ahead of the device).  Wall clock from the
-    # first call to the last result on the host.
-    e2e_steps = steps[: max(1, min(len(steps), 200))]
+    # the extract's (hits, misses, peer hits) -- back into pinned host memory (stream-ordered
+    # D2H); the host consumes the result of step j-D while step j runs (D = the pipeline
+    # depth).  Wall clock from the first call to the last result on the host.
+    e2e_steps = timed_steps[: max(1, min(len(timed_steps), 200))]
     host_seeds = {}
     for i in e2e_steps:
         e, b = batch_of(i)
@@ -641,7 +825,6 @@ def main():
                                      .view(np.int32).copy()).pin_memory()
     cnt_dev = ctx.extract_counts_tensor()
     cnt_host = torch.zeros((len(e2e_steps), 3), dtype=torch.int64).pin_memory()
-
     lag = max(1, args.pipeline)
 
     def e2e_run(sync_api):
@@ -688,159 +871,228 @@ def main():
     e2e_sync_val = float(e2e_n[1].item()) / float(e2e_t[1].item())
     h2d = 4 * statistics.mean(n_seeds(batch_of(i)[1]) for i in e2e_steps)
     d2h = 24  # the step's (hits, misses, peer hits) u64 result
+    e2e = {"value": e2e_val, "unit": "seeds/s", "h2d_bytes_per_step": h2d,
+           "d2h_bytes_per_step": d2h, "steps": len(e2e_steps),
+           "api": "glb_sample_async(pinned host seeds) + glb_extract_sample + "
+                  "D2H of the step's counts (host reads step j-D during step j, "
+                  f"D = pipeline depth {lag})",
+           "result_read_back": "the step's (hits, misses, peer hits) u64 counts; the gathered "
+                               "features and blocks stay in HBM for the on-GPU consumer "
+                               "(GNNLab's Trainer trains on the GPU, L252), so they do not "
+                               "cross the host link",
+           "rows_extracted": e2e_rows, "sync_api_value": e2e_sync_val,
+           "sync_api": "glb_sample(host seeds; sizes D2H, sync) + glb_extract_sample "
+                       "+ stats (sync) every step"}
+
+    res = {"value": value, "ms_per_step": elapsed_max / K, "runs": runs,
+           "runs_range": [min(runs), max(runs)], "runs_ms": run_ms,
+           "roofline": roof, "path_roofline": path, "e2e": e2e, "gpu_launches": launches,
+           "clocks": clk, "host_wall_ms_timed_region": wall_ms[med],
+           "host_enqueue_ms_timed_region": enq_ms[med],
+           "units": {"mean_n_L": statistics.mean(nL), "mean_hits": statistics.mean(hits),
+                     "mean_misses": statistics.mean(misses)},
+           "preprocess_s": {"generate_inputs": t_gen, "load_graph": t_load,
+                            "presample": t_pre, "build_cache": t_cache},
+           "cache": {"layout": args.cache, "rows_cached": ctx_cache_rows},
+           "relabel_table": ctx.relabel_mode, "relabel_l2_window_bytes": ctx.relabel_l2_window,
+           "host_inputs": ("node-shared memfd, generated once by local rank 0 and mapped by "
+                           f"{local_world} ranks") if shared else "private to this rank"}
 
     # ---- hit rate vs Optimal (accesses recorded over measured epochs, untimed)
-    result_hit = None
-    sweep = []
-    k_sweep = []
-    similarity = None
-    peer_share = None
     if args.cache == "sharded":
-        # share of extracted rows served by another rank's shard (last replayed batch)
         k = ctx.last_extract_counts()
-        peer_share = k["peer_hits"] / max(1, k["hits"] + k["misses"])
+        res["cache"]["peer_hit_share"] = k["peer_hits"] / max(1, k["hits"] + k["misses"])
         barrier()  # peers may still read this rank's shard: nobody rebuilds before here
-    if not args.no_sweep:
-        def reduce_counts(t):
-            if world > 1:
-                c = t if args.backend == "nccl" else t.cpu()
-                par.allreduce_counts(c)
-                if c is not t:
-                    t.copy_(c)
-            return t
+    if full and not args.no_sweep:
+        res.update(hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs,
+                                   batch_of, n_seeds, barrier))
+    if full and rank == 0 and world == 1 and not args.no_cpu_baseline:
+        res["cpu_baseline"] = cpu_baseline(g, sh, args.cpu_seconds)
+    ctx.close()
+    del out
+    torch.cuda.empty_cache()
+    return res
 
-        # per-epoch access footprints of the measured epochs: Table 2 similarity of the
-        # first two, and their sum over all measured epochs for H and Optimal H* ("all
-        # sample footprints are recorded ... after training", L148 fn4)
-        per_epoch = []
-        acc_sum = None
-        # measured epochs start after every presample epoch of the K sweep (no overlap)
-        m0 = max([sh.K] + [int(x) for x in args.k_sweep.split(",") if x])
-        for e in range(m0, m0 + args.measure_epochs):
-            ctx.reset_counts(glb.COUNT_ACCESS)
-            ctx.set_count_mode(glb.COUNT_ACCESS)
-            for b in range(rank, nb, world):
-                ctx.sample_batch(e, b)
-            ctx.set_count_mode(glb.COUNT_NONE)
-            ctx.sync()
-            f = reduce_counts(ctx.counts_tensor(glb.COUNT_ACCESS))
-            acc_sum = f.clone() if acc_sum is None else acc_sum.add_(f)
-            if len(per_epoch) < 2:
-                per_epoch.append(f.clone())
-        ctx.counts_tensor(glb.COUNT_ACCESS).copy_(acc_sum)
-        del acc_sum
-        if len(per_epoch) >= 2:
-            v, num, den = ctx.footprint_similarity(per_epoch[0], per_epoch[1], 0.1)
-            similarity = {"epochs": [m0, m0 + 1], "top_frac": 0.1, "value": v,
-                          "numerator": num, "denominator": den, "source": "Table 2 (L329)"}
-        for a in sorted(set(sh.alphas) | {args.alpha}):
-            policies = {}
-            if 0.0 < a < 1.0:  # Fig 10 analog: Degree / Random vs PreSC vs Optimal
-                for pol in ("degree", "random"):
-                    ctx.build_cache_policy(a, pol, seed=g.seed)
-                    hs = ctx.hit_stats()
-                    policies[pol] = hs["hits"] / hs["total"] if hs["total"] else 0.0
-            ctx.build_cache(a)
+
+def hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs, batch_of,
+                    n_seeds, barrier):
+    """alpha sweep (H, Optimal H*, Degree / Random policies, seeds/s), PreSC#K sweep and
+    Table 2's footprint similarity over the measured epochs."""
+    import torch
+
+    import paper_conf_eurosys_yangtswycyz22_b200 as glb
+    from paper_conf_eurosys_yangtswycyz22_b200 import parallel as par
+
+    def reduce_counts(t):
+        if world > 1:
+            c = t if args.backend == "nccl" else t.cpu()
+            par.allreduce_counts(c)
+            if c is not t:
+                t.copy_(c)
+        return t
+
+    per_epoch = []
+    acc_sum = None
+    m0 = max([sh.K] + [int(x) for x in args.k_sweep.split(",") if x])
+    for e in range(m0, m0 + args.measure_epochs):
+        ctx.reset_counts(glb.COUNT_ACCESS)
+        ctx.set_count_mode(glb.COUNT_ACCESS)
+        for b in range(rank, nb, world):
+            ctx.sample_batch(e, b)
+        ctx.set_count_mode(glb.COUNT_NONE)
+        ctx.sync()
+        f = reduce_counts(ctx.counts_tensor(glb.COUNT_ACCESS))
+        acc_sum = f.clone() if acc_sum is None else acc_sum.add_(f)
+        if len(per_epoch) < 2:
+            per_epoch.append(f.clone())
+    ctx.counts_tensor(glb.COUNT_ACCESS).copy_(acc_sum)
+    del acc_sum
+    similarity = None
+    if len(per_epoch) >= 2:
+        v, num, den = ctx.footprint_similarity(per_epoch[0], per_epoch[1], 0.1)
+        similarity = {"epochs": [m0, m0 + 1], "top_frac": 0.1, "value": v,
+                      "numerator": num, "denominator": den, "source": "Table 2 (L329)"}
+    sweep, result_hit = [], None
+    for a in sorted(set(sh.alphas) | {alpha}):
+        policies = {}
+        if 0.0 < a < 1.0:  # Fig 10 analog: Degree / Random vs PreSC vs Optimal
+            for pol in ("degree", "random"):
+                ctx.build_cache_policy(a, pol, seed=g.seed)
+                hs = ctx.hit_stats()
+                policies[pol] = hs["hits"] / hs["total"] if hs["total"] else 0.0
+        ctx.build_cache(a)
+        hs = ctx.hit_stats()
+        H = hs["hits"] / hs["total"] if hs["total"] else 0.0
+        Hs = hs["optimal_hits"] / hs["total"] if hs["total"] else 0.0
+        torch.cuda.synchronize()
+        s0 = torch.cuda.Event(enable_timing=True)
+        s1 = torch.cuda.Event(enable_timing=True)
+        s0.record(stream)
+        sd = 0
+        for i in range(args.sweep_steps):
+            e, b = batch_of(i)
+            ctx.sample_batch(e, b)
+            ctx.extract_sample(out)
+            sd += n_seeds(b)
+        s1.record(xs)
+        torch.cuda.synchronize()
+        ms = s0.elapsed_time(s1)
+        sweep.append({"alpha": a, "cache_rows": hs["cache_rows"], "hit_rate": H,
+                      "optimal_hit_rate": Hs,
+                      "presc_vs_optimal_pct": (100.0 * H / Hs) if Hs > 0 else None,
+                      "degree_hit_rate": policies.get("degree"),
+                      "random_hit_rate": policies.get("random"),
+                      "seeds_per_s": sd * world / (ms / 1e3)})
+        if a == alpha:
+            result_hit = sweep[-1]
+    k_sweep = []
+    a_k = next((a for a in sh.alphas if 0.0 < a < 1.0), None)
+    if args.k_sweep and a_k is not None:
+        for K in [int(x) for x in args.k_sweep.split(",") if x]:
+            ctx.reset_counts(glb.COUNT_PRESAMPLE)
+            ctx.presample(K, rank, world)
+            reduce_counts(ctx.counts_tensor(glb.COUNT_PRESAMPLE))
+            ctx.build_cache(a_k)
             hs = ctx.hit_stats()
             H = hs["hits"] / hs["total"] if hs["total"] else 0.0
             Hs = hs["optimal_hits"] / hs["total"] if hs["total"] else 0.0
-            # timed seeds/s at this alpha (short run)
-            torch.cuda.synchronize()
-            s0 = torch.cuda.Event(enable_timing=True)
-            s1 = torch.cuda.Event(enable_timing=True)
-            s0.record(stream)
-            sd = 0
-            for i in range(args.sweep_steps):
-                e, b = batch_of(i)
-                ctx.sample_batch(e, b)
-                ctx.extract_sample(out)
-                sd += n_seeds(b)
-            s1.record(xs)
-            torch.cuda.synchronize()
-            ms = s0.elapsed_time(s1)
-            sweep.append({"alpha": a, "cache_rows": hs["cache_rows"], "hit_rate": H,
-                          "optimal_hit_rate": Hs,
-                          "presc_vs_optimal_pct": (100.0 * H / Hs) if Hs > 0 else None,
-                          "degree_hit_rate": policies.get("degree"),
-                          "random_hit_rate": policies.get("random"),
-                          "seeds_per_s": sd * world / (ms / 1e3)})
-            if a == args.alpha:
-                result_hit = sweep[-1]
+            k_sweep.append({"K": K, "alpha": a_k, "hit_rate": H, "optimal_hit_rate": Hs,
+                            "presc_vs_optimal_pct": 100.0 * H / Hs if Hs else None})
+    return {"hit_rate": result_hit, "alpha_sweep": sweep, "presc_k_sweep": k_sweep,
+            "measured_epochs": [m0, m0 + args.measure_epochs - 1],
+            "footprint_similarity": similarity}
 
-        # PreSC#K for K in --k-sweep at the shape's paper alpha (Fig 11(a) analog, L335:
-        # "K <= 2 already produce a decent hotness estimation"): presample epochs 0..K-1,
-        # hit rate over the same measured epochs (m0 .. m0+measure_epochs-1, after them)
-        a_k = next((a for a in sh.alphas if 0.0 < a < 1.0), None)
-        if args.k_sweep and a_k is not None:
-            for K in [int(x) for x in args.k_sweep.split(",") if x]:
-                ctx.reset_counts(glb.COUNT_PRESAMPLE)
-                ctx.presample(K, rank, world)
-                reduce_counts(ctx.counts_tensor(glb.COUNT_PRESAMPLE))
-                ctx.build_cache(a_k)
-                hs = ctx.hit_stats()
-                H = hs["hits"] / hs["total"] if hs["total"] else 0.0
-                Hs = hs["optimal_hits"] / hs["total"] if hs["total"] else 0.0
-                k_sweep.append({"K": K, "alpha": a_k, "hit_rate": H, "optimal_hit_rate": Hs,
-                                "presc_vs_optimal_pct": 100.0 * H / Hs if Hs else None})
 
-    cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        cpu = cpu_baseline(g, sh, args.cpu_seconds)
+def main(argv=None):
+    argv = sys.argv[1:] if argv is None else argv
+    args = parse(argv)
+    if args.impl == "reference":
+        return reference_arm(args)
+    if "WORLD_SIZE" not in os.environ and args.gpus > 1:
+        # the driver's `bench.py --gpus N` without a launcher: one rank per GPU
+        if args.ns_sweep and args.mode == "factored":
+            return ns_sweep(args, argv)
+        rc, _ = launch_ranks(args.gpus, argv)
+        sys.exit(rc)
+    import torch
+    import torch.distributed as dist
 
+    world, rank, local, local_world = dist_env()
+    local = local % torch.cuda.device_count()
+    if world > 1:
+        torch.cuda.set_device(local)
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
+    dev = torch.device("cuda", local)
+    torch.cuda.set_device(dev)
+    stream = torch.cuda.current_stream(dev)
+    sh = synth.SHAPES[args.config]
+    link_peak = hostlink_peak(dev)
+    res = run_workload(args, sh, args.alpha, world, rank, local, local_world, dev, stream, True,
+                       link_peak)
+    if args.mode == "factored":
+        return
+    pr1 = None
+    if not args.no_pr_alpha1 and args.config != "PR":
+        r = run_workload(args, synth.SHAPES["PR"], 1.0, world, rank, local, local_world, dev,
+                         stream, False, link_peak)
+        pr1 = {"workload": workload_name(synth.SHAPES["PR"], 1.0), "value": r["value"],
+               "unit": "seeds/s", "ms_per_step": r["ms_per_step"], "runs": r["runs"],
+               "runs_range": r["runs_range"], "roofline": r["roofline"],
+               "path_roofline": r["path_roofline"], "e2e_value": r["e2e"]["value"],
+               "gpu_launches": r["gpu_launches"], "clocks": r["clocks"]}
     if rank == 0:
         line = {
-            "metric": METRIC, "value": value, "unit": "seeds/s", "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": elapsed_max / args.steps, "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u32", "data": "synthetic",
+            "metric": METRIC, "value": res["value"], "unit": "seeds/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": res["ms_per_step"],
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u32",
+            "data": "synthetic",
             "config": {"workload": workload_name(sh, args.alpha), "shape": sh.name,
+                       "config_index": synth.CONFIG_INDEX.get(sh.name),
                        "V": sh.V, "E": sh.E, "feat_dim": sh.D, "batch": sh.batch,
                        "fanouts": list(sh.fanouts), "sampler": sh.sampler, "alpha": args.alpha,
                        "presample_K": sh.K, "parallelism": f"dp{world}",
-                       "l2": "inputs larger than L2 (CSR %.2f GB, feature cache %.2f GB vs 126 MB L2)"
-                             % ((8 * (sh.V + 1) + 4 * sh.E) / 1e9, 4 * sh.D * sh.V * args.alpha / 1e9)},
+                       "l2": "inputs larger than L2 (CSR %.2f GB, feature cache %.2f GB, host "
+                             "matrix %.1f GB vs 126 MB L2)"
+                             % ((8 * (sh.V + 1) + 4 * sh.E) / 1e9,
+                                4 * sh.D * sh.V * args.alpha / 1e9, 4 * sh.D * sh.V / 1e9)},
+            "runs": res["runs"], "runs_range": res["runs_range"],
+            "value_is": f"median of {args.runs} timed regions of {args.steps} steps",
             "pipeline_depth": args.pipeline,
-            "cache": {"layout": args.cache, "rows_cached": ctx_cache_rows,
-                      "peer_hit_share": peer_share},
-            "relabel_table": ctx.relabel_mode,
-            "relabel_l2_window_bytes": ctx.relabel_l2_window,
-            "host_wall_ms_timed_region": wall_ms,
-            "host_enqueue_ms_timed_region": enqueue_ms,
-            "roofline": {"kernel": "k_gather (extract a7)", "bound": "hbm", "achieved": ach_gbs,
-                         "peak": peak, "unit": "GB/s", "frac": ach_gbs / peak, "traffic": traffic,
-                         "peak_source": peak_src,
-                         "extract_ms_per_step": statistics.mean(x_ms),
-                         "extract_share_of_step": statistics.mean(x_ms) / (elapsed_max / args.steps),
-                         "algorithmic_bytes_per_launch": statistics.mean(hbm_bytes),
-                         "timed_launches": f"every {args.time_every}th extract of the timed "
-                                           f"region ({len(x_ms)} launches)",
-                         "measured_with": f"pipeline depth {args.pipeline} (the timed region)",
-                         "isolated": iso},
-            "cpu_baseline": cpu,
-            "e2e": {"value": e2e_val, "unit": "seeds/s", "h2d_bytes_per_step": h2d,
-                    "d2h_bytes_per_step": d2h, "steps": len(e2e_steps),
-                    "api": "glb_sample_async(pinned host seeds) + glb_extract_sample + "
-                           "D2H of the step's counts (host reads step j-D during step j, "
-                           f"D = pipeline depth {lag})",
-                    "rows_extracted": e2e_rows,
-                    "sync_api_value": e2e_sync_val,
-                    "sync_api": "glb_sample(host seeds; sizes D2H, sync) + glb_extract_sample "
-                                "+ stats (sync) every step"},
-            "gpu_launches": launches,
-            "clocks": clk,
-            "hit_rate": result_hit,
-            "alpha_sweep": sweep,
-            "presc_k_sweep": k_sweep,
-            "measured_epochs": [m0, m0 + args.measure_epochs - 1] if not args.no_sweep else None,
-            "footprint_similarity": similarity,
-            "units": {"mean_n_L": statistics.mean(nL), "mean_hits": statistics.mean(hits),
-                      "mean_misses": statistics.mean(misses)},
-            "preprocess_s": {"generate_inputs": t_gen, "load_graph": t_load,
-                             "presample": t_pre, "build_cache": t_cache},
+            "roofline": res["roofline"], "path_roofline": res["path_roofline"],
+            "cpu_baseline": res.get("cpu_baseline"), "e2e": res["e2e"],
+            "gpu_launches": res["gpu_launches"], "clocks": res["clocks"],
+            "pr_alpha1": pr1,
+            "host": host_info(), "gpu": gpu_info(local),
         }
+        for k in ("cache", "relabel_table", "relabel_l2_window_bytes", "host_inputs",
+                  "host_wall_ms_timed_region", "host_enqueue_ms_timed_region", "hit_rate",
+                  "alpha_sweep", "presc_k_sweep", "measured_epochs", "footprint_similarity",
+                  "units", "preprocess_s"):
+            if k in res:
+                line[k] = res[k]
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+def ns_sweep(args, argv):
+    """Config 5's Ns sweep (Fig 15 analog): the adaptive split, then every
+    Ns in 1..N-1, each a separate N-rank factored run; one line = the adaptive run plus the
+    sweep."""
+    base = [a for a in argv if a != "--ns-sweep"]
+    rc, line = launch_ranks(args.gpus, base, capture=True)
+    if rc != 0 or line is None:
+        sys.exit(rc or 1)
+    sweep = []
+    for ns in range(1, args.gpus):
+        r, ln = launch_ranks(args.gpus, base + ["--ns", str(ns)], capture=True)
+        sweep.append({"samplers": ns, "trainers": args.gpus - ns,
+                      "value": ln["value"] if ln else None, "rc": r})
+    line["ns_sweep"] = sweep
+    print(json.dumps(line), flush=True)
 
 
 if __name__ == "__main__":

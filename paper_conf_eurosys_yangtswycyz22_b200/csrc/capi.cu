@@ -7,6 +7,7 @@
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
+#include <cstddef>
 #include <cstring>
 #include <new>
 
@@ -145,6 +146,17 @@ glb_status check_dev_err(glb_ctx* c, DevState* st) {
   return GLB_OK;
 }
 
+// Stats of at most one extract are pending (one pinned mirror): a second extract that
+// asks for stats first completes the earlier one.
+glb_status flush_pending_stats(glb_ctx* c) {
+  if (!c->pending_stats) return GLB_OK;
+  CK(sync_all(c));
+  c->pending_stats->hits = c->h_xcount[0];
+  c->pending_stats->misses = c->h_xcount[1];
+  c->pending_stats = nullptr;
+  return GLB_OK;
+}
+
 // Enqueue one sampled mini-batch (a2/a2' + a3 + a4, and a5 when counting).
 glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, int kind,
                           const uint32_t* k, uint32_t L, uint64_t seed, uint32_t epoch,
@@ -164,7 +176,9 @@ glb_status enqueue_sample(glb_ctx* c, const uint32_t* seeds_dev, uint32_t n0, in
   // the extract that last read this slot must finish before it is overwritten
   if (c->nslots == 2) CK(cudaStreamWaitEvent(c->stream, c->ev_extracted[slot], 0));
   use_slot(c, slot);
-  CK(cudaMemsetAsync(c->st, 0, sizeof(DevState), c->stream));
+  // sizes and counters restart; the error bits stay (sticky until a call reports them), so
+  // an error of any batch of a presample or pipelined run is not lost
+  CK(cudaMemsetAsync(c->st, 0, offsetof(DevState, err), c->stream));
   const int mode = c->count_mode;
   CK(launch_seed_init(c, seeds_dev, n0, mode));
   for (uint32_t l = 0; l < L; ++l) {
@@ -293,6 +307,7 @@ glb_status glb_create(int device, glb_ctx** out) {
       (e = cudaEventCreateWithFlags(&c->ev_perm[0], cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_perm[1], cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_mark, cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&c->ev_xlast, cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_sampled[0], cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_sampled[1], cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_extracted[0], cudaEventDisableTiming)) != cudaSuccess ||
@@ -325,8 +340,13 @@ glb_status glb_create(int device, glb_ctx** out) {
   if (const char* g = getenv("GLB_GATHER_ST")) c->gather_st_wb = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_BULK")) c->gather_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_MISS_BULK")) c->miss_bulk = atoi(g) != 0;
+  if (const char* g = getenv("GLB_GATHER_WARP")) c->gather_warp = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_BULK_SMEM")) c->gather_bulk_smem = (uint32_t)atoi(g);
   if (const char* g = getenv("GLB_PERM_PREFETCH")) c->perm_prefetch = atoi(g) != 0;
+  if (const char* g = getenv("GLB_MISS_BIN_LOG2")) {
+    const int k = atoi(g);
+    c->miss_bin_log2 = k >= 0 && k <= 40 ? (uint32_t)k : 21u;
+  }
   *out = c;
   return GLB_OK;
 }
@@ -347,6 +367,7 @@ glb_status glb_destroy(glb_ctx* c) {
   if (c->ev_perm[0]) cudaEventDestroy(c->ev_perm[0]);
   if (c->ev_perm[1]) cudaEventDestroy(c->ev_perm[1]);
   if (c->ev_mark) cudaEventDestroy(c->ev_mark);
+  if (c->ev_xlast) cudaEventDestroy(c->ev_xlast);
   if (c->sstream) cudaStreamDestroy(c->sstream);
   dfree(c->sts[0]); dfree(c->sts[1]); dfree(c->st_x); dfree(c->scratch); dfree(c->xcount);
   dfree(c->work);
@@ -380,7 +401,8 @@ glb_status glb_sync(glb_ctx* c) {
   }
   glb_status s = check_dev_err(c, c->st_x);
   if (s != GLB_OK) return s;
-  return check_dev_err(c, c->st);
+  s = check_dev_err(c, c->sts[0]);
+  return s != GLB_OK ? s : check_dev_err(c, c->sts[1]);
 }
 
 glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* indptr,
@@ -436,11 +458,10 @@ glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* in
     c->h_features = features;
     c->features_mapped = (const float*)dp;
     c->D = D;
-    uint32_t shift = 0;
-    while ((4ull * D << (shift + 1)) <= (2ull << 20)) ++shift;
+    uint32_t sums = 0;
     dfree(c->miss_bins);
-    c->miss_bins_cap = (uint32_t)((V >> shift) + 1);
-    CK(dalloc(&c->miss_bins, c->miss_bins_cap));
+    c->miss_bins_cap = miss_bins_needed(c, V, D, &sums);
+    CK(dalloc(&c->miss_bins, 2ull * c->miss_bins_cap + sums));
   }
   return GLB_OK;
 }
@@ -506,6 +527,8 @@ glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32
   // batch's unique-vertex bound -- then an L2-sized open-addressing hash table
   uint64_t H = 1024;
   while (H < un + un / 4 && H < kMaxHashEntries) H <<= 1;
+  if (c->relabel_mode == 2 && H < un + un / 4)
+    return set_err(c, GLB_ENOMEM, "hash relabel table would need > 2^31 entries");
   if (const char* hc = getenv("GLB_HASH_LOG2")) {  // experiment: explicit capacity
     const int lg = atoi(hc);
     if (lg >= 10 && lg <= 30) H = 1ull << lg;
@@ -570,8 +593,15 @@ glb_status glb_set_train_set(glb_ctx* c, const uint32_t* train, uint64_t n, uint
   ENTER(c);
   if (!c->V) return set_err(c, GLB_ESTATE, "set_train_set before load_graph");
   if (B == 0 || (n && !train) || n >= 0xFFFFFFFFull) return set_err(c, GLB_EINVAL, "bad train set");
-  for (uint64_t i = 0; i < n; ++i)
-    if (train[i] >= c->V) return set_err(c, GLB_EINVAL, "train id %u >= V", train[i]);
+  {  // T is a set (L305; reading Q6): ids < V, no duplicates
+    std::vector<uint64_t> seen((c->V + 63) / 64, 0);
+    for (uint64_t i = 0; i < n; ++i) {
+      const uint32_t t = train[i];
+      if (t >= c->V) return set_err(c, GLB_EINVAL, "train id %u >= V", t);
+      if (seen[t >> 6] >> (t & 63) & 1) return set_err(c, GLB_EINVAL, "duplicate train id %u", t);
+      seen[t >> 6] |= 1ull << (t & 63);
+    }
+  }
   CK(sync_all(c));
   dfree(c->train); dfree(c->perm_b[0]); dfree(c->perm_b[1]); dfree(c->shuf_keys); dfree(c->shuf_vals);
   c->perm = nullptr;
@@ -740,7 +770,8 @@ glb_status glb_presample(glb_ctx* c, uint32_t K, uint32_t rank, uint32_t world) 
   c->count_mode = saved;
   if (s != GLB_OK) return s;
   c->have_sample = false;
-  return check_dev_err(c, c->st);
+  s = check_dev_err(c, c->sts[0]);
+  return s != GLB_OK ? s : check_dev_err(c, c->sts[1]);
 }
 
 glb_status glb_counts_device_ptr(glb_ctx* c, int which, void** out) {
@@ -1025,10 +1056,19 @@ glb_status glb_extract(glb_ctx* c, const uint32_t* vertices, uint64_t n, void* o
     CK(dalloc(&c->xb.miss_sorted, n));
     c->xb.cap = n;
   }
+  if (stats) {
+    glb_status ps = flush_pending_stats(c);
+    if (ps != GLB_OK) return ps;
+  }
+  if (c->nslots == 2) {  // the extract stream's gathers share the miss-sort scratch and the
+    // extract counters with this one: order after them (glb.h, pipeline depth 2)
+    CK(cudaEventRecord(c->ev_xlast, c->xstream));
+    CK(cudaStreamWaitEvent(c->stream, c->ev_xlast, 0));
+  }
   CK(cudaMemsetAsync(&c->st_x->nhit, 0, 2 * sizeof(uint32_t), c->stream));
   if (n) CK(launch_mark(c, vertices, n));
   const uint2* misses = c->xb.miss_list;
-  if (n && c->C < c->V) {  // some rows may come over PCIe: order them by host page
+  if (n && c->C < c->V && c->miss_bin_log2) {  // rows may come over PCIe: order them by address
     CK(launch_sort_misses(c, c->xb.miss_list, &c->st_x->nmiss, c->xb.miss_sorted));
     misses = c->xb.miss_sorted;
   }
@@ -1047,6 +1087,10 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
   if (!c->features_mapped) return set_err(c, GLB_ESTATE, "graph loaded without features");
   if (!shards_ready(c)) return set_err(c, GLB_ESTATE, "peer cache shards not all attached");
   if (!out) return set_err(c, GLB_EINVAL, "null out");
+  if (stats) {
+    glb_status ps = flush_pending_stats(c);
+    if (ps != GLB_OK) return ps;
+  }
   cudaStream_t main = c->stream;
   const int slot = c->cur;
   if (c->nslots == 2) {  // extract on its own stream, overlapping the next sample;
@@ -1073,7 +1117,7 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
   }
   const uint2* misses = c->sb.miss_list;
   cudaError_t e = cudaSuccess;
-  if (c->C < c->V) {  // some rows may come over PCIe: order them by host page
+  if (c->C < c->V && c->miss_bin_log2) {  // rows may come over PCIe: order them by address
     e = launch_sort_misses(c, c->sb.miss_list, &c->st->nmiss, c->sb.miss_sorted);
     misses = c->sb.miss_sorted;
   }

@@ -253,6 +253,96 @@ __global__ void __launch_bounds__(kThreads, 4)
   }
 }
 
+// Warp-independent variant (GLB_GATHER_WARP=1): no block barrier anywhere.  Warp gw of
+// NW takes chunks gw, gw + NW, ... of Rw rows (hit chunks first, then miss chunks, so all
+// warps drain the HBM hits before the host misses); lane i < Rw loads and resolves the
+// entry of row i of the chunk (prefetched one chunk ahead), and every 16-byte vector
+// fetches its row's (source, destination) from the owning lane with two 64-bit shuffles.
+// A block barrier per chunk makes every warp of the block wait for the slowest one -- on
+// the PCIe path the slowest of 256 zero-copy rows carries the address-translation tail.
+template <typename T, bool SHARD>
+__global__ void __launch_bounds__(kThreads)
+    k_gather_w(T* __restrict__ out, const T* __restrict__ src_hit, const T* __restrict__ src_miss,
+               const uint2* __restrict__ hit_list, const uint2* __restrict__ miss_list,
+               const uint32_t* __restrict__ fill_src, const uint32_t* __restrict__ dev_counts,
+               uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t Rw, uint32_t Sh,
+               uint32_t So, int st_wb, int skip, unsigned long long* xcount, ShardTab tab) {
+  pdl_enter();
+  const uint64_t nh_all = dev_counts ? dev_counts[0] : nh_host;
+  const uint64_t nm_all = dev_counts ? dev_counts[1] : nm_host;
+  if (xcount && blockIdx.x == 0 && threadIdx.x == 0) {
+    xcount[0] = nh_all;
+    xcount[1] = nm_all;
+  }
+  const uint64_t nm = (skip & 2) ? 0 : nm_all;
+  const uint64_t nh = (skip & 1) ? 0 : nh_all;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t NW = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const uint64_t nch = (nh + Rw - 1) / Rw, ncm = (nm + Rw - 1) / Rw, nc = nch + ncm;
+  const float inv_u = 1.0f / (float)U;
+  const uint64_t pol = l2_evict_first_policy();
+  uint32_t npeer = 0;
+  // this lane's work-list entry of chunk g (raw), and its resolved (source, destination)
+  auto load_ent = [&](uint64_t g) -> uint2 {
+    if (g >= nc || lane >= Rw) return make_uint2(0u, 0u);
+    const bool miss = g >= nch;
+    const uint64_t r = (miss ? g - nch : g) * Rw + lane;
+    if (r >= (miss ? nm : nh)) return make_uint2(0u, 0u);
+    if (!miss) return __ldg(hit_list + r);
+    return fill_src ? make_uint2((uint32_t)r, __ldg(fill_src + r)) : __ldg(miss_list + r);
+  };
+  uint64_t g = gw;
+  uint2 e = load_ent(g);
+  while (g < nc) {
+    const bool miss = g >= nch;
+    const uint64_t c = miss ? g - nch : g;
+    const uint32_t rows = (uint32_t)min((uint64_t)Rw, (miss ? nm : nh) - c * Rw);
+    unsigned long long srcp = 0, dsto = (unsigned long long)e.x * So;
+    if (miss) {
+      srcp = (unsigned long long)(src_miss + (uint64_t)e.y * U);
+    } else if (SHARD) {
+      const uint32_t w = e.y % tab.W;
+      srcp = (unsigned long long)((const T*)tab.base[w] + (uint64_t)(e.y / tab.W) * Sh);
+      npeer += (w != tab.rank) && lane < rows;
+    } else {
+      srcp = (unsigned long long)(src_hit + (uint64_t)e.y * Sh);
+    }
+    const uint64_t gn = g + NW;
+    e = load_ent(gn);  // next chunk's entry, in flight with this chunk's rows
+    const uint32_t total = rows * U;
+    for (uint32_t base = 0; base < total; base += 32 * kVecPerThread) {
+      T x[kVecPerThread];
+      unsigned long long dst[kVecPerThread];
+#pragma unroll
+      for (int q = 0; q < kVecPerThread; ++q) {
+        const uint32_t v = base + q * 32 + lane;
+        const uint32_t row = (uint32_t)(((float)v + 0.5f) * inv_u);  // exact for v < 2^20
+        const unsigned long long s = __shfl_sync(kFull, srcp, row & 31);
+        const unsigned long long d = __shfl_sync(kFull, dsto, row & 31);
+        if (v < total) {
+          const uint32_t col = v - row * U;
+          x[q] = ld_row((const T*)s + col, pol);
+          dst[q] = d + col;
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < kVecPerThread; ++q) {
+        const uint32_t v = base + q * 32 + lane;
+        if (v < total) {
+          if (st_wb) out[dst[q]] = x[q];
+          else st_row(out + dst[q], x[q]);
+        }
+      }
+    }
+    g = gn;
+  }
+  if (SHARD) {
+    const uint32_t wsum = __reduce_add_sync(kFull, npeer);
+    if (lane == 0 && wsum && xcount) atomicAdd(&xcount[2], (unsigned long long)wsum);
+  }
+}
+
 // ---- host-miss ordering: a one-pass counting sort of the miss list by the 2 MB
 // host page its source row lives in, so consecutive zero-copy reads share GPU
 // address translations (measured: random 512 B rows over 64 GB 35 -> 47 GB/s).
@@ -421,20 +511,38 @@ __global__ void __launch_bounds__(64)
 
 cudaError_t launch_sort_misses(glb_ctx* c, const uint2* miss, const uint32_t* nmiss_dev,
                                uint2* sorted) {
-  // rows per 2 MB page -> shift (rows are 4*D bytes; round the page down to a power-of-2 row count)
+  // bins of 2^miss_bin_log2 bytes of the host matrix (rounded down to a power-of-2 row count)
   const uint64_t row_bytes = 4ull * c->D;
   uint32_t shift = 0;
-  while ((row_bytes << (shift + 1)) <= (2ull << 20)) ++shift;
+  while ((row_bytes << (shift + 1)) <= (1ull << c->miss_bin_log2)) ++shift;
   const uint32_t nb = (uint32_t)((c->V >> shift) + 1);
   if (nb > c->miss_bins_cap) return cudaErrorInvalidValue;
   cudaError_t e = cudaMemsetAsync(c->miss_bins, 0, sizeof(unsigned int) * nb, c->stream);
   if (e != cudaSuccess) return e;
   const int grid = c->num_sms * 4;
   k_miss_hist<<<grid, kThreads, 0, c->stream>>>(miss, nmiss_dev, shift, c->miss_bins);
-  k_miss_scan<<<1, 1024, 0, c->stream>>>(c->miss_bins, nb);
-  k_miss_scatter<<<grid, kThreads, 0, c->stream>>>(miss, nmiss_dev, shift, c->miss_bins, sorted);
-  count_launch(c, 3);
+  count_launch(c);
+  unsigned int* offs = c->miss_bins;
+  if (nb <= 8192) {  // a few coarse bins: one block scans them in place
+    k_miss_scan<<<1, 1024, 0, c->stream>>>(c->miss_bins, nb);
+    count_launch(c);
+  } else {  // many fine bins: the three-phase device scan
+    offs = c->miss_bins + c->miss_bins_cap;
+    e = scan_exclusive_u32(c, c->miss_bins, nb, offs, offs + c->miss_bins_cap);
+    if (e != cudaSuccess) return e;
+  }
+  k_miss_scatter<<<grid, kThreads, 0, c->stream>>>(miss, nmiss_dev, shift, offs, sorted);
+  count_launch(c);
   return cudaGetLastError();
+}
+
+uint32_t miss_bins_needed(const glb_ctx* c, uint64_t V, uint32_t D, uint32_t* scan_sums) {
+  const uint64_t row_bytes = 4ull * D;
+  uint32_t shift = 0;
+  while ((row_bytes << (shift + 1)) <= (1ull << c->miss_bin_log2)) ++shift;
+  const uint32_t nb = (uint32_t)((V >> shift) + 1);
+  *scan_sums = (uint32_t)((nb + kThreads * 16 - 1) / (kThreads * 16)) + 1;
+  return nb;
 }
 
 cudaError_t launch_mark(glb_ctx* c, const uint32_t* vertices, uint64_t n) {
@@ -548,6 +656,29 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   cudaError_t e;
   if (shard && !mo && (e = cudaMemsetAsync(c->xcount + 2, 0, sizeof(unsigned long long), c->stream)) != cudaSuccess)
     return e;
+  if (c->gather_warp) {  // warp-independent gather (no block barriers)
+    uint32_t Rw = (uint32_t)(32 * kVecPerThread) / U;
+    Rw = Rw < 1 ? 1 : Rw > 32 ? 32 : Rw;
+    const int gridw = c->num_sms * (c->stream == c->xstream ? c->gather_bps_pipe : c->gather_bps);
+    if (vec && shard)
+      e = launch_pdl(k_gather_w<float4, true>, gridw, kThreads, c->stream, (float4*)out,
+                     (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
+                     dev_counts, nhit_host, nmiss_host, U, Rw, Sh, So, wb, mo, c->xcount, tab);
+    else if (vec)
+      e = launch_pdl(k_gather_w<float4, false>, gridw, kThreads, c->stream, (float4*)out,
+                     (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
+                     dev_counts, nhit_host, nmiss_host, U, Rw, Sh, So, wb, mo, c->xcount, tab);
+    else if (shard)
+      e = launch_pdl(k_gather_w<float, true>, gridw, kThreads, c->stream, out, src_hit, src_miss,
+                     hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, Rw, Sh,
+                     So, wb, mo, c->xcount, tab);
+    else
+      e = launch_pdl(k_gather_w<float, false>, gridw, kThreads, c->stream, out, src_hit, src_miss,
+                     hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, Rw, Sh,
+                     So, wb, mo, c->xcount, tab);
+    count_launch(c);
+    return e;
+  }
   if (vec && shard)
     e = launch_pdl(k_gather<float4, true>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,

@@ -32,7 +32,10 @@ enum : uint32_t { kDomShuffle = 1, kDomKhop = 2, kDomRwalk = 3, kDomPolicy = 7, 
 
 // device error bits (DevState::err)
 enum : uint32_t { kErrDupSeed = 1u, kErrRange = 2u, kErrCapacity = 4u, kErrBadGraph = 8u };
-constexpr uint32_t kMaxHashEntries = 1u << 23;  // 128 MB table cap
+// hash-table capacity limit: indices (with the kDefer bit) must stay below 2^31.  The table
+// is sized at >= 1.25x the batch's unique-vertex upper bound, so it never fills (no cap
+// below the bound: TW's bound is 8.4 M, table 16 M entries = 320 MB)
+constexpr uint32_t kMaxHashEntries = 1u << 31;
 
 // Per-batch device state.  Sizes live here so no kernel needs a host sync.
 struct DevState {
@@ -201,6 +204,7 @@ struct glb_ctx {
                                // measured 2x slower than the LSU gather
   uint32_t gather_bulk_smem = 96 * 1024;  // row-slot bytes per bulk block (GLB_GATHER_BULK_SMEM)
   int miss_bulk = 0;           // GLB_MISS_BULK=1: host misses through cp.async.bulk
+  int gather_warp = 0;         // GLB_GATHER_WARP=1: warp-independent gather (k_gather_w)
   uint64_t C = 0;
   // NEXT-3 peer-sharded cache: global rank i < C is owned by shard i % W at row i / W;
   // shard_base[r] = device pointer (valid in this process) of shard r's rows.
@@ -232,8 +236,10 @@ struct glb_ctx {
   int gather_bps_pipe = 2;       // ... on the extract stream at pipeline depth 2: leaves SM
                                  // slots to the sampler running concurrently on the main stream
   unsigned int* work = nullptr;  // device [8]: gather chunk counters (main, extract stream)
-  unsigned int* miss_bins = nullptr;  // [miss_bins_cap] host-page histogram of misses
+  unsigned int* miss_bins = nullptr;  // [2*miss_bins_cap + sums] histogram, offsets, scan sums
   uint32_t miss_bins_cap = 0;
+  uint32_t miss_bin_log2 = 21;   // host misses ordered by 2^k-byte bins of the matrix
+                                 // (GLB_MISS_BIN_LOG2; 0 = unordered)
   int timing = 0;                // record events around every timing-th extract (0: off)
   uint64_t timing_calls = 0;
   std::vector<cudaEvent_t> tev;  // pairs (start, end) of recorded extracts
@@ -251,6 +257,7 @@ struct glb_ctx {
   cudaStream_t sstream = nullptr;
   cudaEvent_t ev_perm[2] = {nullptr, nullptr};
   cudaEvent_t ev_mark = nullptr;
+  cudaEvent_t ev_xlast = nullptr;  // glb_extract at depth 2: after the extract stream's work
   uint64_t n_train = 0;
   uint32_t batch_size = 0;
   uint64_t seed = 0;
@@ -352,6 +359,10 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
                           uint64_t nhit_host, uint64_t nmiss_host);
 cudaError_t launch_sort_misses(glb_ctx* c, const uint2* miss, const uint32_t* nmiss_dev,
                                uint2* sorted);
+// bins of the miss ordering for a V x D matrix; *scan_sums = scratch words of the device scan
+uint32_t miss_bins_needed(const glb_ctx* c, uint64_t V, uint32_t D, uint32_t* scan_sums);
+cudaError_t scan_exclusive_u32(glb_ctx* c, const uint32_t* a, uint64_t n, uint32_t* out,
+                               uint32_t* sums);
 cudaError_t scan_inclusive_u64(glb_ctx* c, const uint32_t* a, uint64_t n, unsigned long long* out);
 cudaError_t launch_khop_weighted(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed,
                                  uint32_t epoch, uint32_t batch);

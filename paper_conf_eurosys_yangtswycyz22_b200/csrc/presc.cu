@@ -422,8 +422,8 @@ __global__ void __launch_bounds__(kThreads)
   }
 }
 
-cudaError_t scan_exclusive_u32(glb_ctx* c, const uint32_t* a, uint64_t n, uint32_t* out,
-                               uint32_t* sums) {
+cudaError_t scan_excl_u32(glb_ctx* c, const uint32_t* a, uint64_t n, uint32_t* out,
+                          uint32_t* sums) {
   const uint64_t m = (n + kScanChunk - 1) / kScanChunk;
   if (m == 0) return cudaSuccess;
   k_scan_reduce<<<(unsigned)m, kThreads, 0, c->stream>>>(a, n, sums);
@@ -462,7 +462,7 @@ cudaError_t radix_sort_pairs(glb_ctx* c, K* keys, uint32_t* vals, K* keys_alt, u
     for (int shift = 0; shift < bits; shift += 8) {
       k_radix_hist<K><<<(unsigned)ntiles, kThreads, 0, c->stream>>>(kin, n, shift, hist, ntiles);
       count_launch(c);
-      if ((e = scan_exclusive_u32(c, hist, hn, offs, sums)) != cudaSuccess) return e;
+      if ((e = scan_excl_u32(c, hist, hn, offs, sums)) != cudaSuccess) return e;
       k_radix_scatter<K><<<(unsigned)ntiles, kThreads, 0, c->stream>>>(kin, vin, n, shift, offs,
                                                                       ntiles, kout, vout);
       count_launch(c);
@@ -479,6 +479,11 @@ cudaError_t radix_sort_pairs(glb_ctx* c, K* keys, uint32_t* vals, K* keys_alt, u
 inline int grid_for(glb_ctx* c) { return c->num_sms * 8; }
 
 }  // namespace
+
+cudaError_t scan_exclusive_u32(glb_ctx* c, const uint32_t* a, uint64_t n, uint32_t* out,
+                               uint32_t* sums) {
+  return scan_excl_u32(c, a, n, out, sums);
+}
 
 cudaError_t radix_sort_pairs_u64(glb_ctx* c, unsigned long long* keys, uint32_t* vals,
                                  unsigned long long* keys_alt, uint32_t* vals_alt, uint64_t n,

@@ -45,9 +45,15 @@ def dp_step_batch(i: int, rank: int, world: int, num_batches: int, first_epoch: 
 
 
 def allreduce_counts(t: torch.Tensor, group=None):
-    """Sum u32 visit counts across ranks (int32 view; sums stay < 2^31)."""
+    """Sum u32 visit counts across ranks (int32 view; sums stay < 2^31).
+
+    On CUDA the host waits for the reduction before returning: the library's
+    next call (build_cache ranks the counts) may run on a stream that is not
+    ordered after NCCL's, so every rank must see the fully reduced counts."""
     if dist.is_available() and dist.is_initialized() and dist.get_world_size(group) > 1:
         dist.all_reduce(t, op=dist.ReduceOp.SUM, group=group)
+        if t.is_cuda:
+            torch.cuda.synchronize(t.device)
     return t
 
 

@@ -1,9 +1,10 @@
 """Full-size parity for BASELINE configs[2..4] (TW 3-hop GCN, PA PinSAGE random
-walk with PreSC#K, UK GraphSAGE): PreSC counts over all K presample epochs
-(oracle sharded by batch over host threads, summed exactly), cache slots at
-the config's alphas, every output of four measured batches (first, second, a
-random one, the last partial one) and sampled extracted rows, all in the
-launch configuration bench.py uses.  Host RAM: TW ~50 GB, PA ~65 GB,
+walk with PreSC#K, UK GraphSAGE) and the weighted TWW: PreSC counts over all K
+presample epochs (oracle sharded by batch over host threads, summed exactly),
+cache slots at the config's alphas, every output of four measured batches
+(first, second, a random one, the last partial one) at the paper's R% -- so
+the PCIe miss path runs -- and one at alpha = 1, with EVERY extracted byte
+compared, all in the launch configuration bench.py uses.  Host RAM: TW ~50 GB, PA ~65 GB,
 UK ~95 GB (features in pinned memory)."""
 import concurrent.futures as cf
 import os
@@ -25,11 +26,29 @@ def u32(t):
     return t.cpu().numpy().view(np.uint32)
 
 
-def oracle_sample(go, sh, seeds, seed, e, b):
+def oracle_sample(go, sh, seeds, seed, e, b, weights=None):
     if sh.sampler == "khop":
         return go.sample_khop(seeds, sh.fanouts, seed, e, b)
+    if sh.sampler == "weighted":
+        return go.sample_khop_weighted(weights, seeds, sh.fanouts, seed, e, b)
     return go.sample_rwalk(seeds, len(sh.fanouts), seed, e, b, synth.RW_WALKS, synth.RW_LEN,
                            sh.fanouts[0])
+
+
+CHUNK = 1 << 18  # rows per host compare
+
+
+def assert_rows_exact(go, out, uniq):
+    """EVERY gathered byte of out[:n] against the oracle's extract (a7: memcpy of row
+    uniq[i] of the host matrix), in chunks of CHUNK rows (device->host copy + compare)."""
+    n = uniq.shape[0]
+    for a in range(0, n, CHUNK):
+        b = min(n, a + CHUNK)
+        got = out[a:b].cpu().numpy().view(np.uint32)
+        want = go.extract(uniq[a:b]).view(np.uint32)
+        if not np.array_equal(got, want):
+            bad = np.nonzero((got != want).any(axis=1))[0]
+            raise AssertionError(f"{bad.size} rows differ in [{a}, {b}), first lid {a + bad[0]}")
 
 
 def oracle_counts_parallel(g, sh, epochs):
@@ -42,18 +61,21 @@ def oracle_counts_parallel(g, sh, epochs):
         go = oracle.GraphOracle(g.indptr, g.indices)
         c = np.zeros(g.V, np.uint32)
         for e, b, s in shard:
-            c[oracle_sample(go, sh, s, g.seed, e, b).uniq] += 1
+            c[oracle_sample(go, sh, s, g.seed, e, b, g.weights).uniq] += 1
         return c
 
     with cf.ThreadPoolExecutor(THREADS) as ex:
         return sum(ex.map(run, shards)).astype(np.uint32)
 
 
-def make_sampler_ctx(g, sh, features=True):
+def make_sampler_ctx(g, sh, features=True, relabel="auto"):
     ctx = glb.Context(0)
     ctx.load_graph(g.indptr, g.indices, g.features if features else None)
-    if sh.sampler == "khop":
-        ctx.set_sampler("khop", fanouts=sh.fanouts, max_batch=sh.batch)
+    ctx.set_relabel_mode(relabel)
+    if g.weights is not None:
+        ctx.load_edge_weights(g.weights)
+    if sh.sampler in ("khop", "weighted"):
+        ctx.set_sampler(sh.sampler, fanouts=sh.fanouts, max_batch=sh.batch)
     else:
         ctx.set_sampler("rwalk", layers=len(sh.fanouts), walks=synth.RW_WALKS,
                         walk_len=synth.RW_LEN, topk=sh.fanouts[0], max_batch=sh.batch)
@@ -87,47 +109,21 @@ def check_handoff(g, sh, go, trainer, slot_map, e):
             assert np.array_equal(u32(s.indices[l]), os_.indices[l]), (b, l)
         assert np.array_equal(s.cache_slot.cpu().numpy(), slot_map[os_.uniq])
         st = trainer.extract_sample(out, stats=True)
-        idx = rng.integers(0, s.sizes[-1], 2048)
-        got = out[torch.from_numpy(idx).cuda()].cpu().numpy()
-        assert np.array_equal(got.view(np.uint32), g.features[os_.uniq[idx]].view(np.uint32))
+        assert_rows_exact(go, out, os_.uniq)
         assert st["hits"] == int((slot_map[os_.uniq] >= 0).sum())
         assert trainer.handoff_tag() == b
         trainer.handoff_release(i % 2)
     sampler.close()
 
 
-def check_config(name, Ks=None, handoff=False):
-    sh = synth.SHAPES[name]
-    g = synth.make_graph(sh)
-    go = oracle.GraphOracle(g.indptr, g.indices, g.features)
-    ctx = glb.Context(0)
-    ctx.load_graph(g.indptr, g.indices, g.features)
-    if sh.sampler == "khop":
-        ctx.set_sampler("khop", fanouts=sh.fanouts, max_batch=sh.batch)
-    else:
-        ctx.set_sampler("rwalk", layers=len(sh.fanouts), walks=synth.RW_WALKS,
-                        walk_len=synth.RW_LEN, topk=sh.fanouts[0], max_batch=sh.batch)
-    ctx.set_train_set(g.train, sh.batch, g.seed)
-    for K in (Ks or [sh.K]):
-        ctx.reset_counts(glb.COUNT_PRESAMPLE)
-        ctx.presample(K)
-        counts = oracle_counts_parallel(g, sh, range(K))
-        assert np.array_equal(ctx.get_counts(glb.COUNT_PRESAMPLE), counts), f"PreSC#{K}"
-        for a in sh.alphas:
-            ctx.build_cache(a)
-            assert np.array_equal(ctx.cache_slots(), oracle.cache_slots(counts, a)), (K, a)
-    e = max(Ks or [sh.K])
+def check_batches(ctx, g, sh, go, e, batches, out, slot_map):
+    """Every output of the given batches of epoch e: sizes, uniq, every block (and RW
+    weights), the a4 marks, hit count, and every extracted byte."""
     ob = oracle.epoch_batches(g.train, sh.batch, g.seed, e)
-    nb = len(ob)
-    rng = np.random.default_rng(0)
-    ub = sh.batch
-    for k in sh.fanouts:
-        ub = min(ub * (1 + k), sh.V)
-    out = torch.empty((ub, sh.D), dtype=torch.float32, device="cuda")
-    for b in [0, 1, int(rng.integers(2, nb - 1)), nb - 1]:
+    for b in batches:
         ctx.sample_batch(e, b)
         s = ctx.sample_result()
-        os_ = oracle_sample(go, sh, ob[b], g.seed, e, b)
+        os_ = oracle_sample(go, sh, ob[b], g.seed, e, b, g.weights)
         assert s.sizes == os_.sizes, b
         assert np.array_equal(u32(s.uniq), os_.uniq)
         for l in range(len(sh.fanouts)):
@@ -135,19 +131,70 @@ def check_config(name, Ks=None, handoff=False):
             assert np.array_equal(u32(s.indices[l]), os_.indices[l]), (b, l)
             if sh.sampler == "rwalk":
                 assert np.array_equal(u32(s.weights[l]), os_.weights[l]), (b, l)
+        assert np.array_equal(s.cache_slot.cpu().numpy(), slot_map[os_.uniq]), b
         st = ctx.extract_sample(out, stats=True)
-        idx = rng.integers(0, s.sizes[-1], 2048)
-        got = out[torch.from_numpy(idx).cuda()].cpu().numpy()
-        assert np.array_equal(got.view(np.uint32), g.features[os_.uniq[idx]].view(np.uint32))
-        slot = ctx.cache_slots()
-        assert st["hits"] == int((slot[os_.uniq] >= 0).sum())
+        assert st["hits"] == int((slot_map[os_.uniq] >= 0).sum())
+        assert st["misses"] == int((slot_map[os_.uniq] < 0).sum())
+        assert_rows_exact(go, out, os_.uniq)
+
+
+def check_config(name, Ks=None, handoff=False, relabel_modes=("auto",)):
+    """PreSC#K counts in full (every K), cache slots at every alpha of the config, then
+    four measured batches (first, second, a random one, the last partial one) at the
+    paper's R% (sh.alphas[0]: misses over PCIe) and one at alpha = 1 (all HBM hits), every
+    output and every extracted byte; optionally again in other relabel modes."""
+    sh = synth.SHAPES[name]
+    g = synth.make_graph(sh)
+    go = oracle.GraphOracle(g.indptr, g.indices, g.features)
+    counts_by_K = {}
+    ub = sh.batch
+    for k in sh.fanouts:
+        ub = min(ub * (1 + k), sh.V)
+    out = torch.empty((ub, sh.D), dtype=torch.float32, device="cuda")
+    ctx = None
+    for mode in relabel_modes:
+        ctx = make_sampler_ctx(g, sh, relabel=mode)
+        if mode != "auto":
+            assert ctx.relabel_mode == mode
+        for K in (Ks or [sh.K]):
+            ctx.reset_counts(glb.COUNT_PRESAMPLE)
+            ctx.presample(K)
+            if K not in counts_by_K:
+                counts_by_K[K] = oracle_counts_parallel(g, sh, range(K))
+            counts = counts_by_K[K]
+            assert np.array_equal(ctx.get_counts(glb.COUNT_PRESAMPLE), counts), (mode, K)
+            if mode == relabel_modes[0]:
+                for a in sh.alphas:
+                    ctx.build_cache(a)
+                    assert np.array_equal(ctx.cache_slots(), oracle.cache_slots(counts, a)), (K, a)
+        e = max(Ks or [sh.K])
+        nb = -(-len(g.train) // sh.batch)
+        rng = np.random.default_rng(0)
+        a0 = sh.alphas[0]
+        ctx.build_cache(a0)
+        slot_map = oracle.cache_slots(counts, a0)
+        assert a0 < 1.0
+        check_batches(ctx, g, sh, go, e, [0, 1, int(rng.integers(2, nb - 1)), nb - 1], out,
+                      slot_map)
+        ctx.build_cache(1.0)
+        check_batches(ctx, g, sh, go, e, [int(rng.integers(0, nb))], out,
+                      oracle.cache_slots(counts, 1.0))
+        if mode != relabel_modes[-1]:
+            ctx.close()
     if handoff:
-        check_handoff(g, sh, go, ctx, oracle.cache_slots(counts, sh.alphas[-1]), e)
+        ctx.build_cache(a0)
+        check_handoff(g, sh, go, ctx, oracle.cache_slots(counts, a0), e)
     ctx.close()
 
 
 def test_tw_fullsize():
-    check_config("TW")
+    """configs[2]; also in hash relabel mode (bit-identical by construction)."""
+    check_config("TW", relabel_modes=("auto", "hash"))
+
+
+def test_tww_weighted_fullsize():
+    """NEXT-1 at Twitter size: 3-hop weighted k-hop (edge weight = target year)."""
+    check_config("TWW")
 
 
 def test_pa_fullsize_presc_k123():

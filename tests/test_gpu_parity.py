@@ -224,17 +224,26 @@ def test_presample_cache_and_hit_stats(tiny, mode):
         assert hs["hits"] <= hs["optimal_hits"]
 
 
-@pytest.mark.parametrize("mode", MODES + ["bulk", "bulkmiss", "bulkboth"])
+GATHER_ENV = {"warp": {"GLB_GATHER_WARP": "1"}, "block": {"GLB_GATHER_WARP": "0"},
+              "nobins": {"GLB_MISS_BIN_LOG2": "0"},
+              "finebins": {"GLB_MISS_BIN_LOG2": "7"},  # one bin per row: the device-scan path
+              "warp_finebins": {"GLB_GATHER_WARP": "1", "GLB_MISS_BIN_LOG2": "7"}}
+
+
+@pytest.mark.parametrize("mode", MODES + ["bulk", "bulkmiss", "bulkboth"] + list(GATHER_ENV))
 @pytest.mark.parametrize("alpha", [0.0, 0.1, 0.5, 1.0])
 def test_extract_sample_bytes(tiny, alpha, mode, monkeypatch):
     """mode 'bulk': hits through the cp.async.bulk gather (GLB_GATHER_BULK=1, off by
-    default), misses through the LSU gather."""
+    default), misses through the LSU gather; GATHER_ENV: the block / warp-independent
+    gathers and the miss orderings (none, 2 MB bins, one bin per row)."""
     g, go = tiny
     sh = g.shape
     if mode in ("bulk", "bulkboth"):
         monkeypatch.setenv("GLB_GATHER_BULK", "1")
     if mode in ("bulkmiss", "bulkboth"):
         monkeypatch.setenv("GLB_MISS_BULK", "1")
+    for k, v in GATHER_ENV.get(mode, {}).items():
+        monkeypatch.setenv(k, v)
     ctx = make_ctx(g, fanouts=sh.fanouts, mode=mode if mode in MODES else "auto")
     ctx.presample(1)
     ctx.build_cache(alpha)
@@ -255,8 +264,11 @@ def test_extract_sample_bytes(tiny, alpha, mode, monkeypatch):
         assert np.array_equal(s.cache_slot.cpu().numpy(), slot[os_.uniq])
 
 
+@pytest.mark.parametrize("variant", ["default"] + list(GATHER_ENV))
 @pytest.mark.parametrize("D", [7, 32, 64, 100, 128, 256])
-def test_extract_generic_ids_dims(D):
+def test_extract_generic_ids_dims(D, variant, monkeypatch):
+    for k, v in GATHER_ENV.get(variant, {}).items():
+        monkeypatch.setenv(k, v)
     V = 3000
     g = synth.small_graph(V, 20000, 2.2, D, 300, seed=D)
     go = oracle.GraphOracle(g.indptr, g.indices, g.features)
@@ -294,7 +306,9 @@ def pr():
 @pytest.mark.slow
 def test_pr_full_size_parity(pr):
     """configs[1] at full size, bench launch configuration: PreSC#1 counts in
-    full, cache slots at the sweep's alphas, and every output of four batches."""
+    full, cache slots at the sweep's alphas, and every output of four batches --
+    every extracted byte -- at alpha = 1 (all HBM hits) and at alpha = 0.05 (most rows
+    over PCIe from the pinned host matrix)."""
     g, go = pr
     sh = g.shape
     ctx = make_ctx(g, fanouts=sh.fanouts)
@@ -304,22 +318,24 @@ def test_pr_full_size_parity(pr):
     for a in (0.05, 0.25):
         ctx.build_cache(a)
         assert np.array_equal(ctx.cache_slots(), oracle.cache_slots(counts, a))
-    ctx.build_cache(1.0)
     e = sh.K
     ob = oracle.epoch_batches(g.train, sh.batch, g.seed, e)
     nb = len(ob)
     rng = np.random.default_rng(0)
     out = torch.empty((sh.batch * 26 * 11, g.D), device="cuda")
-    for b in [0, 1, int(rng.integers(2, nb - 1)), nb - 1]:
-        ctx.sample_batch(e, b)
-        s = ctx.sample_result()
-        os_ = go.sample_khop(ob[b], sh.fanouts, g.seed, e, b)
-        assert_same_sample(s, os_)
-        ctx.extract_sample(out)
-        torch.cuda.synchronize()
-        idx = rng.integers(0, s.sizes[-1], 4096)
-        got = out[torch.from_numpy(idx).cuda()].cpu().numpy()
-        assert np.array_equal(got.view(np.uint32), g.features[os_.uniq[idx]].view(np.uint32))
+    for a in (1.0, 0.05):
+        ctx.build_cache(a)
+        slot = oracle.cache_slots(counts, a)
+        for b in [0, 1, int(rng.integers(2, nb - 1)), nb - 1]:
+            ctx.sample_batch(e, b)
+            s = ctx.sample_result()
+            os_ = go.sample_khop(ob[b], sh.fanouts, g.seed, e, b)
+            assert_same_sample(s, os_)
+            st = ctx.extract_sample(out, stats=True)
+            assert st["hits"] == int((slot[os_.uniq] >= 0).sum())
+            n = s.sizes[-1]
+            got = out[:n].cpu().numpy().view(np.uint32)
+            assert np.array_equal(got, go.extract(os_.uniq).view(np.uint32)), (a, b)
 
 
 @pytest.mark.parametrize("alpha", [1.0, 0.3])

@@ -336,3 +336,37 @@ def test_dynamic_switching_protocol(tmp_path, world, ns, t_standby, expect_switc
         mine = [g for g in roles.trainer_batches(r, total) if g not in set(local)]
         assert np.load(tmp_path / f"t{r}.npy").tolist() == mine
     assert sum(int(np.load(tmp_path / f"s{r}.npy")[0]) for r in range(ns)) == total
+
+
+# ------------------------------------------------- node-shared host inputs
+def _shm_worker(rank, world, port, outdir):
+    import synth
+    from synth import shm
+    _init(rank, world, port)
+    store = dist.distributed_c10d._get_default_store()
+    sg = shm.make_graph_shared("tiny", rank, world, store)
+    g = sg.graph
+    ref = synth.make_graph("tiny")
+    same = all(np.array_equal(getattr(g, n), getattr(ref, n))
+               for n in ("indptr", "indices", "train", "features"))
+    dist.barrier()
+    if rank == 0:  # a write by the owner is seen by every rank: one physical copy
+        g.features[5, 3] = 1234.5
+    dist.barrier()
+    seen = float(g.features[5, 3])
+    with open(os.path.join(outdir, f"r{rank}.txt"), "w") as f:
+        f.write(f"{int(same)} {seen} {int(sg.owner)} {g.features.ctypes.data % 4096}")
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_node_shared_graph(tmp_path, world):
+    """Local rank 0 generates the graph into memfds; the other ranks map the same pages
+    (values equal the private generator's, writes are shared, features page-aligned for
+    cudaHostRegister)."""
+    mp.spawn(_shm_worker, args=(world, free_port(), str(tmp_path)), nprocs=world, join=True)
+    for r in range(world):
+        same, seen, owner, align = open(tmp_path / f"r{r}.txt").read().split()
+        assert same == "1" and float(seen) == 1234.5 and int(align) == 0
+        assert int(owner) == (r == 0)
