@@ -806,11 +806,54 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
             "extract_hbm_bytes_per_step": statistics.mean(hbm_bytes),
             "host_link_bytes_per_step": statistics.mean(link_bytes)}
 
-    # ---- e2e through the public API with host buffers: every step copies its seeds from
-    # pinned host memory (glb_sample_async, H2D on the ctx stream) and reads its result --
-    # the extract's (hits, misses, peer hits) -- back into pinned host memory (stream-ordered
-    # D2H); the host consumes the result of step j-D while step j runs (D = the pipeline
-    # depth).  Wall clock from the first call to the last result on the host.
+    e2e = e2e_measure(args, ctx, g, sh, timed_steps, batch_of, n_seeds, out, xs, world, dev)
+    import gc
+    gc.collect()  # pinned host tensors used on the ctx's extract stream die before the ctx
+    torch.cuda.synchronize()
+
+    res = {"value": value, "ms_per_step": elapsed_max / K, "runs": runs,
+           "runs_range": [min(runs), max(runs)], "runs_ms": run_ms,
+           "roofline": roof, "path_roofline": path, "e2e": e2e, "gpu_launches": launches,
+           "clocks": clk, "host_wall_ms_timed_region": wall_ms[med],
+           "host_enqueue_ms_timed_region": enq_ms[med],
+           "units": {"mean_n_L": statistics.mean(nL), "mean_hits": statistics.mean(hits),
+                     "mean_misses": statistics.mean(misses)},
+           "preprocess_s": {"generate_inputs": t_gen, "load_graph": t_load,
+                            "presample": t_pre, "build_cache": t_cache},
+           "cache": {"layout": args.cache, "rows_cached": ctx_cache_rows},
+           "relabel_table": ctx.relabel_mode, "relabel_l2_window_bytes": ctx.relabel_l2_window,
+           "host_inputs": ("node-shared memfd, generated once by local rank 0 and mapped by "
+                           f"{local_world} ranks") if shared else "private to this rank"}
+
+    # ---- hit rate vs Optimal (accesses recorded over measured epochs, untimed)
+    if args.cache == "sharded":
+        k = ctx.last_extract_counts()
+        res["cache"]["peer_hit_share"] = k["peer_hits"] / max(1, k["hits"] + k["misses"])
+        barrier()  # peers may still read this rank's shard: nobody rebuilds before here
+    if full and not args.no_sweep:
+        res.update(hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs,
+                                   batch_of, n_seeds, barrier))
+    if full and rank == 0 and world == 1 and not args.no_cpu_baseline:
+        res["cpu_baseline"] = cpu_baseline(g, sh, args.cpu_seconds)
+    ctx.close()
+    del out
+    torch.cuda.empty_cache()
+    return res
+
+
+def e2e_measure(args, ctx, g, sh, timed_steps, batch_of, n_seeds, out, xs, world, dev):
+    """e2e through the public API with host buffers: every step copies its seeds from
+    pinned host memory (glb_sample_async, H2D on the ctx stream) and reads its result --
+    the extract's (hits, misses, peer hits) -- back into pinned host memory (stream-ordered
+    D2H); the host consumes the result of step j-D while step j runs (D = the pipeline
+    depth).  Wall clock from the first call to the last result on the host."""
+    import torch
+    import torch.distributed as dist
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
     e2e_steps = timed_steps[: max(1, min(len(timed_steps), 200))]
     host_seeds = {}
     for i in e2e_steps:
@@ -883,35 +926,8 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
            "rows_extracted": e2e_rows, "sync_api_value": e2e_sync_val,
            "sync_api": "glb_sample(host seeds; sizes D2H, sync) + glb_extract_sample "
                        "+ stats (sync) every step"}
-
-    res = {"value": value, "ms_per_step": elapsed_max / K, "runs": runs,
-           "runs_range": [min(runs), max(runs)], "runs_ms": run_ms,
-           "roofline": roof, "path_roofline": path, "e2e": e2e, "gpu_launches": launches,
-           "clocks": clk, "host_wall_ms_timed_region": wall_ms[med],
-           "host_enqueue_ms_timed_region": enq_ms[med],
-           "units": {"mean_n_L": statistics.mean(nL), "mean_hits": statistics.mean(hits),
-                     "mean_misses": statistics.mean(misses)},
-           "preprocess_s": {"generate_inputs": t_gen, "load_graph": t_load,
-                            "presample": t_pre, "build_cache": t_cache},
-           "cache": {"layout": args.cache, "rows_cached": ctx_cache_rows},
-           "relabel_table": ctx.relabel_mode, "relabel_l2_window_bytes": ctx.relabel_l2_window,
-           "host_inputs": ("node-shared memfd, generated once by local rank 0 and mapped by "
-                           f"{local_world} ranks") if shared else "private to this rank"}
-
-    # ---- hit rate vs Optimal (accesses recorded over measured epochs, untimed)
-    if args.cache == "sharded":
-        k = ctx.last_extract_counts()
-        res["cache"]["peer_hit_share"] = k["peer_hits"] / max(1, k["hits"] + k["misses"])
-        barrier()  # peers may still read this rank's shard: nobody rebuilds before here
-    if full and not args.no_sweep:
-        res.update(hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs,
-                                   batch_of, n_seeds, barrier))
-    if full and rank == 0 and world == 1 and not args.no_cpu_baseline:
-        res["cpu_baseline"] = cpu_baseline(g, sh, args.cpu_seconds)
-    ctx.close()
-    del out
-    torch.cuda.empty_cache()
-    return res
+    torch.cuda.synchronize()
+    return e2e
 
 
 def hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs, batch_of,

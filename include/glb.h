@@ -104,7 +104,7 @@ glb_status glb_relabel_mode(const glb_ctx* ctx, int* out);
  * environment GLB_L2_PIN=0 / 1 forces it off / on. */
 glb_status glb_relabel_l2_window(const glb_ctx* ctx, uint64_t* bytes_out);
 
-/* Training set T (host u32[n], distinct, each < V) and mini-batch size B
+/* Training set T (host u32[n], distinct -- a duplicate is EINVAL -- each < V) and mini-batch size B
  * (L305 §6.2: shuffle T each epoch and divide it; last batch partial).
  * seed keys every draw of the ctx (shuffle and sampling).  Synchronous. */
 glb_status glb_set_train_set(glb_ctx* ctx, const uint32_t* train, uint64_t n, uint32_t batch_size,
@@ -244,7 +244,10 @@ glb_status glb_hit_stats_get(glb_ctx* ctx, glb_hit_stats* out);
  * for i < n, bytes exact; cache hits read the HBM cache, misses read the
  * mapped pinned host matrix over PCIe (zero copy).  vertices: device u32[n]
  * (any ids < V, duplicates allowed); out: device f32[n][D], caller-owned.
- * stats (nullable, HOST pointer): filled at the next glb_sync. */
+ * stats (nullable, HOST pointer): filled at the next glb_sync; one extract's stats can be
+ * pending at a time -- an extract that asks for stats while another's are pending
+ * synchronises first.  At pipeline depth 2 glb_extract is ordered after every extract
+ * already enqueued on the extract stream (they share the miss-ordering scratch). */
 typedef struct { uint64_t hits, misses; } glb_extract_stats;
 glb_status glb_extract(glb_ctx* ctx, const uint32_t* vertices, uint64_t n, void* out,
                        glb_extract_stats* stats);
@@ -262,6 +265,21 @@ glb_status glb_extract_sample(glb_ctx* ctx, void* out, glb_extract_stats* stats)
  * work on the main stream.  Synchronous. */
 glb_status glb_set_pipeline(glb_ctx* ctx, int depth);
 glb_status glb_extract_stream(glb_ctx* ctx, void** cuda_stream_out);
+/* Host-assisted misses (L252: the Trainer extracts "from host memory and the feature cache
+ * in GPU memory" simultaneously; L79: Extract is bound by the host link).  glb_extract_sample
+ * orders a batch's misses by host address; the extract kernel reads the first (1 - fraction)
+ * of them from the mapped host matrix (zero copy), while `threads` host threads copy the rest
+ * into a pinned staging buffer that the GPU then reads sequentially and scatters into `out`
+ * -- random 512-byte zero-copy reads are bound by per-row address translation, the staged
+ * rows are not, and the two streams share the link.  Asynchronous: the host
+ * copies run in stream host functions (no host sync in the caller).  Results are identical
+ * for every fraction.  fraction 0 = off (default; environment GLB_HOST_GATHER = permille,
+ * GLB_HOST_GATHER_THREADS); threads 0 = the usable cores minus two.  Applies to samples of
+ * this ctx (not to handoff-received ones) and to caches with C < V.  Synchronous (creates the
+ * thread pool).  Errors: EINVAL (fraction not in [0,1), threads > 256). */
+glb_status glb_set_host_gather(glb_ctx* ctx, uint32_t threads, double fraction);
+glb_status glb_host_gather(const glb_ctx* ctx, uint32_t* threads, double* fraction);
+
 /* Timing of the extract kernel itself: CUDA events around every `period`-th
  * glb_extract_sample launch (period 1 = each; 0 = off), on the stream it runs on -- events
  * between the launches of a pipelined step cost overlap, so a bench samples them.

@@ -42,6 +42,7 @@ EXPORTS = [
     "glb_sample_async", "glb_extract_counts_device_ptr",
     "glb_handoff_create", "glb_handoff_attach", "glb_handoff_connect", "glb_handoff_send",
     "glb_handoff_recv", "glb_handoff_tag", "glb_handoff_release", "glb_relabel_l2_window",
+    "glb_set_host_gather", "glb_host_gather",
 ]
 MAX_SHARDS = 16
 IPC_HANDLE_BYTES = 64
@@ -147,6 +148,8 @@ def lib(auto_build: bool = True):
         "glb_handoff_recv": ([vp, u32, u32], i32),
         "glb_handoff_tag": ([vp, ctypes.POINTER(u64)], i32),
         "glb_handoff_release": ([vp, u32], i32),
+        "glb_set_host_gather": ([vp, u32, dbl], i32),
+        "glb_host_gather": ([vp, ctypes.POINTER(u32), ctypes.POINTER(dbl)], i32),
         "glb_footprint_similarity": ([vp, vp, vp, dbl, ctypes.POINTER(u64), ctypes.POINTER(u64),
                                       ctypes.POINTER(dbl)], i32),
     }
@@ -533,6 +536,18 @@ class Context:
             self.sync()
             return {"hits": st.hits, "misses": st.misses}
         return None
+
+    def set_host_gather(self, fraction: float, threads: int = 0):
+        """Host-assisted misses: `fraction` of each sample's (address-ordered) misses are
+        copied by `threads` host threads into pinned staging that the GPU reads back
+        sequentially (include/glb.h glb_set_host_gather); 0 turns it off."""
+        self._ck(self._lib.glb_set_host_gather(self._h, int(threads), float(fraction)))
+
+    @property
+    def host_gather(self):
+        t, f = ctypes.c_uint32(), ctypes.c_double()
+        self._ck(self._lib.glb_host_gather(self._h, ctypes.byref(t), ctypes.byref(f)))
+        return {"threads": t.value, "fraction": f.value}
 
     def set_pipeline(self, depth: int):
         """depth 2: double-buffered samples, extract on its own stream overlapping the

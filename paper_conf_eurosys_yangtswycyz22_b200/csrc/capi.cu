@@ -10,6 +10,7 @@
 #include <cstddef>
 #include <cstring>
 #include <new>
+#include <thread>
 
 #include "glb_internal.cuh"
 
@@ -87,6 +88,7 @@ cudaError_t sync_all(glb_ctx* c) {
   cudaError_t e = cudaStreamSynchronize(c->stream);
   if (e == cudaSuccess && c->xstream) e = cudaStreamSynchronize(c->xstream);
   if (e == cudaSuccess && c->sstream) e = cudaStreamSynchronize(c->sstream);
+  if (e == cudaSuccess) e = hg_sync(c);
   return e;
 }
 
@@ -341,6 +343,17 @@ glb_status glb_create(int device, glb_ctx** out) {
   if (const char* g = getenv("GLB_GATHER_BULK")) c->gather_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_MISS_BULK")) c->miss_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_WARP")) c->gather_warp = atoi(g) != 0;
+  if (const char* g = getenv("GLB_RELABEL_DEDUP")) c->relabel_dedup = atoi(g) != 0;
+  if (const char* g = getenv("GLB_HOST_GATHER")) {  // permille of the misses, host-gathered
+    const int pm = atoi(g);
+    const char* t = getenv("GLB_HOST_GATHER_THREADS");
+    if (pm > 0 && pm < 1000 &&
+        glb_set_host_gather(c, t ? (uint32_t)atoi(t) : 0u, pm / 1000.0) != GLB_OK) {
+      glb_status s = set_err(nullptr, GLB_ECUDA, "glb_create: host gather: %s", c->err.c_str());
+      glb_destroy(c);
+      return s;
+    }
+  }
   if (const char* g = getenv("GLB_GATHER_BULK_SMEM")) c->gather_bulk_smem = (uint32_t)atoi(g);
   if (const char* g = getenv("GLB_PERM_PREFETCH")) c->perm_prefetch = atoi(g) != 0;
   if (const char* g = getenv("GLB_MISS_BIN_LOG2")) {
@@ -357,6 +370,7 @@ glb_status glb_destroy(glb_ctx* c) {
   if (c->stream) cudaStreamSynchronize(c->stream);
   if (c->xstream) cudaStreamSynchronize(c->xstream);
   if (c->sstream) cudaStreamSynchronize(c->sstream);
+  hg_free(c);
   handoff_free(c);
   free_sample_bufs(c);
   free_graph(c);
@@ -1121,9 +1135,14 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
     e = launch_sort_misses(c, c->sb.miss_list, &c->st->nmiss, c->sb.miss_sorted);
     misses = c->sb.miss_sorted;
   }
+  // host-assisted misses: the tail of the ordered list is gathered by host threads
+  const bool hg = hg_active(c);
+  uint32_t* dcnt = nullptr;
+  if (e == cudaSuccess && hg) e = hg_enqueue(c, (float*)out, misses, &dcnt);
   if (e == cudaSuccess)
     e = launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_list, misses,
-                      nullptr, &c->st->nhit, 0, 0);
+                      nullptr, dcnt ? dcnt : &c->st->nhit, 0, 0);
+  if (e == cudaSuccess && hg) e = hg_join(c);
   if (e == cudaSuccess && t1) e = cudaEventRecord(t1, c->stream);
   if (e == cudaSuccess && stats) {
     e = cudaMemcpyAsync(c->h_xcount, c->xcount, 3 * sizeof(unsigned long long),
@@ -1177,6 +1196,35 @@ glb_status glb_set_timing(glb_ctx* c, int enable /* period */) {
   c->timing = enable;
   c->timing_calls = 0;
   c->tev_used = 0;
+  return GLB_OK;
+}
+
+glb_status glb_set_host_gather(glb_ctx* c, uint32_t threads, double fraction) {
+  ENTER(c);
+  if (!(fraction >= 0.0 && fraction < 1.0)) return set_err(c, GLB_EINVAL, "fraction %g not in [0,1)", fraction);
+  if (threads > 256) return set_err(c, GLB_EINVAL, "threads %u > 256", threads);
+  CK(sync_all(c));
+  const uint32_t pm = (uint32_t)std::lround(fraction * 1000.0);
+  if (pm == 0) {
+    hg_free(c);
+    c->hg_permille = 0;
+    c->hg_threads = 0;
+    return GLB_OK;
+  }
+  if (threads == 0) {  // auto: the usable cores minus two (the caller's thread, the driver's)
+    const unsigned n = std::thread::hardware_concurrency();
+    threads = n > 3 ? n - 2 : 1;
+  }
+  CK(hg_configure(c, threads - 1));  // the host-function thread itself is the last worker
+  c->hg_permille = pm;
+  c->hg_threads = threads;
+  return GLB_OK;
+}
+
+glb_status glb_host_gather(const glb_ctx* c, uint32_t* threads, double* fraction) {
+  if (!c) return GLB_EINVAL;
+  if (threads) *threads = c->hg_threads;
+  if (fraction) *fraction = c->hg_permille / 1000.0;
   return GLB_OK;
 }
 

@@ -162,6 +162,8 @@ struct HandoffSend {  // sampler side, one per attached trainer
   cudaEvent_t ready[kHandoffMaxSlots] = {};     // own, interprocess
 };
 
+struct HostGather;  // hostgather.cu: host-assisted miss gather (threads, streams, staging)
+
 }  // namespace glb
 
 struct glb_ctx {
@@ -190,6 +192,7 @@ struct glb_ctx {
   uint32_t hmask = 0;
   bool hash_mode = false;
   int relabel_mode = 0;         // 0 auto, 1 dense, 2 hash (glb_set_relabel_mode)
+  int relabel_dedup = 0;        // GLB_RELABEL_DEDUP=1: warp-level pre-dedup of picks (k_khop)
   glb::L2Window pin;            // persisting-L2 window over the relabel table
   int l2_pin = -1;              // -1 auto (small tables only), GLB_L2_PIN=0 off / 1 on
   uint32_t gen = 0;
@@ -205,6 +208,9 @@ struct glb_ctx {
   uint32_t gather_bulk_smem = 96 * 1024;  // row-slot bytes per bulk block (GLB_GATHER_BULK_SMEM)
   int miss_bulk = 0;           // GLB_MISS_BULK=1: host misses through cp.async.bulk
   int gather_warp = 0;         // GLB_GATHER_WARP=1: warp-independent gather (k_gather_w)
+  glb::HostGather* hg = nullptr;  // host-assisted misses (glb_set_host_gather)
+  uint32_t hg_permille = 0;       // share of a batch's misses gathered by host threads
+  uint32_t hg_threads = 0;
   uint64_t C = 0;
   // NEXT-3 peer-sharded cache: global rank i < C is owned by shard i % W at row i / W;
   // shard_base[r] = device pointer (valid in this process) of shard r's rows.
@@ -390,6 +396,15 @@ cudaError_t launch_similarity(glb_ctx* c, const uint32_t* fi, const uint32_t* fj
 cudaError_t launch_hit_stats(glb_ctx* c, unsigned long long* out3 /* total,hits,max */);
 cudaError_t launch_value_hist(glb_ctx* c, const uint32_t* a, uint64_t n, unsigned long long* bins,
                               uint32_t nbins);
+
+// hostgather.cu: a fraction of the misses gathered by host threads into pinned staging,
+// read back sequentially by the GPU (glb_set_host_gather)
+cudaError_t hg_configure(glb_ctx* c, uint32_t threads);
+void hg_free(glb_ctx* c);
+bool hg_active(const glb_ctx* c);
+cudaError_t hg_enqueue(glb_ctx* c, float* out, const uint2* miss_sorted, uint32_t** dcnt_out);
+cudaError_t hg_join(glb_ctx* c);
+cudaError_t hg_sync(glb_ctx* c);
 
 inline void count_launch(glb_ctx* c, int n = 1) { c->launches += (uint64_t)n; }
 

@@ -238,7 +238,13 @@ __global__ void __launch_bounds__(kThreads)
 // ---------------------------------------------------------------- k-hop (k lanes / vertex)
 // Fanout k <= 32: floor(32/k) frontier vertices per warp, lane s of a group
 // owns Floyd slot s.
-template <bool HASH>
+//
+// DEDUP (GLB_RELABEL_DEDUP=1, the north star's staged insert at warp scope): picks of the
+// same gid within a warp are combined first (__match_any_sync) -- only the lowest lane,
+// which holds the smallest flat position, probes / inserts into the relabel table, and
+// the value it read is broadcast to its peers, so a hub picked by several frontier
+// vertices of one warp costs one table access instead of several.
+template <bool HASH, bool DEDUP>
 __global__ void __launch_bounds__(kThreads)
     k_khop(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch, Table T,
            const DevState* __restrict__ st, DevState* st_w, const uint64_t* __restrict__ indptr,
@@ -298,7 +304,24 @@ __global__ void __launch_bounds__(kThreads)
     }
     if (!big && active && s < deg) sel = s;
     uint32_t u = kEmpty, idx = kEmpty;
-    if (sel != kEmpty) {
+    if (DEDUP) {
+      if (sel != kEmpty) u = __ldg(indices + lo + sel);
+      // lanes with the same gid: flat positions grow with the lane, so the lowest lane
+      // holds the first occurrence within the warp
+      const unsigned long long key =
+          sel != kEmpty ? (unsigned long long)u : ((1ull << 63) | (unsigned)lane);
+      const uint32_t peers = __match_any_sync(kFull, key);
+      const int leader = __ffs(peers) - 1;
+      unsigned long long old = ~0ull;
+      if (sel != kEmpty && lane == leader) {
+        idx = entry_of<HASH>(T, u, st_w);
+        if (idx != kEmpty) old = vmap_insert(T.e, idx, enc_pos(gen, base + d * k + s));
+      }
+      idx = __shfl_sync(kFull, idx, leader);
+      old = __shfl_sync(kFull, old, leader);
+      if (sel != kEmpty)
+        u = idx != kEmpty ? encode_pick(u, old, enc_pos(gen, base + d * k + s), base) : kEmpty;
+    } else if (sel != kEmpty) {
       u = __ldg(indices + lo + sel);
       idx = entry_of<HASH>(T, u, st_w);
       if (idx != kEmpty) {
@@ -937,9 +960,12 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
   const Table T = table_of(c);
   cudaError_t e;
 #define GLB_KH_ARGS hop, k, seed, epoch, batch, T, stc, c->st, ip, ix, uq, b.picks, b.pidx, fix
-  if (k <= 32)
-    e = c->hash_mode ? launch_pdl_w(c->pin, k_khop<true>, grid, kThreads, c->stream, GLB_KH_ARGS)
-                     : launch_pdl_w(c->pin, k_khop<false>, grid, kThreads, c->stream, GLB_KH_ARGS);
+  if (k <= 32 && c->relabel_dedup)
+    e = c->hash_mode ? launch_pdl_w(c->pin, k_khop<true, true>, grid, kThreads, c->stream, GLB_KH_ARGS)
+                     : launch_pdl_w(c->pin, k_khop<false, true>, grid, kThreads, c->stream, GLB_KH_ARGS);
+  else if (k <= 32)
+    e = c->hash_mode ? launch_pdl_w(c->pin, k_khop<true, false>, grid, kThreads, c->stream, GLB_KH_ARGS)
+                     : launch_pdl_w(c->pin, k_khop<false, false>, grid, kThreads, c->stream, GLB_KH_ARGS);
   else
     e = c->hash_mode ? launch_pdl_w(c->pin, k_khop_wide<true>, grid, kThreads, c->stream, GLB_KH_ARGS)
                      : launch_pdl_w(c->pin, k_khop_wide<false>, grid, kThreads, c->stream, GLB_KH_ARGS);

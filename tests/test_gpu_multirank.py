@@ -86,3 +86,22 @@ def test_bench_two_ranks(mode, cache, handoff):
         assert d["cache"]["layout"] == "sharded"
         assert d["cache"]["rows_cached"] == 2 * int(0.3 * 10000)
         assert d["cache"]["peer_hit_share"] > 0
+
+
+def test_bench_self_launch_two_ranks():
+    """`bench.py --gpus 2` without a launcher re-executes itself under torch.distributed.run
+    (the driver's command line measures N ranks); local rank 0 generates the host inputs
+    once and the other rank maps them (synth/shm.py)."""
+    cmd = [sys.executable, "bench.py", "--gpus", "2", "--steps", "8", "--warmup", "3",
+           "--runs", "2", "--config", "tiny", "--backend", "gloo", "--no-sweep",
+           "--no-cpu-baseline", "--no-pr-alpha1"]
+    env = {k: v for k, v in os.environ.items()
+           if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK", "LOCAL_WORLD_SIZE")}
+    r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=600, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and len(d["runs"]) == 2
+    assert d["host_inputs"].startswith("node-shared")
+    assert d["config"]["parallelism"] == "dp2"

@@ -84,8 +84,11 @@ def test_worked_example_on_gpu():
     assert ctx.permutation(8).tolist() == gold["shuffle"]["epoch1"]
 
 
-@pytest.mark.parametrize("mode", MODES)
-def test_tiny_every_batch_bit_exact(tiny, mode):
+@pytest.mark.parametrize("mode", MODES + ["dense_dedup", "hash_dedup"])
+def test_tiny_every_batch_bit_exact(tiny, mode, monkeypatch):
+    if mode.endswith("_dedup"):
+        monkeypatch.setenv("GLB_RELABEL_DEDUP", "1")
+        mode = mode[:-6]
     g, go = tiny
     sh = g.shape
     ctx = make_ctx(g, fanouts=sh.fanouts, mode=mode)
@@ -112,8 +115,13 @@ def test_host_and_device_seed_paths(tiny):
 
 
 @pytest.mark.parametrize("fanouts", [(25, 10), (15, 10, 5), (3,), (1, 1, 1), (32, 2), (40, 33)])
-@pytest.mark.parametrize("mode", MODES)
-def test_fanout_variants_power_law(fanouts, mode):
+@pytest.mark.parametrize("mode", MODES + ["dense_dedup", "hash_dedup"])
+def test_fanout_variants_power_law(fanouts, mode, monkeypatch):
+    """*_dedup: picks pre-deduplicated per warp before the relabel-table insert
+    (GLB_RELABEL_DEDUP=1); a small graph with hubs (gamma 2.1), so peers are common."""
+    if mode.endswith("_dedup"):
+        monkeypatch.setenv("GLB_RELABEL_DEDUP", "1")
+        mode = mode[:-6]
     g = synth.small_graph(6000, 90000, 2.1, 8, 700, seed=11)
     go = oracle.GraphOracle(g.indptr, g.indices)
     ctx = make_ctx(g, fanouts=fanouts, max_batch=300, mode=mode)
@@ -227,7 +235,11 @@ def test_presample_cache_and_hit_stats(tiny, mode):
 GATHER_ENV = {"warp": {"GLB_GATHER_WARP": "1"}, "block": {"GLB_GATHER_WARP": "0"},
               "nobins": {"GLB_MISS_BIN_LOG2": "0"},
               "finebins": {"GLB_MISS_BIN_LOG2": "7"},  # one bin per row: the device-scan path
-              "warp_finebins": {"GLB_GATHER_WARP": "1", "GLB_MISS_BIN_LOG2": "7"}}
+              "warp_finebins": {"GLB_GATHER_WARP": "1", "GLB_MISS_BIN_LOG2": "7"},
+              # host-assisted misses (glb_set_host_gather): 40 % / 90 % of them by host threads
+              "host400": {"GLB_HOST_GATHER": "400", "GLB_HOST_GATHER_THREADS": "4"},
+              "host900_nobins": {"GLB_HOST_GATHER": "900", "GLB_HOST_GATHER_THREADS": "3",
+                                 "GLB_MISS_BIN_LOG2": "0"}}
 
 
 @pytest.mark.parametrize("mode", MODES + ["bulk", "bulkmiss", "bulkboth"] + list(GATHER_ENV))
@@ -455,3 +467,41 @@ def test_sample_async_pinned_seeds_and_device_counts(tiny):
         assert np.array_equal(out.cpu().numpy().view(np.uint32), go.extract(uniq).view(np.uint32))
     with pytest.raises(AssertionError):
         ctx.sample_async(torch.from_numpy(batches[0].view(np.int32).copy()))  # pageable
+
+
+@pytest.mark.parametrize("D", [7, 100])
+@pytest.mark.parametrize("depth", [1, 2])
+@pytest.mark.parametrize("fraction", [0.3, 0.75])
+def test_host_gather_every_batch(D, depth, fraction):
+    """Host-assisted misses (glb_set_host_gather): every batch of an epoch, pipelined or not,
+    gives the oracle's bytes and counts; fraction 0 turns it off again."""
+    g = synth.small_graph(6000, 60000, 2.2, D, 500, seed=11 + D)
+    go = oracle.GraphOracle(g.indptr, g.indices, g.features)
+    sh = g.shape
+    ctx = make_ctx(g, fanouts=sh.fanouts, max_batch=sh.batch)
+    ctx.presample(1)
+    ctx.build_cache(0.2)
+    ctx.set_host_gather(fraction, threads=3)
+    assert ctx.host_gather["threads"] == 3 and abs(ctx.host_gather["fraction"] - fraction) < 1e-9
+    ctx.set_pipeline(depth)
+    slot = ctx.cache_slots()
+    e = 1
+    ob = oracle.epoch_batches(g.train, sh.batch, g.seed, e)
+    outs = []
+    for b in range(len(ob)):
+        ctx.sample_batch(e, b)
+        out = torch.full((sh.batch * 11 * 6 + 1, D), float("nan"), device="cuda")
+        st = ctx.extract_sample(out, stats=(depth == 1))  # depth 2: batches stay in flight
+        outs.append((b, out, st))
+    torch.cuda.synchronize()
+    for b, out, st in outs:
+        os_ = go.sample_khop(ob[b], sh.fanouts, g.seed, e, b)
+        n = os_.uniq.shape[0]
+        assert np.array_equal(out[:n].cpu().numpy().view(np.uint32),
+                              go.extract(os_.uniq).view(np.uint32)), b
+        assert torch.isnan(out[n:]).all()
+        if st is not None:
+            assert st["hits"] == int((slot[os_.uniq] >= 0).sum())
+            assert st["misses"] == n - st["hits"]
+    ctx.set_host_gather(0.0)
+    assert ctx.host_gather["fraction"] == 0.0

@@ -33,6 +33,8 @@ def main():
     ap.add_argument("--bins", default="21,0,16,12,9")
     ap.add_argument("--steps", type=int, default=30)
     ap.add_argument("--env", default="", help="extra env k=v,k=v applied before each ctx")
+    ap.add_argument("--hg", default="0", help="host-gather fractions in permille (glb_set_host_gather)")
+    ap.add_argument("--hg-threads", type=int, default=0)
     args = ap.parse_args()
     import paper_conf_eurosys_yangtswycyz22_b200 as glb
     from paper_conf_eurosys_yangtswycyz22_b200 import parallel as par
@@ -43,7 +45,7 @@ def main():
     for kv in filter(None, args.env.split(",")):
         k, v = kv.split("=")
         os.environ[k] = v
-    for b in [int(x) for x in args.bins.split(",")]:
+    for b, hg in [(int(x), int(y)) for x in args.bins.split(",") for y in args.hg.split(",")]:
         os.environ["GLB_MISS_BIN_LOG2"] = str(b)
         ctx = glb.Context(0)
         ctx.load_graph(g.indptr, g.indices, g.features)
@@ -58,6 +60,8 @@ def main():
         nb = ctx.num_batches
         ctx.presample(sh.K)
         ctx.build_cache(args.alpha)
+        if hg:
+            ctx.set_host_gather(hg / 1000.0, threads=args.hg_threads)
         ub = sh.batch
         for k in sh.fanouts:
             ub = min(ub * (1 + k), sh.V)
@@ -95,7 +99,8 @@ def main():
                               "depth": depth, "ms_per_step": s0.elapsed_time(s1) / args.steps,
                               "extract_ms": statistics.mean(xms),
                               "misses_per_step": statistics.mean(misses),
-                              "host_gbs": gbs, "env": args.env}), flush=True)
+                              "host_gbs": gbs, "env": args.env, "host_gather": ctx.host_gather}),
+                  flush=True)
         ctx.close()
         del out
         torch.cuda.empty_cache()
