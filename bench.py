@@ -44,6 +44,10 @@ sys.path.insert(0, ROOT)
 import synth  # noqa: E402
 
 METRIC = "sample+extract seeds/sec at 1/2/4/8 B200; cache hit rate vs optimal (%)"
+# cache ratio R% the paper ran each workload at (Table 5): GSG-PR 100 %,
+# GCN-TW 25 %, PSG-PA 22 %, GSG-UK 18 %; the weighted variants follow their base graph
+PAPER_ALPHA = {"tiny": 0.25, "PR": 1.0, "PRW": 1.0, "TW": 0.25, "TWW": 0.25, "PA": 0.22,
+               "UK": 0.18}
 PCIE_GEN5_X16_GBS = 64.0  # nominal per direction (context only)
 
 
@@ -55,7 +59,7 @@ def parse(argv=None):
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
     p.add_argument("--config", default="PA", choices=list(synth.SHAPES))
     p.add_argument("--alpha", type=float, default=None,
-                   help="cache ratio (default: the shape's paper R%%, synth.SHAPES alphas[0])")
+                   help="cache ratio (default: the paper's R%% for the workload, PAPER_ALPHA)")
     p.add_argument("--runs", type=int, default=3,
                    help="timed regions of K steps each; value = their median (SURVEY §8(d))")
     p.add_argument("--sweep-steps", type=int, default=10)
@@ -94,11 +98,17 @@ def parse(argv=None):
                         "NVLink (NEXT-3; glb_build_cache_sharded)")
     p.add_argument("--time-every", type=int, default=8,
                    help="CUDA events around every n-th extract launch of the timed region")
+    p.add_argument("--host-gather", default="auto",
+                   help="share of each batch's misses gathered by host threads "
+                        "(glb_set_host_gather): a fraction, or 'auto' = 0.25 when a feature "
+                        "row is <= 512 B and alpha < 1 (measured: 512-B zero-copy rows are "
+                        "bound by address translation, 1-KB rows are not; DESIGN.md §10)")
+    p.add_argument("--host-gather-threads", type=int, default=8)
     p.add_argument("--pipeline", type=int, default=2, choices=[1, 2],
                    help="2: extract of batch b overlaps sampling of batch b+1 (two streams)")
     a = p.parse_args(argv)
     if a.alpha is None:
-        a.alpha = synth.SHAPES[a.config].alphas[0]
+        a.alpha = PAPER_ALPHA.get(a.config, 1.0)
     return a
 
 
@@ -640,6 +650,10 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
     torch.cuda.synchronize()
     t_cache = time.perf_counter() - t0
 
+    hg = args.host_gather
+    hg = (0.25 if 4 * sh.D <= 512 and alpha < 1.0 else 0.0) if hg == "auto" else float(hg)
+    if hg > 0:
+        ctx.set_host_gather(hg, threads=args.host_gather_threads)
     ctx_cache_rows = ctx.cache_size
     ub = sh.batch
     for k in sh.fanouts:
@@ -821,6 +835,7 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
            "preprocess_s": {"generate_inputs": t_gen, "load_graph": t_load,
                             "presample": t_pre, "build_cache": t_cache},
            "cache": {"layout": args.cache, "rows_cached": ctx_cache_rows},
+           "host_gather": ctx.host_gather,
            "relabel_table": ctx.relabel_mode, "relabel_l2_window_bytes": ctx.relabel_l2_window,
            "host_inputs": ("node-shared memfd, generated once by local rank 0 and mapped by "
                            f"{local_world} ranks") if shared else "private to this rank"}
@@ -1083,7 +1098,7 @@ def main(argv=None):
             "pr_alpha1": pr1,
             "host": host_info(), "gpu": gpu_info(local),
         }
-        for k in ("cache", "relabel_table", "relabel_l2_window_bytes", "host_inputs",
+        for k in ("cache", "host_gather", "relabel_table", "relabel_l2_window_bytes", "host_inputs",
                   "host_wall_ms_timed_region", "host_enqueue_ms_timed_region", "hit_rate",
                   "alpha_sweep", "presc_k_sweep", "measured_epochs", "footprint_similarity",
                   "units", "preprocess_s"):

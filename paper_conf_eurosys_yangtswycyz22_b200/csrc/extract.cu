@@ -5,10 +5,12 @@
 // time is "mainly dominated by loading features ... from host memory ... due
 // to the limited PCIe bandwidth" (L79 §2).
 //
-// One persistent launch serves both halves: blocks [0, H) gather cache hits
-// from HBM, blocks [H, grid) gather misses straight from the mapped pinned
-// host matrix (zero copy over PCIe), so the HBM gather never waits behind
-// PCIe latency and no CPU thread touches feature bytes.
+// One persistent launch serves both halves: every block first claims chunks of
+// cache hits (HBM) from one device counter and, once those run out, chunks of
+// misses read straight from the mapped pinned host matrix (zero copy over PCIe)
+// from a second counter -- all blocks drain the HBM work before any waits on the
+// host link.  Misses arrive ordered by host address (launch_sort_misses); a
+// share of them can be gathered by host threads instead (hostgather.cu).
 //
 // A block copies a chunk of R rows per iteration: the chunk's (dst, src)
 // work-list entries are staged in shared memory (double-buffered, the next

@@ -87,7 +87,7 @@ SHAPES = {
     "TW": Shape("TW", 41_652_230, 1_468_365_182, 2.1, 2.1, 256, 417_000, 8000, "khop",
                 (15, 10, 5), 1, (0.25, 0.10, 1.0)),
     "PA": Shape("PA", 111_059_956, 1_615_685_872, 3.5, 2.5, 128, 1_207_179, 8000, "rwalk",
-                (5, 5, 5), 1, (0.22, 0.05, 0.10)),
+                (5, 5, 5), 1, (0.22, 0.05, 0.10, 1.0)),
     "UK": Shape("UK", 77_741_046, 2_965_197_340, 3.0, 2.1, 256, 1_000_000, 8000, "khop", (25, 10),
                 1, (0.18, 1.0)),
     # NEXT-1 (not a BASELINE config): Twitter with 3-hop WEIGHTED sampling, edge weight =
