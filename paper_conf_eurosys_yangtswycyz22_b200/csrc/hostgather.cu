@@ -182,6 +182,7 @@ struct HostGather {
   cudaEvent_t ev_split = nullptr, ev_d2h = nullptr, ev_end[2] = {nullptr, nullptr};
   bool dma = false;  // staged rows cross the link by DMA (GLB_HOST_GATHER_DMA=1; measured slower)
   int nch = 4;       // chunks per extract (GLB_HOST_GATHER_CHUNKS)
+  int sblocks = 0;   // scatter grid (GLB_HOST_GATHER_SCATTER_BLOCKS; 0 = one per SM)
   uint64_t cap = 0;  // rows of the host part per slot
   uint32_t D = 0;
   double nm_est = 0;                 // misses per batch (recent batches)
@@ -282,6 +283,7 @@ cudaError_t hg_configure(glb_ctx* c, uint32_t threads) {
     if (!h) return cudaErrorMemoryAllocation;
     c->hg = h;
     if (const char* g = getenv("GLB_HOST_GATHER_DMA")) h->dma = atoi(g) != 0;
+    if (const char* g = getenv("GLB_HOST_GATHER_SCATTER_BLOCKS")) h->sblocks = atoi(g) > 0 ? atoi(g) : 0;
     if (const char* g = getenv("GLB_HOST_GATHER_CHUNKS")) {
       const int n = atoi(g);
       h->nch = n < 1 ? 1 : n > kMaxChunks ? kMaxChunks : n;
@@ -401,11 +403,12 @@ cudaError_t hg_enqueue(glb_ctx* c, float* out, const uint2* miss_sorted, uint32_
         return e;
       src = h->dstage[s];
     }
+    const int sg = h->sblocks ? h->sblocks : c->num_sms;
     if (vec)
-      k_hg_scatter<float4><<<c->num_sms, kThreads, 0, q>>>(
+      k_hg_scatter<float4><<<sg, kThreads, 0, q>>>(
           (float4*)out, (const float4*)src, h->ent_dev[s], h->dcnt[s], lo, hi, U, U);
     else
-      k_hg_scatter<float><<<c->num_sms, kThreads, 0, q>>>(
+      k_hg_scatter<float><<<sg, kThreads, 0, q>>>(
           out, (const float*)src, h->ent_dev[s], h->dcnt[s], lo, hi, U, U);
     count_launch(c);
     if ((e = cudaGetLastError()) != cudaSuccess) return e;

@@ -32,3 +32,31 @@ def test_cpu_baseline_all_cores():
     assert c["kind"] == "oracle" and c["value"] > 0 and c["cores"] >= 1
     if c["cores"] > 1:
         assert c["single_thread"]["cores"] == 1
+
+
+def test_bench_defaults_and_self_launch(monkeypatch):
+    """The default workload is the headline (PA-shaped configs[3] at the paper's R% 0.22);
+    `--gpus N` without a launcher re-executes bench.py under torch.distributed.run."""
+    sys.path.insert(0, ROOT)
+    import bench
+    a = bench.parse([])
+    assert a.config == "PA" and a.alpha == 0.22 and a.gpus == 1 and a.runs == 3
+    assert bench.parse(["--config", "PR"]).alpha == 1.0
+    assert bench.parse(["--config", "UK"]).alpha == 0.18
+    calls = []
+
+    def fake_call(cmd):
+        calls.append(cmd)
+        return 0
+
+    monkeypatch.delenv("WORLD_SIZE", raising=False)
+    monkeypatch.setattr(bench.subprocess, "call", fake_call)
+    try:
+        bench.main(["--gpus", "4", "--steps", "7"])
+    except SystemExit as e:
+        assert e.code == 0
+    assert len(calls) == 1
+    cmd = calls[0]
+    assert "torch.distributed.run" in cmd and "--nproc-per-node=4" in cmd
+    assert cmd[cmd.index("--master-addr") + 1] == "127.0.0.1"
+    assert cmd[-4:] == ["--gpus", "4", "--steps", "7"]
