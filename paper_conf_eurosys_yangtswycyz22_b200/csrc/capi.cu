@@ -343,7 +343,10 @@ glb_status glb_create(int device, glb_ctx** out) {
   if (const char* g = getenv("GLB_GATHER_BULK")) c->gather_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_MISS_BULK")) c->miss_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_WARP")) c->gather_warp = atoi(g) != 0;
-  if (const char* g = getenv("GLB_RELABEL_DEDUP")) c->relabel_dedup = atoi(g) != 0;
+  if (const char* g = getenv("GLB_RELABEL_DEDUP")) {  // 1 warp-level, 2 block smem-staged
+    const int m = atoi(g);
+    c->relabel_dedup = m >= 0 && m <= 2 ? m : 0;
+  }
   if (const char* g = getenv("GLB_HOST_GATHER")) {  // permille of the misses, host-gathered
     const int pm = atoi(g);
     const char* t = getenv("GLB_HOST_GATHER_THREADS");

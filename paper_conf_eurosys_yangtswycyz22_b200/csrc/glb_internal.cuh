@@ -192,7 +192,8 @@ struct glb_ctx {
   uint32_t hmask = 0;
   bool hash_mode = false;
   int relabel_mode = 0;         // 0 auto, 1 dense, 2 hash (glb_set_relabel_mode)
-  int relabel_dedup = 0;        // GLB_RELABEL_DEDUP=1: warp-level pre-dedup of picks (k_khop)
+  int relabel_dedup = 0;        // GLB_RELABEL_DEDUP: 1 warp-level / 2 block smem-staged pre-dedup
+                                // of picks before the relabel-table insert (k_khop)
   glb::L2Window pin;            // persisting-L2 window over the relabel table
   int l2_pin = -1;              // -1 auto (small tables only), GLB_L2_PIN=0 off / 1 on
   uint32_t gen = 0;

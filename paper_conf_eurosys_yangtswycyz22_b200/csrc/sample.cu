@@ -244,7 +244,15 @@ __global__ void __launch_bounds__(kThreads)
 // which holds the smallest flat position, probes / inserts into the relabel table, and
 // the value it read is broadcast to its peers, so a hub picked by several frontier
 // vertices of one warp costs one table access instead of several.
-template <bool HASH, bool DEDUP>
+//
+// DEDUP == 2 (GLB_RELABEL_DEDUP=2, the north star's "shared-memory-staged open-addressing
+// hash insert"): the whole block's picks of one iteration (8 warps) are first
+// inserted into a 512-entry open-addressing table in shared memory keyed by gid, with the
+// smallest flat position per gid (smem atomicMin); after a barrier only that pick probes /
+// inserts into the global relabel table, and its result is shared through the smem table.
+// The loop is block-uniform (same vertex-to-warp mapping as the warp-strided loop).
+constexpr uint32_t kStageEntries = 2 * kThreads;  // smem table (load factor <= 1/2)
+template <bool HASH, int DEDUP>
 __global__ void __launch_bounds__(kThreads)
     k_khop(uint32_t hop, uint32_t k, uint64_t seed, uint32_t epoch, uint32_t batch, Table T,
            const DevState* __restrict__ st, DevState* st_w, const uint64_t* __restrict__ indptr,
@@ -264,7 +272,24 @@ __global__ void __launch_bounds__(kThreads)
   const int gbase = (int)(gi * k);
   const uint32_t warp_global = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
-  for (uint32_t w0 = warp_global * gpw; w0 < n_l; w0 += nwarps * gpw) {
+  __shared__ uint32_t sk[DEDUP == 2 ? kStageEntries : 1];             // gid (kEmpty = free)
+  __shared__ uint32_t sp[DEDUP == 2 ? kStageEntries : 1];             // min flat position
+  __shared__ unsigned long long so[DEDUP == 2 ? kStageEntries : 1];   // table value read
+  __shared__ uint32_t si[DEDUP == 2 ? kStageEntries : 1];             // table index
+  if (DEDUP == 2) {
+    for (uint32_t i = threadIdx.x; i < kStageEntries; i += blockDim.x) {
+      sk[i] = kEmpty;
+      sp[i] = kEmpty;
+    }
+    __syncthreads();
+  }
+  // block-uniform bound for DEDUP == 2 (barriers inside); warp w of block b starts at the
+  // same vertex as in the warp-strided loop
+  const uint32_t wib = threadIdx.x >> 5, wpb = blockDim.x >> 5;
+  for (uint32_t b0 = blockIdx.x * wpb * gpw; DEDUP == 2 ? b0 < n_l : b0 + wib * gpw < n_l;
+       b0 += nwarps * gpw) {
+    const uint32_t w0 = b0 + wib * gpw;
+    (void)warp_global;
     const uint32_t d = w0 + gi;
     const bool active = gi < gpw && d < n_l;
     uint32_t v = 0, deg = 0;
@@ -304,7 +329,38 @@ __global__ void __launch_bounds__(kThreads)
     }
     if (!big && active && s < deg) sel = s;
     uint32_t u = kEmpty, idx = kEmpty;
-    if (DEDUP) {
+    if (DEDUP == 2) {
+      const uint32_t pos = base + d * k + s;
+      uint32_t h = kEmpty;
+      if (sel != kEmpty) {  // stage: find / claim the gid's smem entry, keep the min position
+        u = __ldg(indices + lo + sel);
+        h = hash32(u) & (kStageEntries - 1);
+        for (;;) {
+          const uint32_t prev = atomicCAS(&sk[h], kEmpty, u);
+          if (prev == kEmpty || prev == u) break;
+          h = (h + 1) & (kStageEntries - 1);
+        }
+        atomicMin(&sp[h], pos);
+      }
+      __syncthreads();
+      if (sel != kEmpty && sp[h] == pos) {  // first occurrence in this block: one table access
+        const uint32_t ix = entry_of<HASH>(T, u, st_w);
+        si[h] = ix;
+        so[h] = ix != kEmpty ? vmap_insert(T.e, ix, enc_pos(gen, pos)) : ~0ull;
+      }
+      __syncthreads();
+      if (sel != kEmpty) {
+        idx = si[h];
+        const unsigned long long old = so[h];
+        u = idx != kEmpty ? encode_pick(u, old, enc_pos(gen, pos), base) : kEmpty;
+      }
+      __syncthreads();
+      if (sel != kEmpty) {  // free the entry for the next iteration
+        sk[h] = kEmpty;
+        sp[h] = kEmpty;
+      }
+      __syncthreads();
+    } else if (DEDUP == 1) {
       if (sel != kEmpty) u = __ldg(indices + lo + sel);
       // lanes with the same gid: flat positions grow with the lane, so the lowest lane
       // holds the first occurrence within the warp
@@ -960,12 +1016,15 @@ cudaError_t launch_khop(glb_ctx* c, uint32_t hop, uint32_t k, uint64_t seed, uin
   const Table T = table_of(c);
   cudaError_t e;
 #define GLB_KH_ARGS hop, k, seed, epoch, batch, T, stc, c->st, ip, ix, uq, b.picks, b.pidx, fix
-  if (k <= 32 && c->relabel_dedup)
-    e = c->hash_mode ? launch_pdl_w(c->pin, k_khop<true, true>, grid, kThreads, c->stream, GLB_KH_ARGS)
-                     : launch_pdl_w(c->pin, k_khop<false, true>, grid, kThreads, c->stream, GLB_KH_ARGS);
+  if (k <= 32 && c->relabel_dedup == 2)
+    e = c->hash_mode ? launch_pdl_w(c->pin, k_khop<true, 2>, grid, kThreads, c->stream, GLB_KH_ARGS)
+                     : launch_pdl_w(c->pin, k_khop<false, 2>, grid, kThreads, c->stream, GLB_KH_ARGS);
+  else if (k <= 32 && c->relabel_dedup == 1)
+    e = c->hash_mode ? launch_pdl_w(c->pin, k_khop<true, 1>, grid, kThreads, c->stream, GLB_KH_ARGS)
+                     : launch_pdl_w(c->pin, k_khop<false, 1>, grid, kThreads, c->stream, GLB_KH_ARGS);
   else if (k <= 32)
-    e = c->hash_mode ? launch_pdl_w(c->pin, k_khop<true, false>, grid, kThreads, c->stream, GLB_KH_ARGS)
-                     : launch_pdl_w(c->pin, k_khop<false, false>, grid, kThreads, c->stream, GLB_KH_ARGS);
+    e = c->hash_mode ? launch_pdl_w(c->pin, k_khop<true, 0>, grid, kThreads, c->stream, GLB_KH_ARGS)
+                     : launch_pdl_w(c->pin, k_khop<false, 0>, grid, kThreads, c->stream, GLB_KH_ARGS);
   else
     e = c->hash_mode ? launch_pdl_w(c->pin, k_khop_wide<true>, grid, kThreads, c->stream, GLB_KH_ARGS)
                      : launch_pdl_w(c->pin, k_khop_wide<false>, grid, kThreads, c->stream, GLB_KH_ARGS);

@@ -84,11 +84,24 @@ def test_worked_example_on_gpu():
     assert ctx.permutation(8).tolist() == gold["shuffle"]["epoch1"]
 
 
-@pytest.mark.parametrize("mode", MODES + ["dense_dedup", "hash_dedup"])
+DEDUP_MODES = ["dense_dedup1", "hash_dedup1", "dense_dedup2", "hash_dedup2"]
+
+
+def _dedup(mode, monkeypatch):
+    """'<mode>_dedup<n>': GLB_RELABEL_DEDUP=n (1 warp-level, 2 block smem-staged pre-dedup
+    of picks before the relabel-table insert); returns the relabel mode."""
+    if "_dedup" in mode:
+        mode, n = mode.split("_dedup")
+        monkeypatch.setenv("GLB_RELABEL_DEDUP", n)
+    return mode
+
+
+@pytest.mark.parametrize("mode", MODES + ["dense_dedup1", "hash_dedup1", "dense_dedup2",
+                                          "hash_dedup2"])
 def test_tiny_every_batch_bit_exact(tiny, mode, monkeypatch):
-    if mode.endswith("_dedup"):
-        monkeypatch.setenv("GLB_RELABEL_DEDUP", "1")
-        mode = mode[:-6]
+    if "_dedup" in mode:
+        mode, n = mode.split("_dedup")
+        monkeypatch.setenv("GLB_RELABEL_DEDUP", n)
     g, go = tiny
     sh = g.shape
     ctx = make_ctx(g, fanouts=sh.fanouts, mode=mode)
@@ -115,13 +128,11 @@ def test_host_and_device_seed_paths(tiny):
 
 
 @pytest.mark.parametrize("fanouts", [(25, 10), (15, 10, 5), (3,), (1, 1, 1), (32, 2), (40, 33)])
-@pytest.mark.parametrize("mode", MODES + ["dense_dedup", "hash_dedup"])
+@pytest.mark.parametrize("mode", MODES + DEDUP_MODES)
 def test_fanout_variants_power_law(fanouts, mode, monkeypatch):
-    """*_dedup: picks pre-deduplicated per warp before the relabel-table insert
-    (GLB_RELABEL_DEDUP=1); a small graph with hubs (gamma 2.1), so peers are common."""
-    if mode.endswith("_dedup"):
-        monkeypatch.setenv("GLB_RELABEL_DEDUP", "1")
-        mode = mode[:-6]
+    """*_dedup*: picks pre-deduplicated (warp / block) before the relabel-table insert; a
+    small graph with hubs (gamma 2.1), so duplicate picks within a warp / block are common."""
+    mode = _dedup(mode, monkeypatch)
     g = synth.small_graph(6000, 90000, 2.1, 8, 700, seed=11)
     go = oracle.GraphOracle(g.indptr, g.indices)
     ctx = make_ctx(g, fanouts=fanouts, max_batch=300, mode=mode)
