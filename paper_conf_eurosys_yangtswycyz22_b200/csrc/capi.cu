@@ -343,6 +343,7 @@ glb_status glb_create(int device, glb_ctx** out) {
   if (const char* g = getenv("GLB_GATHER_BULK")) c->gather_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_MISS_BULK")) c->miss_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_WARP")) c->gather_warp = atoi(g) != 0;
+  if (const char* g = getenv("GLB_MISS_BLOCKS")) c->miss_blocks = atoi(g) > 0 ? (uint32_t)atoi(g) : 0u;
   if (const char* g = getenv("GLB_RELABEL_DEDUP")) {  // 1 warp-level, 2 block smem-staged
     const int m = atoi(g);
     c->relabel_dedup = m >= 0 && m <= 2 ? m : 0;

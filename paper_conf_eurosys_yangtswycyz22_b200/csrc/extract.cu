@@ -160,8 +160,11 @@ __global__ void __launch_bounds__(kThreads, 4)
     xcount[1] = nm_all;
   }
   const uint64_t nm = (misses_only & 2) ? 0 : nm_all;
-  // skip bit 0: hits gathered by k_gather_bulk instead; bit 1: misses gathered by it
+  // skip bit 0: hits gathered by k_gather_bulk instead; bit 1: misses gathered by it;
+  // bits 8..: how many blocks take host-miss chunks (0 = all; GLB_MISS_BLOCKS) -- fewer
+  // requests in flight over the link touch fewer host pages at a time
   const uint64_t nh = (misses_only & 1) ? 0 : nh_all;
+  const uint32_t miss_blocks = (uint32_t)misses_only >> 8;
   const uint32_t t = threadIdx.x;
   const uint64_t nch = (nh + R - 1) / R, ncm = (nm + R - 1) / R;  // hit / miss chunks
   const float inv_u = 1.0f / (float)U;
@@ -170,7 +173,9 @@ __global__ void __launch_bounds__(kThreads, 4)
   auto claim = [&]() -> uint64_t {
     if (t == 0) {
       unsigned int g = atomicAdd(&work[0], 1u);
-      if (g >= nch) g = (unsigned int)nch + atomicAdd(&work[1], 1u);
+      if (g >= nch)  // only the first miss_blocks blocks take host chunks (0 = all)
+        g = (miss_blocks && blockIdx.x >= miss_blocks) ? (unsigned int)(nch + ncm)
+                                                       : (unsigned int)nch + atomicAdd(&work[1], 1u);
       s_next = g;
     }
     __syncthreads();
@@ -684,19 +689,19 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   if (vec && shard)
     e = launch_pdl(k_gather<float4, true>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo, c->xcount, work, tab);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(c->miss_blocks << 8), c->xcount, work, tab);
   else if (vec)
     e = launch_pdl(k_gather<float4, false>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo, c->xcount, work, tab);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(c->miss_blocks << 8), c->xcount, work, tab);
   else if (shard)
     e = launch_pdl(k_gather<float, true>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   Sh, So, wb, mo, c->xcount, work, tab);
+                   Sh, So, wb, mo | (int)(c->miss_blocks << 8), c->xcount, work, tab);
   else
     e = launch_pdl(k_gather<float, false>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   Sh, So, wb, mo, c->xcount, work, tab);
+                   Sh, So, wb, mo | (int)(c->miss_blocks << 8), c->xcount, work, tab);
   count_launch(c);
   return e;
 }

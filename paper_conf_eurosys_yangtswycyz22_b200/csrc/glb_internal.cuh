@@ -209,6 +209,7 @@ struct glb_ctx {
   uint32_t gather_bulk_smem = 96 * 1024;  // row-slot bytes per bulk block (GLB_GATHER_BULK_SMEM)
   int miss_bulk = 0;           // GLB_MISS_BULK=1: host misses through cp.async.bulk
   int gather_warp = 0;         // GLB_GATHER_WARP=1: warp-independent gather (k_gather_w)
+  uint32_t miss_blocks = 0;    // GLB_MISS_BLOCKS: blocks of k_gather that take host misses (0 all)
   glb::HostGather* hg = nullptr;  // host-assisted misses (glb_set_host_gather)
   uint32_t hg_permille = 0;       // share of a batch's misses gathered by host threads
   uint32_t hg_threads = 0;

@@ -250,7 +250,9 @@ GATHER_ENV = {"warp": {"GLB_GATHER_WARP": "1"}, "block": {"GLB_GATHER_WARP": "0"
               # host-assisted misses (glb_set_host_gather): 40 % / 90 % of them by host threads
               "host400": {"GLB_HOST_GATHER": "400", "GLB_HOST_GATHER_THREADS": "4"},
               "host900_nobins": {"GLB_HOST_GATHER": "900", "GLB_HOST_GATHER_THREADS": "3",
-                                 "GLB_MISS_BIN_LOG2": "0"}}
+                                 "GLB_MISS_BIN_LOG2": "0"},
+              "missblocks3": {"GLB_MISS_BLOCKS": "3"},  # 3 blocks take every host miss
+              "dedup2_host": {"GLB_RELABEL_DEDUP": "2", "GLB_HOST_GATHER": "500"}}
 
 
 @pytest.mark.parametrize("mode", MODES + ["bulk", "bulkmiss", "bulkboth"] + list(GATHER_ENV))

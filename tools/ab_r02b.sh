@@ -10,3 +10,8 @@ for f in 250 300 350; do for b in 1 2; do for sb in 0 32; do
   V="$V;f${f}_bps${b}_sb${sb}:GLB_HOST_GATHER=$f,GLB_HOST_GATHER_THREADS=8,GLB_GATHER_BPS_PIPE=$b,GLB_HOST_GATHER_SCATTER_BLOCKS=$sb"
 done; done; done
 python tools/ab_env.py --config PA --alpha 0.22 --steps 40 --repeat 1 --variants "$V" > gpurun_out/hg_tune_PA.jsonl 2>&1
+for mb in 0 148 64 32 16 8; do GLB_MISS_BLOCKS=$mb python tools/miss_probe.py --spans 1.0 --bins 21 --reps 3 > gpurun_out/missblocks_probe_$mb.jsonl 2>&1; done
+V="zc:GLB_HOST_GATHER=0"
+for mb in 148 64 32 16; do V="$V;zc_mb$mb:GLB_HOST_GATHER=0,GLB_MISS_BLOCKS=$mb;hg_mb$mb:GLB_HOST_GATHER=250,GLB_HOST_GATHER_THREADS=8,GLB_MISS_BLOCKS=$mb"; done
+python tools/ab_env.py --config PA --alpha 0.22 --steps 40 --repeat 1 --variants "$V" > gpurun_out/missblocks_PA.jsonl 2>&1
+python -m pytest tests/test_gpu_parity.py -m gpu -x -q -k "extract" > gpurun_out/pytest_extract2.log 2>&1; tail -2 gpurun_out/pytest_extract2.log
