@@ -1143,9 +1143,11 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
   const bool hg = hg_active(c);
   uint32_t* dcnt = nullptr;
   if (e == cudaSuccess && hg) e = hg_enqueue(c, (float*)out, misses, &dcnt);
+  c->hg_inflight = hg && dcnt;
   if (e == cudaSuccess)
     e = launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_list, misses,
                       nullptr, dcnt ? dcnt : &c->st->nhit, 0, 0);
+  c->hg_inflight = false;
   if (e == cudaSuccess && hg) e = hg_join(c);
   if (e == cudaSuccess && t1) e = cudaEventRecord(t1, c->stream);
   if (e == cudaSuccess && stats) {

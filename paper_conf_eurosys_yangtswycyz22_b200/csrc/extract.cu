@@ -651,6 +651,10 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
       mo = 2;                      // the LSU gather does the hits only
     }
   }
+  // blocks that take host-miss chunks: GLB_MISS_BLOCKS, else one per SM while the host
+  // takes a share of the misses (measured on PA: fewer zero-copy rows in flight touch
+  // fewer host pages at once -- 5.20-5.23 vs 5.35 ms per step; profiles/r02_missblocks.txt)
+  const uint32_t mb = c->miss_blocks ? c->miss_blocks : (c->hg_inflight ? (uint32_t)c->num_sms : 0u);
   // chunk counters of the launching stream (this ctx's gathers are serial on it; each
   // launch leaves them zeroed for the next)
   unsigned int* work = c->stream == c->xstream ? c->work + 4 : c->work;
@@ -689,19 +693,19 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   if (vec && shard)
     e = launch_pdl(k_gather<float4, true>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(c->miss_blocks << 8), c->xcount, work, tab);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab);
   else if (vec)
     e = launch_pdl(k_gather<float4, false>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(c->miss_blocks << 8), c->xcount, work, tab);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab);
   else if (shard)
     e = launch_pdl(k_gather<float, true>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   Sh, So, wb, mo | (int)(c->miss_blocks << 8), c->xcount, work, tab);
+                   Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab);
   else
     e = launch_pdl(k_gather<float, false>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   Sh, So, wb, mo | (int)(c->miss_blocks << 8), c->xcount, work, tab);
+                   Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab);
   count_launch(c);
   return e;
 }

@@ -213,6 +213,7 @@ struct glb_ctx {
   glb::HostGather* hg = nullptr;  // host-assisted misses (glb_set_host_gather)
   uint32_t hg_permille = 0;       // share of a batch's misses gathered by host threads
   uint32_t hg_threads = 0;
+  bool hg_inflight = false;       // the extract being enqueued has a host-assisted part
   uint64_t C = 0;
   // NEXT-3 peer-sharded cache: global rank i < C is owned by shard i % W at row i / W;
   // shard_base[r] = device pointer (valid in this process) of shard r's rows.
