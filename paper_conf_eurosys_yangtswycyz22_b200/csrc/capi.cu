@@ -13,12 +13,21 @@
 #include <thread>
 
 #include "glb_internal.cuh"
+#include <nvtx3/nvToolsExt.h>
 
 using namespace glb;
 
 namespace {
 
 thread_local std::string g_create_err;
+
+// NVTX range per API call (SURVEY §5 tracing): a profiler (nsys / ncu --nvtx) sees each
+// stage's enqueue -- sample, presample, load_cache, extract -- and the kernels it launched.
+// Header-only NVTX v3: no cost when no tool is attached.
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
 
 glb_status set_err(glb_ctx* c, glb_status s, const char* fmt, ...) {
   char buf[512];
@@ -425,6 +434,7 @@ glb_status glb_sync(glb_ctx* c) {
 
 glb_status glb_load_graph(glb_ctx* c, uint64_t V, uint64_t E, const uint64_t* indptr,
                           const uint32_t* indices, const void* features, uint32_t D) {
+  NvtxRange nvtx_("glb_load_graph");
   ENTER(c);
   if (V == 0 || V >= 0x80000000ull) return set_err(c, GLB_EINVAL, "V=%llu out of range [1, 2^31)", (unsigned long long)V);
   if (!indptr || (E && !indices)) return set_err(c, GLB_EINVAL, "null CSR");
@@ -693,6 +703,7 @@ glb_status glb_sample_result(glb_ctx* c, glb_blocks* out) {
 
 glb_status glb_sample(glb_ctx* c, const uint32_t* seeds, uint32_t n0, const uint32_t* fanouts,
                       uint32_t L, uint64_t seed, uint32_t epoch, uint32_t batch, glb_blocks* out) {
+  NvtxRange nvtx_("glb_sample");
   ENTER(c);
   if (!c->V) return set_err(c, GLB_ESTATE, "sample before load_graph");
   if (!c->sampler_set) return set_err(c, GLB_ESTATE, "sample before set_sampler");
@@ -722,6 +733,7 @@ glb_status glb_sample(glb_ctx* c, const uint32_t* seeds, uint32_t n0, const uint
 
 glb_status glb_sample_async(glb_ctx* c, const uint32_t* seeds, uint32_t n0, uint64_t seed,
                             uint32_t epoch, uint32_t batch) {
+  NvtxRange nvtx_("glb_sample_async");
   ENTER(c);
   if (!c->V || !c->sampler_set) return set_err(c, GLB_ESTATE, "sample before load_graph/set_sampler");
   if (n0 && !seeds) return set_err(c, GLB_EINVAL, "null seeds");
@@ -746,6 +758,7 @@ glb_status glb_extract_counts_device_ptr(glb_ctx* c, void** out) {
 }
 
 glb_status glb_sample_batch(glb_ctx* c, uint32_t epoch, uint32_t b) {
+  NvtxRange nvtx_("glb_sample_batch");
   ENTER(c);
   if (!c->V || !c->sampler_set || !c->train_set) return set_err(c, GLB_ESTATE, "sample_batch needs graph, sampler, train set");
   const uint64_t nb = (c->n_train + c->batch_size - 1) / c->batch_size;
@@ -776,6 +789,7 @@ glb_status glb_reset_counts(glb_ctx* c, int which) {
 }
 
 glb_status glb_presample(glb_ctx* c, uint32_t K, uint32_t rank, uint32_t world) {
+  NvtxRange nvtx_("glb_presample");
   ENTER(c);
   if (!c->V || !c->sampler_set || !c->train_set) return set_err(c, GLB_ESTATE, "presample needs graph, sampler, train set");
   if (world == 0 || rank >= world) return set_err(c, GLB_EINVAL, "bad rank/world");
@@ -879,6 +893,7 @@ static glb_status build_cache_impl(glb_ctx* c, uint64_t C, const uint32_t* hotne
 }
 
 glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
+  NvtxRange nvtx_("glb_build_cache");
   ENTER(c);
   if (!c->V) return set_err(c, GLB_ESTATE, "build_cache before load_graph");
   if (!(alpha >= 0.0 && alpha <= 1.0)) return set_err(c, GLB_EINVAL, "alpha %g not in [0,1]", alpha);
@@ -889,6 +904,7 @@ glb_status glb_build_cache(glb_ctx* c, double alpha, const uint32_t* hotness) {
 
 glb_status glb_build_cache_sharded(glb_ctx* c, double alpha, const uint32_t* hotness,
                                    uint32_t rank, uint32_t world) {
+  NvtxRange nvtx_("glb_build_cache_sharded");
   ENTER(c);
   if (!c->V) return set_err(c, GLB_ESTATE, "build_cache before load_graph");
   if (!(alpha >= 0.0 && alpha <= 1.0)) return set_err(c, GLB_EINVAL, "alpha %g not in [0,1]", alpha);
@@ -1060,6 +1076,7 @@ glb_status glb_hit_stats_get(glb_ctx* c, glb_hit_stats* out) {
 
 glb_status glb_extract(glb_ctx* c, const uint32_t* vertices, uint64_t n, void* out,
                        glb_extract_stats* stats) {
+  NvtxRange nvtx_("glb_extract");
   ENTER(c);
   if (!c->V || !c->features_mapped) return set_err(c, GLB_ESTATE, "extract needs a graph with features");
   if (!shards_ready(c)) return set_err(c, GLB_ESTATE, "peer cache shards not all attached");
@@ -1100,6 +1117,7 @@ glb_status glb_extract(glb_ctx* c, const uint32_t* vertices, uint64_t n, void* o
 }
 
 glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
+  NvtxRange nvtx_("glb_extract_sample");
   ENTER(c);
   if (!c->have_sample) return set_err(c, GLB_ESTATE, "extract_sample without a current sample");
   if (!c->features_mapped) return set_err(c, GLB_ESTATE, "graph loaded without features");
