@@ -1073,6 +1073,7 @@ def main(argv=None):
                "unit": "seeds/s", "ms_per_step": r["ms_per_step"], "runs": r["runs"],
                "runs_range": r["runs_range"], "roofline": r["roofline"],
                "path_roofline": r["path_roofline"], "e2e_value": r["e2e"]["value"],
+               "host_enqueue_ms_per_step": r["host_enqueue_ms_timed_region"] / args.steps,
                "gpu_launches": r["gpu_launches"], "clocks": r["clocks"]}
     if rank == 0:
         line = {
