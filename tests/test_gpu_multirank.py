@@ -105,3 +105,21 @@ def test_bench_self_launch_two_ranks():
     assert d["n_gpus"] == 2 and d["value"] > 0 and len(d["runs"]) == 2
     assert d["host_inputs"].startswith("node-shared")
     assert d["config"]["parallelism"] == "dp2"
+
+
+def test_bench_ns_sweep_three_ranks():
+    """Config 5's Ns sweep (Fig 15 analog): the adaptive factored split, then every
+    Ns in 1..N-1 as its own N-rank run (3 ranks sharing cuda:0 over gloo + CUDA IPC)."""
+    cmd = [sys.executable, "bench.py", "--gpus", "3", "--steps", "6", "--warmup", "3",
+           "--config", "tiny", "--backend", "gloo", "--mode", "factored", "--ns-sweep",
+           "--no-sweep", "--no-cpu-baseline", "--no-pr-alpha1", "--alpha", "1.0"]
+    env = {k: v for k, v in os.environ.items()
+           if k not in ("WORLD_SIZE", "RANK", "LOCAL_RANK", "LOCAL_WORLD_SIZE")}
+    r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=900, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout[-2000:]
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 3 and d["config"]["mode"] == "factored"
+    sw = d["ns_sweep"]
+    assert [x["samplers"] for x in sw] == [1, 2] and all(x["value"] and x["value"] > 0 for x in sw)
