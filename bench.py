@@ -193,6 +193,16 @@ def gpu_info(index):
         phys = int(vis.split(",")[index]) if vis and vis.split(",")[0].isdigit() else index
         h = nv.nvmlDeviceGetHandleByIndex(phys)
         d = {"name": nv.nvmlDeviceGetName(h), "driver": nv.nvmlSystemGetDriverVersion()}
+        try:
+            v = nv.nvmlSystemGetCudaDriverVersion()
+            d["driver_cuda"] = f"{v // 1000}.{v % 1000 // 10}"
+        except Exception:
+            pass
+        try:
+            import torch
+            d["torch_cuda_runtime"] = torch.version.cuda
+        except Exception:
+            pass
         for k, f in (("ecc_mode", lambda: nv.nvmlDeviceGetCurrentEccMode(h)),
                      ("sm_max_mhz", lambda: nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)),
                      ("mem_max_mhz", lambda: nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_MEM)),

@@ -133,8 +133,11 @@ __device__ __forceinline__ void st_row(T* p, T v) { __stcs(p, v); }
 // by shard i % W at row i / W; tab.base[w] is shard w's rows (this GPU's own HBM or
 // a peer's, mapped over NVLink).  The owner is resolved once per entry when the
 // entry is staged, so the per-vector loop only indexes the shard table.
+#ifndef GLB_GATHER_MINB  // min resident gather blocks per SM (register cap; A/B builds)
+#define GLB_GATHER_MINB 4
+#endif
 template <typename T, bool SHARD>
-__global__ void __launch_bounds__(kThreads, 4)
+__global__ void __launch_bounds__(kThreads, GLB_GATHER_MINB)
     k_gather(T* __restrict__ out, const T* __restrict__ src_hit, const T* __restrict__ src_miss,
              const uint2* __restrict__ hit_list, const uint2* __restrict__ miss_list,
              const uint32_t* __restrict__ fill_src, const uint32_t* __restrict__ dev_counts,
