@@ -178,6 +178,20 @@ def test_errors(mode):
     with pytest.raises(glb.GlbError) as e:
         ctx.build_cache(1.5)
     assert e.value.code == glb.EINVAL
+    # T is a set (L305; reading Q6): a duplicate training id is rejected up front
+    with pytest.raises(glb.GlbError) as e:
+        ctx.set_train_set(np.array([3, 7, 3], np.uint32), 2, 1)
+    assert e.value.code == glb.EINVAL
+    # device-side errors are sticky: a bad asynchronous batch followed by a good one still
+    # reports at the next sync (an earlier batch's error is not lost)
+    ctx.set_pipeline(2)
+    ctx.sample_async(torch.tensor([4, 5, 4], dtype=torch.int32).pin_memory(), seed=1)
+    ctx.sample_async(torch.tensor([6, 8], dtype=torch.int32).pin_memory(), seed=1)
+    with pytest.raises(glb.GlbError) as e:
+        ctx.sync()
+    assert e.value.code == glb.EINVAL
+    ctx.sync()  # reported once, then cleared
+    ctx.set_pipeline(1)
     # the ctx still works after errors
     go = oracle.GraphOracle(g.indptr, g.indices)
     assert_same_sample(ctx.sample(np.array([1, 2], np.uint32), seed=3),
