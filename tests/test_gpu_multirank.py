@@ -123,3 +123,52 @@ def test_bench_ns_sweep_three_ranks():
     assert d["n_gpus"] == 3 and d["config"]["mode"] == "factored"
     sw = d["ns_sweep"]
     assert [x["samplers"] for x in sw] == [1, 2] and all(x["value"] and x["value"] > 0 for x in sw)
+
+
+def _shm_parity_worker(rank, world, port, out):
+    import torch.distributed as dist
+
+    import oracle
+    import paper_conf_eurosys_yangtswycyz22_b200 as glb
+    from synth import shm
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    store = dist.distributed_c10d._get_default_store()
+    g = shm.make_graph_shared("tiny", rank, world, store).graph
+    sh = g.shape
+    ctx = glb.Context(0)
+    ctx.load_graph(g.indptr, g.indices, g.features)  # every rank registers the SAME pages
+    ctx.set_sampler("khop", fanouts=sh.fanouts, max_batch=sh.batch)
+    ctx.set_train_set(g.train, sh.batch, g.seed)
+    ctx.presample(1, rank, world)
+    c = ctx.counts_tensor(glb.COUNT_PRESAMPLE).cpu()
+    import paper_conf_eurosys_yangtswycyz22_b200.parallel as par
+    par.allreduce_counts(c)
+    ctx.counts_tensor(glb.COUNT_PRESAMPLE).copy_(c.cuda())
+    ctx.build_cache(0.2)
+    go = oracle.GraphOracle(g.indptr, g.indices, g.features)
+    ob = oracle.epoch_batches(g.train, sh.batch, g.seed, 1)
+    ok = True
+    for b in range(rank, len(ob), world):  # DP: this rank's batches
+        ctx.sample_batch(1, b)
+        s = ctx.sample_result()
+        o = torch.empty((s.sizes[-1], sh.D), dtype=torch.float32, device="cuda")
+        ctx.extract_sample(o, stats=True)
+        exp = go.sample_khop(ob[b], sh.fanouts, g.seed, 1, b)
+        ok &= np.array_equal(s.uniq.cpu().numpy().view(np.uint32), exp.uniq)
+        ok &= np.array_equal(o.cpu().numpy().view(np.uint32), go.extract(exp.uniq).view(np.uint32))
+    with open(os.path.join(out, f"r{rank}"), "w") as f:
+        f.write(str(int(ok)))
+    ctx.close()
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_node_shared_inputs_registered_by_every_rank(tmp_path):
+    """Node-shared host inputs (synth/shm.py) under DP: both ranks register the same pinned
+    pages for their GPU (here both cuda:0) and every batch's samples and extracted bytes
+    equal the oracle's; the PreSC counts are summed over the ranks' shares."""
+    import torch.multiprocessing as mp
+    mp.spawn(_shm_parity_worker, args=(2, free_port(), str(tmp_path)), nprocs=2, join=True)
+    assert open(tmp_path / "r0").read() == "1" and open(tmp_path / "r1").read() == "1"
