@@ -784,6 +784,15 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
         ctx.set_timing(False)
         ctx.set_pipeline(2)
         ims = i0.elapsed_time(i1)
+        # the sampling half alone (a1-a5 of the same batches, no extract)
+        torch.cuda.synchronize()
+        i0.record(stream)
+        for i in iso_steps:
+            e, b = batch_of(i)
+            ctx.sample_batch(e, b)
+        i1.record(stream)
+        torch.cuda.synchronize()
+        sms = i0.elapsed_time(i1) / len(iso_steps)
         a_hbm = statistics.mean(bb / (t * 1e-3) for bb, t in zip(hbm_bytes, xi)) / 1e9
         a_link = statistics.mean(bb / (t * 1e-3) for bb, t in zip(link_bytes, xi)) / 1e9
         iso = {"pipeline_depth": 1, "steps": len(iso_steps),
@@ -791,7 +800,9 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
                "frac": (a_link / link_peak) if host_bound else (a_hbm / hbm_peak),
                "hbm_achieved": a_hbm, "hbm_frac": a_hbm / hbm_peak,
                "extract_ms_per_step": statistics.mean(xi),
-               "ms_per_step": ims / len(iso_steps), "seeds_per_s": world * sd / (ims / 1e3)}
+               "ms_per_step": ims / len(iso_steps), "seeds_per_s": world * sd / (ims / 1e3),
+               "sampling_ms_per_step": sms,
+               "sampling_ms_per_step_is": "the same batches sampled alone (no extract), depth 1"}
     traffic = None
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
