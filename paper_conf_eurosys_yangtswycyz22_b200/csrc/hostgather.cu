@@ -23,6 +23,8 @@
 #include <cuda_runtime.h>
 
 #include <atomic>
+#include <chrono>
+#include <cstdio>
 #include <cstdlib>
 #include <condition_variable>
 #include <cstring>
@@ -195,6 +197,9 @@ struct HostGather {
   uint8_t* stage_dev[kSlots] = {};   // device alias of stage
   HgJob job[kJobRing];
   uint64_t njobs = 0;
+  // GLB_HG_STATS=1: host-function wall time, printed by hg_free (A/B instrumentation)
+  bool stats = false;
+  std::atomic<uint64_t> st_ns{0}, st_rows{0}, st_calls{0};
 };
 
 namespace {
@@ -223,7 +228,14 @@ void hg_gather(const HgJob* j);
 
 void CUDART_CB hg_host_fn(void* p) {
   HgJob* j = static_cast<HgJob*>(p);
+  HostGather* h = j->c->hg;
+  const auto t0 = std::chrono::steady_clock::now();
   hg_gather(j);
+  if (h->stats) {
+    h->st_ns += (uint64_t)std::chrono::duration_cast<std::chrono::nanoseconds>(
+                    std::chrono::steady_clock::now() - t0).count();
+    h->st_calls += 1;
+  }
   j->done.store(1, std::memory_order_release);
 }
 
@@ -240,6 +252,7 @@ void hg_gather(const HgJob* j) {
   uint8_t* stage = h->stage[j->slot];
   const uint2* ent = h->ent[j->slot];
   const uint32_t ntask = (uint32_t)((hi - lo + kTaskRows - 1) / kTaskRows);
+  if (h->stats) h->st_rows += hi - lo;
   std::function<void(uint32_t)> fn = [&](uint32_t t) {
     const uint64_t a = lo + (uint64_t)t * kTaskRows;
     const uint64_t b = a + kTaskRows < hi ? a + kTaskRows : hi;
@@ -263,6 +276,12 @@ void hg_free(glb_ctx* c) {
   if (!h) return;
   for (int i = 0; i < 2; ++i)
     if (h->cs[i]) cudaStreamSynchronize(h->cs[i]);
+  if (h->stats && h->st_calls)
+    fprintf(stderr, "glb host gather: %llu host functions, %.3f ms total, %.1f us mean, "
+            "%llu rows, %.2f GB/s while gathering\n",
+            (unsigned long long)h->st_calls.load(), h->st_ns.load() / 1e6,
+            h->st_ns.load() / 1e3 / h->st_calls.load(), (unsigned long long)h->st_rows.load(),
+            h->st_rows.load() * 4.0 * c->D / (h->st_ns.load() ? h->st_ns.load() : 1));
   delete h->pool;
   hg_free_bufs(h);
   for (int i = 0; i < 2; ++i) {
@@ -283,6 +302,7 @@ cudaError_t hg_configure(glb_ctx* c, uint32_t threads) {
     if (!h) return cudaErrorMemoryAllocation;
     c->hg = h;
     if (const char* g = getenv("GLB_HOST_GATHER_DMA")) h->dma = atoi(g) != 0;
+    if (const char* g = getenv("GLB_HG_STATS")) h->stats = atoi(g) != 0;
     if (const char* g = getenv("GLB_HOST_GATHER_SCATTER_BLOCKS")) h->sblocks = atoi(g) > 0 ? atoi(g) : 0;
     if (const char* g = getenv("GLB_HOST_GATHER_CHUNKS")) {
       const int n = atoi(g);
