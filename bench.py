@@ -103,7 +103,8 @@ def parse(argv=None):
                         "(glb_set_host_gather): a fraction, or 'auto' = 0.25 when a feature "
                         "row is <= 512 B and alpha < 1 (measured: 512-B zero-copy rows are "
                         "bound by address translation, 1-KB rows are not; DESIGN.md §10)")
-    p.add_argument("--host-gather-threads", type=int, default=8)
+    p.add_argument("--host-gather-threads", type=int, default=0,
+                   help="host threads per rank (0: min(8, usable cores / local ranks - 1))")
     p.add_argument("--pipeline", type=int, default=2, choices=[1, 2],
                    help="2: extract of batch b overlaps sampling of batch b+1 (two streams)")
     a = p.parse_args(argv)
@@ -663,7 +664,10 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
     hg = args.host_gather
     hg = (0.25 if 4 * sh.D <= 512 and alpha < 1.0 else 0.0) if hg == "auto" else float(hg)
     if hg > 0:
-        ctx.set_host_gather(hg, threads=args.host_gather_threads)
+        nt = args.host_gather_threads
+        if nt <= 0:  # share the node's cores between the local ranks
+            nt = min(8, max(2, host_info()["nproc"] // max(1, local_world) - 1))
+        ctx.set_host_gather(hg, threads=nt)
     ctx_cache_rows = ctx.cache_size
     ub = sh.batch
     for k in sh.fanouts:
@@ -1081,6 +1085,8 @@ def main(argv=None):
     torch.cuda.set_device(dev)
     stream = torch.cuda.current_stream(dev)
     sh = synth.SHAPES[args.config]
+    if world > 1:  # every rank measures its link while the others do (as in the run)
+        dist.barrier()
     link_peak = hostlink_peak(dev)
     res = run_workload(args, sh, args.alpha, world, rank, local, local_world, dev, stream, True,
                        link_peak)
