@@ -102,6 +102,16 @@ __device__ __forceinline__ float4 ld_row<float4>(const float4* p, uint64_t pol) 
   asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0,%1,%2,%3}, [%4], %5;"
                : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pol));
   return v;
+#elif GLB_GATHER_LD == 3  // explicit 64-byte L2 prefetch size (A/B: DRAM over-fetch per row)
+  float4 v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::64B.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+  return v;
+#elif GLB_GATHER_LD == 4  // 256-byte L2 prefetch size
+  float4 v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::256B.v4.f32 {%0,%1,%2,%3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+  return v;
 #elif GLB_GATHER_LD == 1
   return __ldcs(p);
 #else
@@ -114,6 +124,14 @@ __device__ __forceinline__ float ld_row<float>(const float* p, uint64_t pol) {
   float v;
   asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;"
                : "=f"(v) : "l"(p), "l"(pol));
+  return v;
+#elif GLB_GATHER_LD == 3
+  float v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::64B.f32 %0, [%1];" : "=f"(v) : "l"(p));
+  return v;
+#elif GLB_GATHER_LD == 4
+  float v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::256B.f32 %0, [%1];" : "=f"(v) : "l"(p));
   return v;
 #elif GLB_GATHER_LD == 1
   return __ldcs(p);

@@ -68,6 +68,21 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
   return m;
 }
 
+// Random 4-byte reads of the CSR (GLB_SAMPLE_LD=1: with an explicit 64-byte L2 prefetch size,
+// A/B builds -- the sampler touches one 4-byte word per 32-byte sector it pulls in)
+#ifndef GLB_SAMPLE_LD
+#define GLB_SAMPLE_LD 0
+#endif
+__device__ __forceinline__ uint32_t ld_csr(const uint32_t* p) {
+#if GLB_SAMPLE_LD == 1
+  uint32_t v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::64B.u32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+#else
+  return __ldg(p);
+#endif
+}
+
 // Insert one pick into the relabel table: keep the smallest position of this
 // generation.  Values only decrease over time, so a (possibly stale) read that
 // is already <= e proves the atomic would be a no-op.
@@ -333,7 +348,7 @@ __global__ void __launch_bounds__(kThreads)
       const uint32_t pos = base + d * k + s;
       uint32_t h = kEmpty;
       if (sel != kEmpty) {  // stage: find / claim the gid's smem entry, keep the min position
-        u = __ldg(indices + lo + sel);
+        u = ld_csr(indices + lo + sel);
         h = hash32(u) & (kStageEntries - 1);
         for (;;) {
           const uint32_t prev = atomicCAS(&sk[h], kEmpty, u);
@@ -361,7 +376,7 @@ __global__ void __launch_bounds__(kThreads)
       }
       __syncthreads();
     } else if (DEDUP == 1) {
-      if (sel != kEmpty) u = __ldg(indices + lo + sel);
+      if (sel != kEmpty) u = ld_csr(indices + lo + sel);
       // lanes with the same gid: flat positions grow with the lane, so the lowest lane
       // holds the first occurrence within the warp
       const unsigned long long key =
@@ -378,7 +393,7 @@ __global__ void __launch_bounds__(kThreads)
       if (sel != kEmpty)
         u = idx != kEmpty ? encode_pick(u, old, enc_pos(gen, base + d * k + s), base) : kEmpty;
     } else if (sel != kEmpty) {
-      u = __ldg(indices + lo + sel);
+      u = ld_csr(indices + lo + sel);
       idx = entry_of<HASH>(T, u, st_w);
       if (idx != kEmpty) {
         const unsigned long long e = enc_pos(gen, base + d * k + s);
@@ -441,7 +456,7 @@ __global__ void __launch_bounds__(kThreads)
           if (__ldg(wprefix + m) > target) b = m;
           else a = m + 1;
         }
-        u = __ldg(indices + a);
+        u = ld_csr(indices + a);
         idx = entry_of<HASH>(T, u, st_w);
         if (idx != kEmpty) {
           const unsigned long long e = enc_pos(gen, base + d * k + s);
@@ -497,7 +512,7 @@ __global__ void __launch_bounds__(kThreads)
       uint32_t sel = kEmpty;
       if (deg > k) sel = ch[s];
       else if (s < deg) sel = s;
-      uint32_t u = sel != kEmpty ? __ldg(indices + lo + sel) : kEmpty, idx = kEmpty;
+      uint32_t u = sel != kEmpty ? ld_csr(indices + lo + sel) : kEmpty, idx = kEmpty;
       if (u != kEmpty) {
         idx = entry_of<HASH>(T, u, st_w);
         if (idx != kEmpty) {
@@ -561,7 +576,7 @@ __global__ void __launch_bounds__(kThreads, GLB_RWALK_MINB)
             const uint32_t deg = (uint32_t)(indptr[cur + 1] - b);
             if (deg == 0) break;
             const uint64_t r = draw64(seed, v, (w << 8) | ((uint32_t)t >> 1), batch, c3, t & 1);
-            cur = __ldg(indices + b + bounded(r, deg));
+            cur = ld_csr(indices + b + bounded(r, deg));
             if (cur != v) vis[t] = cur;
           }
         }
