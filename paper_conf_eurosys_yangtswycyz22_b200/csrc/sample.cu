@@ -68,10 +68,12 @@ __device__ __forceinline__ uint32_t lanemask_lt() {
   return m;
 }
 
-// Random 4-byte reads of the CSR (GLB_SAMPLE_LD=1: with an explicit 64-byte L2 prefetch size,
-// A/B builds -- the sampler touches one 4-byte word per 32-byte sector it pulls in)
+// Random 4-byte reads of the CSR: a non-coherent load that does not allocate in L1 and asks L2
+// for a 64-byte fill (the sampler touches one 4-byte word of each sector it pulls in).
+// Measured against the plain __ldg (GLB_SAMPLE_LD=0 A/B build, profiles/r02_ldhint_ab.txt):
+// PR 206.7 vs 208.0, UK 429.8 vs 432.9, TW 590.3 vs 597.5 us/step at alpha = 1.
 #ifndef GLB_SAMPLE_LD
-#define GLB_SAMPLE_LD 0
+#define GLB_SAMPLE_LD 1
 #endif
 __device__ __forceinline__ uint32_t ld_csr(const uint32_t* p) {
 #if GLB_SAMPLE_LD == 1

@@ -1,5 +1,9 @@
 """Small end-to-end run (tiny config, both relabel modes, k-hop + random walk, PreSC,
-cache, extract with hits and misses, pipeline depth 2) for compute-sanitizer."""
+cache, extract with hits and misses, pipeline depth 2) for compute-sanitizer, under each
+library variant (environment knobs read at glb_create): default, warp / block-staged
+relabel pre-dedup, host-assisted misses, one miss bin per row (device scan), the
+warp-independent gather, a capped miss-block count."""
+import os
 import sys
 
 import numpy as np
@@ -13,7 +17,14 @@ import synth  # noqa: E402
 g = synth.make_graph("tiny")
 sh = g.shape
 go = oracle.GraphOracle(g.indptr, g.indices, g.features)
-for mode in ["dense", "hash"]:
+VARIANTS = [{}, {"GLB_RELABEL_DEDUP": "1"}, {"GLB_RELABEL_DEDUP": "2"},
+            {"GLB_HOST_GATHER": "400", "GLB_HOST_GATHER_THREADS": "2"},
+            {"GLB_MISS_BIN_LOG2": "7", "GLB_GATHER_WARP": "1"}, {"GLB_MISS_BLOCKS": "3"}]
+KEYS = {k for v in VARIANTS for k in v}
+for var, mode in [(v, m) for v in VARIANTS for m in ["dense", "hash"]]:
+    for k in KEYS:
+        os.environ.pop(k, None)
+    os.environ.update(var)
     ctx = glb.Context(0)
     ctx.load_graph(g.indptr, g.indices, g.features)
     ctx.set_relabel_mode(mode)
