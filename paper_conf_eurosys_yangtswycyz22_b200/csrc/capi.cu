@@ -352,6 +352,7 @@ glb_status glb_create(int device, glb_ctx** out) {
   if (const char* g = getenv("GLB_GATHER_BULK")) c->gather_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_MISS_BULK")) c->miss_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_WARP")) c->gather_warp = atoi(g) != 0;
+  if (const char* g = getenv("GLB_GATHER_LIDORDER")) c->gather_lidorder = atoi(g) != 0;
   if (const char* g = getenv("GLB_MISS_BLOCKS")) c->miss_blocks = atoi(g) > 0 ? (uint32_t)atoi(g) : 0u;
   if (const char* g = getenv("GLB_RELABEL_DEDUP")) {  // 1 warp-level, 2 block smem-staged
     const int m = atoi(g);
@@ -1164,7 +1165,9 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
   c->hg_inflight = hg && dcnt;
   if (e == cudaSuccess)
     e = launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_list, misses,
-                      nullptr, dcnt ? dcnt : &c->st->nhit, 0, 0);
+                      nullptr, dcnt ? dcnt : &c->st->nhit, 0, 0,
+                      c->gather_lidorder && !c->gather_warp ? c->sb.lidslot : nullptr,
+                      &c->st->n[c->last_L]);
   c->hg_inflight = false;
   if (e == cudaSuccess && hg) e = hg_join(c);
   if (e == cudaSuccess && t1) e = cudaEventRecord(t1, c->stream);

@@ -161,9 +161,13 @@ __global__ void __launch_bounds__(kThreads, GLB_GATHER_MINB)
              const uint32_t* __restrict__ fill_src, const uint32_t* __restrict__ dev_counts,
              uint64_t nh_host, uint64_t nm_host, uint32_t U, uint32_t R, uint32_t Sh, uint32_t So,
              int st_wb, int misses_only, unsigned long long* xcount, unsigned int* work,
-             ShardTab tab) {
+             ShardTab tab, const int32_t* __restrict__ lidslot, const uint32_t* __restrict__ nl_dev) {
   // U: T-units per row moved; Sh: row stride of src_hit (the HBM cache may pad its rows);
   // So: row stride of out; host rows (src_miss) are dense (stride U)
+  // lidslot (GLB_GATHER_LIDORDER): the hit phase walks lids 0..n_L-1 in order (nl_dev = n_L)
+  // and takes the cached ones (lidslot[lid] >= 0) instead of the hit list, so a chunk writes
+  // consecutive output rows: row boundaries that share a 32-byte sector are written by the
+  // same block at nearly the same time
   pdl_enter();
   // staged work entry: source row address and destination element offset, resolved once
   // per row so the per-vector loop is one LDS.128 + two adds
@@ -184,7 +188,7 @@ __global__ void __launch_bounds__(kThreads, GLB_GATHER_MINB)
   // skip bit 0: hits gathered by k_gather_bulk instead; bit 1: misses gathered by it;
   // bits 8..: how many blocks take host-miss chunks (0 = all; GLB_MISS_BLOCKS) -- fewer
   // requests in flight over the link touch fewer host pages at a time
-  const uint64_t nh = (misses_only & 1) ? 0 : nh_all;
+  const uint64_t nh = (misses_only & 1) ? 0 : (lidslot ? (uint64_t)*nl_dev : nh_all);
   const uint32_t miss_blocks = (uint32_t)misses_only >> 8;
   const uint32_t t = threadIdx.x;
   const uint64_t nch = (nh + R - 1) / R, ncm = (nm + R - 1) / R;  // hit / miss chunks
@@ -211,6 +215,10 @@ __global__ void __launch_bounds__(kThreads, GLB_GATHER_MINB)
     const bool miss = g >= nch;
     const uint64_t r = (miss ? g - nch : g) * R + t;
     if (r >= (miss ? nm : nh)) return make_uint2(0u, 0u);
+    if (!miss && lidslot) {  // lid order: a miss lid is a hole in this chunk
+      const int32_t sl = __ldg(lidslot + r);
+      return make_uint2((uint32_t)r, sl >= 0 ? (uint32_t)sl : kEmpty);
+    }
     if (!miss) return __ldg(hit_list + r);
     return fill_src ? make_uint2((uint32_t)r, __ldg(fill_src + r)) : __ldg(miss_list + r);
   };
@@ -219,6 +227,8 @@ __global__ void __launch_bounds__(kThreads, GLB_GATHER_MINB)
     RowEnt re;
     if (g >= nch) {
       re.src = src_miss + (uint64_t)h.y * U;
+    } else if (h.y == kEmpty) {  // lid order: not cached (the miss phase gathers it)
+      re.src = nullptr;
     } else if (SHARD) {
       const uint32_t w = h.y % tab.W;
       re.src = (const T*)tab.base[w] + (uint64_t)(h.y / tab.W) * Sh;
@@ -243,6 +253,7 @@ __global__ void __launch_bounds__(kThreads, GLB_GATHER_MINB)
     for (uint32_t base = 0; base < total; base += kChunkUnits) {
       T x[kVecPerThread];
       unsigned long long dst[kVecPerThread];
+      uint32_t live = 0;  // vectors of this thread that move a row (holes: lid order)
 #pragma unroll
       for (int q = 0; q < kVecPerThread; ++q) {
         const uint32_t v = base + q * kThreads + t;
@@ -250,14 +261,16 @@ __global__ void __launch_bounds__(kThreads, GLB_GATHER_MINB)
           uint32_t row = (uint32_t)(((float)v + 0.5f) * inv_u);  // exact for v < 2^20
           const uint32_t col = v - row * U;
           const RowEnt en = ent[buf][row];
-          x[q] = ld_row(en.src + col, pol);
-          dst[q] = en.dst + col;
+          if (en.src) {
+            x[q] = ld_row(en.src + col, pol);
+            dst[q] = en.dst + col;
+            live |= 1u << q;
+          }
         }
       }
 #pragma unroll
       for (int q = 0; q < kVecPerThread; ++q) {
-        const uint32_t v = base + q * kThreads + t;
-        if (v < total) {
+        if (live >> q & 1u) {
           if (st_wb) out[dst[q]] = x[q];
           else st_row(out + dst[q], x[q]);
         }
@@ -590,7 +603,8 @@ cudaError_t launch_mark_to(glb_ctx* c, const uint32_t* vertices, uint64_t n, con
 
 cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const float* src_miss,
                           const uint2* hit_list, const uint2* miss_list, const uint32_t* fill_src,
-                          const uint32_t* dev_counts, uint64_t nhit_host, uint64_t nmiss_host) {
+                          const uint32_t* dev_counts, uint64_t nhit_host, uint64_t nmiss_host,
+                          const int32_t* lidslot, const uint32_t* nl_dev) {
   const uint32_t D = c->D;
   const bool vec = (D % 4) == 0;
   const uint32_t U = vec ? D / 4 : D;
@@ -688,7 +702,7 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   cudaError_t e;
   if (shard && !mo && (e = cudaMemsetAsync(c->xcount + 2, 0, sizeof(unsigned long long), c->stream)) != cudaSuccess)
     return e;
-  if (c->gather_warp) {  // warp-independent gather (no block barriers)
+  if (c->gather_warp) {  // warp-independent gather (no block barriers; hit list order)
     uint32_t Rw = (uint32_t)(32 * kVecPerThread) / U;
     Rw = Rw < 1 ? 1 : Rw > 32 ? 32 : Rw;
     const int gridw = c->num_sms * (c->stream == c->xstream ? c->gather_bps_pipe : c->gather_bps);
@@ -714,19 +728,19 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   if (vec && shard)
     e = launch_pdl(k_gather<float4, true>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
   else if (vec)
     e = launch_pdl(k_gather<float4, false>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
   else if (shard)
     e = launch_pdl(k_gather<float, true>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab);
+                   Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
   else
     e = launch_pdl(k_gather<float, false>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab);
+                   Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
   count_launch(c);
   return e;
 }

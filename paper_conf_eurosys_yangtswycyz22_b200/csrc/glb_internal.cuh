@@ -210,6 +210,7 @@ struct glb_ctx {
   int miss_bulk = 0;           // GLB_MISS_BULK=1: host misses through cp.async.bulk
   int gather_warp = 0;         // GLB_GATHER_WARP=1: warp-independent gather (k_gather_w)
   uint32_t miss_blocks = 0;    // GLB_MISS_BLOCKS: blocks of k_gather that take host misses (0 all)
+  int gather_lidorder = 0;     // GLB_GATHER_LIDORDER=1: sample extracts gather hits in lid order
   glb::HostGather* hg = nullptr;  // host-assisted misses (glb_set_host_gather)
   uint32_t hg_permille = 0;       // share of a batch's misses gathered by host threads
   uint32_t hg_threads = 0;
@@ -365,7 +366,9 @@ void handoff_free(glb_ctx* c);  // handoff.cu: drop the a8 ring / peer mappings
 cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const float* src_miss,
                           const uint2* hit_list, const uint2* miss_list, const uint32_t* fill_src,
                           const uint32_t* dev_counts /* [nhit, nmiss] on device or null */,
-                          uint64_t nhit_host, uint64_t nmiss_host);
+                          uint64_t nhit_host, uint64_t nmiss_host,
+                          const int32_t* lidslot = nullptr /* hits in lid order (marks) */,
+                          const uint32_t* nl_dev = nullptr /* device n_L for lidslot */);
 cudaError_t launch_sort_misses(glb_ctx* c, const uint2* miss, const uint32_t* nmiss_dev,
                                uint2* sorted);
 // bins of the miss ordering for a V x D matrix; *scan_sums = scratch words of the device scan
