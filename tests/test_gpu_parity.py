@@ -266,8 +266,9 @@ GATHER_ENV = {"warp": {"GLB_GATHER_WARP": "1"}, "block": {"GLB_GATHER_WARP": "0"
               "host900_nobins": {"GLB_HOST_GATHER": "900", "GLB_HOST_GATHER_THREADS": "3",
                                  "GLB_MISS_BIN_LOG2": "0"},
               "missblocks3": {"GLB_MISS_BLOCKS": "3"},  # 3 blocks take every host miss
-              # hits gathered in lid order from the marks (holes = misses)
+              # hits gathered in lid order from the marks (the default) / from the hit list
               "lidorder": {"GLB_GATHER_LIDORDER": "1"},
+              "hitlist": {"GLB_GATHER_LIDORDER": "0"},
               "lidorder_host": {"GLB_GATHER_LIDORDER": "1", "GLB_HOST_GATHER": "400",
                                 "GLB_HOST_GATHER_THREADS": "2"},
               "dedup2_host": {"GLB_RELABEL_DEDUP": "2", "GLB_HOST_GATHER": "500"}}

@@ -53,12 +53,13 @@ def tiny():
 
 
 @pytest.mark.parametrize("world,alpha", [(2, 0.05), (3, 0.1), (4, 0.3), (8, 0.02), (2, 0.0)])
-@pytest.mark.parametrize("mode", ["dense", "hash", "dense_lidorder"])
+@pytest.mark.parametrize("mode", ["dense", "hash", "dense_hitlist"])
 def test_sharded_extract_sample_bit_exact(tiny, world, alpha, mode, monkeypatch):
-    """dense_lidorder: hits gathered in lid order from the marks (GLB_GATHER_LIDORDER=1)."""
-    if mode.endswith("_lidorder"):
-        monkeypatch.setenv("GLB_GATHER_LIDORDER", "1")
-        mode = mode[:-9]
+    """dense_hitlist: hits gathered from the hit list (GLB_GATHER_LIDORDER=0) instead of in
+    lid order from the marks (the default)."""
+    if mode.endswith("_hitlist"):
+        monkeypatch.setenv("GLB_GATHER_LIDORDER", "0")
+        mode = mode[:-8]
     g, go, counts = tiny
     sh = g.shape
     slot, shards = oracle.sharded_cache(counts, alpha, world)

@@ -20,7 +20,7 @@ go = oracle.GraphOracle(g.indptr, g.indices, g.features)
 VARIANTS = [{}, {"GLB_RELABEL_DEDUP": "1"}, {"GLB_RELABEL_DEDUP": "2"},
             {"GLB_HOST_GATHER": "400", "GLB_HOST_GATHER_THREADS": "2"},
             {"GLB_MISS_BIN_LOG2": "7", "GLB_GATHER_WARP": "1"}, {"GLB_MISS_BLOCKS": "3"},
-            {"GLB_GATHER_LIDORDER": "1", "GLB_HOST_GATHER": "400", "GLB_HOST_GATHER_THREADS": "2"}]
+            {"GLB_GATHER_LIDORDER": "0", "GLB_HOST_GATHER": "400", "GLB_HOST_GATHER_THREADS": "2"}]
 KEYS = {k for v in VARIANTS for k in v}
 for var, mode in [(v, m) for v in VARIANTS for m in ["dense", "hash"]]:
     for k in KEYS:
