@@ -96,8 +96,12 @@ def parse(argv=None):
     p.add_argument("--cache", default="replicated", choices=["replicated", "sharded"],
                    help="sharded: each rank caches alpha*V distinct rows, peers read them over "
                         "NVLink (NEXT-3; glb_build_cache_sharded)")
-    p.add_argument("--time-every", type=int, default=8,
-                   help="CUDA events around every n-th extract launch of the timed region")
+    p.add_argument("--time-every", type=int, default=0,
+                   help="CUDA events around every n-th extract launch of the timed region "
+                        "(0: every launch when alpha < 1 -- ms-long, host-bound extracts -- else "
+                        "every 8th: events between the launches of a 0.2-ms pipelined step cost "
+                        "overlap; the first extract of a region, which starts with an empty "
+                        "pipeline, is always among the timed ones)")
     p.add_argument("--host-gather", default="auto",
                    help="share of each batch's misses gathered by host threads "
                         "(glb_set_host_gather): a fraction, or 'auto' = 0.25 when a feature "
@@ -105,6 +109,8 @@ def parse(argv=None):
                         "bound by address translation, 1-KB rows are not; DESIGN.md §10)")
     p.add_argument("--host-gather-threads", type=int, default=0,
                    help="host threads per rank (0: min(8, usable cores / local ranks - 1))")
+    p.add_argument("--clock-ms", type=float, default=2.0,
+                   help="NVML clock / throttle-reason sampling period during the timed regions")
     p.add_argument("--pipeline", type=int, default=2, choices=[1, 2],
                    help="2: extract of batch b overlaps sampling of batch b+1 (two streams)")
     a = p.parse_args(argv)
@@ -253,8 +259,9 @@ class Clocks:
                "sw_power_cap": "nvmlClocksEventReasonSwPowerCap",
                "hw_power_brake": "nvmlClocksEventReasonHwPowerBrakeSlowdown"}
 
-    def __init__(self, index):
+    def __init__(self, index, interval_s=0.002):
         self.index = index
+        self.interval = interval_s
         self.ok = False
         try:
             import pynvml
@@ -276,21 +283,33 @@ class Clocks:
                 self.rs |= nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
             except Exception:
                 pass
-            time.sleep(0.002)
+            time.sleep(self.interval)
+
+    def _sample(self):
+        try:
+            self.sm.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+            self.rs |= self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+        except Exception:
+            pass
 
     def start(self):
         if not self.ok:
             return
         import threading
         self.sm, self.rs, self.stop_flag = [], 0, False
-        self.th = threading.Thread(target=self._run, daemon=True)
-        self.th.start()
+        self._sample()
+        self.th = None
+        if self.interval > 0:  # <= 0: one sample at start and one at stop only
+            self.th = threading.Thread(target=self._run, daemon=True)
+            self.th.start()
 
     def stop(self):
         if not self.ok:
             return None
         self.stop_flag = True
-        self.th.join()
+        if self.th is not None:
+            self.th.join()
+        self._sample()
         if not self.sm:
             return None
         reasons = sorted(k for k, a in self.REASONS.items()
@@ -699,9 +718,10 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
     # main stream, extract on the extract stream; the last kernel of a region is an extract).
     # Run r times steps [W + r*K, W + (r+1)*K): different batches, same protocol.
     K = args.steps
-    clocks = Clocks(local)
+    te = args.time_every if args.time_every > 0 else (1 if alpha < 1.0 else 8)
+    clocks = Clocks(local, args.clock_ms / 1e3)
     launches0 = ctx.launches
-    ctx.set_timing(args.time_every)  # events around every time_every-th extract launch
+    ctx.set_timing(te)  # events around every te-th extract launch
     clocks.start()
     runs, run_ms, enq_ms, wall_ms = [], [], [], []
     for r in range(args.runs):
@@ -758,7 +778,7 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
     # miss rows read over PCIe
     hbm_bytes = [h * (2 * 4 * D + 8) + m * (4 * D + 8) for h, m in zip(hits, misses)]
     link_bytes = [m * 4 * D for m in misses]
-    sel = list(range(0, len(timed_steps), args.time_every))[: len(x_ms)]  # the timed launches
+    sel = list(range(0, len(timed_steps), te))[: len(x_ms)]  # the timed launches
     ach_hbm = statistics.mean(hbm_bytes[j] / (t * 1e-3) for j, t in zip(sel, x_ms)) / 1e9
     ach_link = statistics.mean(link_bytes[j] / (t * 1e-3) for j, t in zip(sel, x_ms)) / 1e9
     x_mean = statistics.mean(x_ms)
@@ -830,7 +850,7 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
         "extract_ms_per_step": x_mean,
         "extract_share_of_step": x_mean / (elapsed_max / K),
         "kernel_bound_ms": bound_ms, "frac_of_binding_bound": bound_ms / x_mean,
-        "timed_launches": f"every {args.time_every}th extract of the {args.runs} timed regions "
+        "timed_launches": f"every {te}th extract of the {args.runs} timed regions "
                           f"({len(x_ms)} launches)",
         "measured_with": f"pipeline depth {args.pipeline} (the timed region)",
         "isolated": iso})

@@ -34,6 +34,7 @@ def main():
     ap.add_argument("--repeat", type=int, default=2, help="rounds over all variants")
     ap.add_argument("--host-gather", type=float, default=0.0)
     ap.add_argument("--relabel", default="auto")
+    ap.add_argument("--depths", default="2", help="pipeline depths to time, e.g. 2,1")
     args = ap.parse_args()
     import paper_conf_eurosys_yangtswycyz22_b200 as glb
     from paper_conf_eurosys_yangtswycyz22_b200 import parallel as par
@@ -72,36 +73,37 @@ def main():
                 ub = min(ub * (1 + k), sh.V)
             out = torch.empty((ub, sh.D), dtype=torch.float32, device="cuda")
             stream = torch.cuda.current_stream()
-            ctx.set_pipeline(2)
-            xs = ctx.extract_stream()
-            for i in range(5):
-                e, b = par.dp_step_batch(i, 0, 1, nb, sh.K)
-                ctx.sample_batch(e, b)
-                ctx.extract_sample(out)
-            ctx.sync()
-            ctx.set_timing(1)
-            s0 = torch.cuda.Event(enable_timing=True)
-            s1 = torch.cuda.Event(enable_timing=True)
-            s0.record(stream)
-            for i in range(5, 5 + args.steps):
-                e, b = par.dp_step_batch(i, 0, 1, nb, sh.K)
-                ctx.sample_batch(e, b)
-                ctx.extract_sample(out)
-            s1.record(xs)
-            torch.cuda.synchronize()
-            xms = ctx.extract_times()
-            ctx.set_timing(0)
-            misses = []
-            for i in range(5, 5 + min(args.steps, 10)):
-                e, b = par.dp_step_batch(i, 0, 1, nb, sh.K)
-                ctx.sample_batch(e, b)
-                misses.append(ctx.extract_sample(out, stats=True)["misses"])
-            m = statistics.mean(misses)
-            print(json.dumps({"config": sh.name, "alpha": args.alpha, "variant": name, "env": env,
-                              "round": rnd, "ms_per_step": s0.elapsed_time(s1) / args.steps,
-                              "extract_ms": statistics.mean(xms), "misses_per_step": m,
-                              "host_gbs": m * 4 * sh.D / (statistics.mean(xms) * 1e-3) / 1e9}),
-                  flush=True)
+            for depth in [int(x) for x in args.depths.split(",")]:
+                ctx.set_pipeline(depth)
+                xs = ctx.extract_stream() if depth == 2 else stream
+                for i in range(5):
+                    e, b = par.dp_step_batch(i, 0, 1, nb, sh.K)
+                    ctx.sample_batch(e, b)
+                    ctx.extract_sample(out)
+                ctx.sync()
+                ctx.set_timing(1)
+                s0 = torch.cuda.Event(enable_timing=True)
+                s1 = torch.cuda.Event(enable_timing=True)
+                s0.record(stream)
+                for i in range(5, 5 + args.steps):
+                    e, b = par.dp_step_batch(i, 0, 1, nb, sh.K)
+                    ctx.sample_batch(e, b)
+                    ctx.extract_sample(out)
+                s1.record(xs)
+                torch.cuda.synchronize()
+                xms = ctx.extract_times()
+                ctx.set_timing(0)
+                misses = []
+                for i in range(5, 5 + min(args.steps, 10)):
+                    e, b = par.dp_step_batch(i, 0, 1, nb, sh.K)
+                    ctx.sample_batch(e, b)
+                    misses.append(ctx.extract_sample(out, stats=True)["misses"])
+                m = statistics.mean(misses)
+                print(json.dumps({"config": sh.name, "alpha": args.alpha, "variant": name, "env": env,
+                                  "round": rnd, "depth": depth, "ms_per_step": s0.elapsed_time(s1) / args.steps,
+                                  "extract_ms": statistics.mean(xms), "misses_per_step": m,
+                                  "host_gbs": m * 4 * sh.D / (statistics.mean(xms) * 1e-3) / 1e9}),
+                      flush=True)
             ctx.close()
             del out
             torch.cuda.empty_cache()
