@@ -313,7 +313,9 @@ glb_status glb_create(int device, glb_ctx** out) {
       (e = cudaStreamCreateWithFlags(&c->own_stream, cudaStreamNonBlocking)) != cudaSuccess ||
       (e = cudaDeviceGetStreamPriorityRange(&prio_low, &prio_high)) != cudaSuccess ||
       // the extract stream (pipeline depth 2) yields SMs to the latency-bound sampler
-      (e = cudaStreamCreateWithPriority(&c->xstream, cudaStreamNonBlocking, prio_low)) != cudaSuccess ||
+      (e = cudaStreamCreateWithPriority(&c->xstream, cudaStreamNonBlocking,
+                                        getenv("GLB_XSTREAM_HIGH") && atoi(getenv("GLB_XSTREAM_HIGH"))
+                                            ? prio_high : prio_low)) != cudaSuccess ||
       (e = cudaStreamCreateWithPriority(&c->sstream, cudaStreamNonBlocking, prio_low)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_perm[0], cudaEventDisableTiming)) != cudaSuccess ||
       (e = cudaEventCreateWithFlags(&c->ev_perm[1], cudaEventDisableTiming)) != cudaSuccess ||

@@ -311,7 +311,9 @@ cudaError_t hg_configure(glb_ctx* c, uint32_t threads) {
     int lo = 0, hi = 0;
     cudaDeviceGetStreamPriorityRange(&lo, &hi);
     for (int i = 0; i < 2 && e == cudaSuccess; ++i) {
-      e = cudaStreamCreateWithPriority(&h->cs[i], cudaStreamNonBlocking, lo);
+      e = cudaStreamCreateWithPriority(&h->cs[i], cudaStreamNonBlocking,
+                                       getenv("GLB_XSTREAM_HIGH") && atoi(getenv("GLB_XSTREAM_HIGH"))
+                                           ? hi : lo);
       if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_end[i], cudaEventDisableTiming);
     }
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_split, cudaEventDisableTiming);
