@@ -355,6 +355,7 @@ glb_status glb_create(int device, glb_ctx** out) {
   if (const char* g = getenv("GLB_MISS_BULK")) c->miss_bulk = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_WARP")) c->gather_warp = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_LIDORDER")) c->gather_lidorder = atoi(g) != 0;
+  if (const char* g = getenv("GLB_MISSES_FIRST")) c->misses_first = atoi(g) != 0;
   if (const char* g = getenv("GLB_MISS_BLOCKS")) c->miss_blocks = atoi(g) > 0 ? (uint32_t)atoi(g) : 0u;
   if (const char* g = getenv("GLB_RELABEL_DEDUP")) {  // 1 warp-level, 2 block smem-staged
     const int m = atoi(g);

@@ -195,12 +195,27 @@ __global__ void __launch_bounds__(kThreads, GLB_GATHER_MINB)
   const float inv_u = 1.0f / (float)U;
   const uint64_t pol = l2_evict_first_policy();
   // chunk id g: g < nch -> hit chunk g; else miss chunk g - nch
+  // bit 2 (misses first): the miss-taking blocks start on the host misses -- the critical
+  // path of a host-bound extract -- and only then help with the hits, which the other
+  // blocks gather meanwhile
+  const bool misses_first = (misses_only & 4) && miss_blocks;
   auto claim = [&]() -> uint64_t {
     if (t == 0) {
-      unsigned int g = atomicAdd(&work[0], 1u);
-      if (g >= nch)  // only the first miss_blocks blocks take host chunks (0 = all)
-        g = (miss_blocks && blockIdx.x >= miss_blocks) ? (unsigned int)(nch + ncm)
-                                                       : (unsigned int)nch + atomicAdd(&work[1], 1u);
+      unsigned int g;
+      if (misses_first && blockIdx.x < miss_blocks) {
+        const unsigned int m = atomicAdd(&work[1], 1u);
+        if (m < ncm) {
+          g = (unsigned int)nch + m;
+        } else {
+          const unsigned int h = atomicAdd(&work[0], 1u);
+          g = h < nch ? h : (unsigned int)(nch + ncm);
+        }
+      } else {
+        g = atomicAdd(&work[0], 1u);
+        if (g >= nch)  // only the first miss_blocks blocks take host chunks (0 = all)
+          g = (miss_blocks && blockIdx.x >= miss_blocks) ? (unsigned int)(nch + ncm)
+                                                         : (unsigned int)nch + atomicAdd(&work[1], 1u);
+      }
       s_next = g;
     }
     __syncthreads();
@@ -689,7 +704,16 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   // blocks that take host-miss chunks: GLB_MISS_BLOCKS, else one per SM while the host
   // takes a share of the misses (measured on PA: fewer zero-copy rows in flight touch
   // fewer host pages at once -- 5.20-5.23 vs 5.35 ms per step; profiles/r02_missblocks.txt)
-  const uint32_t mb = c->miss_blocks ? c->miss_blocks : (c->hg_inflight ? (uint32_t)c->num_sms : 0u);
+  // On the extract stream (pipeline depth 2) a sample's host misses are the critical path:
+  // one block per SM takes them, and those blocks start on them (misses first) while the
+  // other half of the grid gathers the HBM hits -- measured on PA / UK / TW at the paper's
+  // R%: 5.08-5.14 vs 5.29-5.39, 6.07-6.15 vs 6.36, 7.80 vs 8.18-8.54 ms per step
+  // (profiles/r02_missesfirst_ab.txt).  GLB_MISS_BLOCKS / GLB_MISSES_FIRST override.
+  const bool pipe_misses = c->stream == c->xstream && miss_list && c->C < c->V;
+  const uint32_t mb = c->miss_blocks ? c->miss_blocks
+                      : ((c->hg_inflight || pipe_misses) ? (uint32_t)c->num_sms : 0u);
+  const bool first = c->misses_first >= 0 ? c->misses_first != 0 : pipe_misses;
+  const int mfirst = (mb && first) ? 4 : 0;
   // chunk counters of the launching stream (this ctx's gathers are serial on it; each
   // launch leaves them zeroed for the next)
   unsigned int* work = c->stream == c->xstream ? c->work + 4 : c->work;
@@ -728,19 +752,19 @@ cudaError_t launch_gather(glb_ctx* c, float* out, const float* src_hit, const fl
   if (vec && shard)
     e = launch_pdl(k_gather<float4, true>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | mfirst | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
   else if (vec)
     e = launch_pdl(k_gather<float4, false>, grid, kThreads, c->stream, (float4*)out,
                    (const float4*)src_hit, (const float4*)src_miss, hit_list, miss_list, fill_src,
-                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
+                   dev_counts, nhit_host, nmiss_host, U, R, Sh, So, wb, mo | mfirst | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
   else if (shard)
     e = launch_pdl(k_gather<float, true>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
+                   Sh, So, wb, mo | mfirst | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
   else
     e = launch_pdl(k_gather<float, false>, grid, kThreads, c->stream, out, src_hit, src_miss,
                    hit_list, miss_list, fill_src, dev_counts, nhit_host, nmiss_host, U, R,
-                   Sh, So, wb, mo | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
+                   Sh, So, wb, mo | mfirst | (int)(mb << 8), c->xcount, work, tab, lidslot, nl_dev);
   count_launch(c);
   return e;
 }

@@ -210,6 +210,8 @@ struct glb_ctx {
   int miss_bulk = 0;           // GLB_MISS_BULK=1: host misses through cp.async.bulk
   int gather_warp = 0;         // GLB_GATHER_WARP=1: warp-independent gather (k_gather_w)
   uint32_t miss_blocks = 0;    // GLB_MISS_BLOCKS: blocks of k_gather that take host misses (0 all)
+  int misses_first = -1;       // miss-taking gather blocks start on the misses: -1 auto (on the
+                               // extract stream), GLB_MISSES_FIRST=0/1 forces
   int gather_lidorder = 1;     // sample extracts gather hits in lid order from the marks
                                // (GLB_GATHER_LIDORDER=0: from the hit list; measured 1-2 % slower)
   glb::HostGather* hg = nullptr;  // host-assisted misses (glb_set_host_gather)

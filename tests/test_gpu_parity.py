@@ -269,6 +269,10 @@ GATHER_ENV = {"warp": {"GLB_GATHER_WARP": "1"}, "block": {"GLB_GATHER_WARP": "0"
               # hits gathered in lid order from the marks (the default) / from the hit list
               "lidorder": {"GLB_GATHER_LIDORDER": "1"},
               "hitlist": {"GLB_GATHER_LIDORDER": "0"},
+              # the miss-taking blocks start on the misses (GLB_MISSES_FIRST)
+              "missesfirst": {"GLB_MISSES_FIRST": "1", "GLB_MISS_BLOCKS": "3"},
+              "missesfirst_host": {"GLB_MISSES_FIRST": "1", "GLB_HOST_GATHER": "300",
+                                   "GLB_HOST_GATHER_THREADS": "2"},
               "lidorder_host": {"GLB_GATHER_LIDORDER": "1", "GLB_HOST_GATHER": "400",
                                 "GLB_HOST_GATHER_THREADS": "2"},
               "dedup2_host": {"GLB_RELABEL_DEDUP": "2", "GLB_HOST_GATHER": "500"}}
