@@ -154,6 +154,9 @@ def check_config(name, Ks=None, handoff=False, relabel_modes=("auto",)):
     ctx = None
     for mode in relabel_modes:
         ctx = make_sampler_ctx(g, sh, relabel=mode)
+        ctx.set_pipeline(2)  # bench.py's launch configuration (extract stream, misses first)
+        if 4 * sh.D <= 512:  # ... and its host-assisted misses for <= 512-byte rows
+            ctx.set_host_gather(0.25, threads=8)
         if mode != "auto":
             assert ctx.relabel_mode == mode
         for K in (Ks or [sh.K]):
