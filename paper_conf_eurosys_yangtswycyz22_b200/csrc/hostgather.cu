@@ -182,6 +182,7 @@ struct HostGather {
   HostPool* pool = nullptr;
   cudaStream_t cs[2] = {nullptr, nullptr};
   cudaEvent_t ev_split = nullptr, ev_d2h = nullptr, ev_end[2] = {nullptr, nullptr};
+  cudaEvent_t ev_chunk[kMaxChunks] = {};  // host function k done (its staged rows are ready)
   bool dma = false;  // staged rows cross the link by DMA (GLB_HOST_GATHER_DMA=1; measured slower)
   int nch = 4;       // chunks per extract (GLB_HOST_GATHER_CHUNKS)
   int sblocks = 0;   // scatter grid (GLB_HOST_GATHER_SCATTER_BLOCKS; 0 = one per SM)
@@ -290,6 +291,8 @@ void hg_free(glb_ctx* c) {
   }
   if (h->ev_split) cudaEventDestroy(h->ev_split);
   if (h->ev_d2h) cudaEventDestroy(h->ev_d2h);
+  for (int k = 0; k < kMaxChunks; ++k)
+    if (h->ev_chunk[k]) cudaEventDestroy(h->ev_chunk[k]);
   delete h;
   c->hg = nullptr;
 }
@@ -318,6 +321,8 @@ cudaError_t hg_configure(glb_ctx* c, uint32_t threads) {
     }
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_split, cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev_d2h, cudaEventDisableTiming);
+    for (int k = 0; k < kMaxChunks && e == cudaSuccess; ++k)
+      e = cudaEventCreateWithFlags(&h->ev_chunk[k], cudaEventDisableTiming);
     if (e != cudaSuccess) return e;
   }
   if (!h->pool || h->pool->size() != (int)threads) {
@@ -402,8 +407,11 @@ cudaError_t hg_enqueue(glb_ctx* c, float* out, const uint2* miss_sorted, uint32_
   const bool vec = (c->D % 4) == 0;
   const uint32_t U = vec ? c->D / 4 : c->D;
   const size_t rb = 4ull * c->D;
+  // The host functions run back to back on cs[0] (the host gathers without waiting for any
+  // scatter); chunk k's copy-out and scatter run on cs[1] once its host function is done
+  // (ev_chunk[k]), so the staged rows cross the link while the host gathers the next chunk.
   for (int k = 0; k < h->nch; ++k) {  // gather chunk k on the host, move it, scatter it
-    cudaStream_t q = h->cs[k & 1];
+    cudaStream_t q = h->cs[1];
     const uint64_t lo = chunk_lo(target, k, h->nch), hi = chunk_lo(target, k + 1, h->nch);
     if (hi <= lo) continue;
     HgJob* j = &h->job[h->njobs++ % kJobRing];
@@ -414,10 +422,13 @@ cudaError_t hg_enqueue(glb_ctx* c, float* out, const uint2* miss_sorted, uint32_
     j->nch = h->nch;
     j->target = target;
     j->done.store(0, std::memory_order_relaxed);
-    if ((e = cudaLaunchHostFunc(q, hg_host_fn, j)) != cudaSuccess) {
+    if ((e = cudaLaunchHostFunc(h->cs[0], hg_host_fn, j)) != cudaSuccess) {
       j->done.store(1);
       return e;
     }
+    if ((e = cudaEventRecord(h->ev_chunk[k], h->cs[0])) != cudaSuccess ||
+        (e = cudaStreamWaitEvent(q, h->ev_chunk[k], 0)) != cudaSuccess)
+      return e;
     const uint8_t* src = h->stage_dev[s];
     if (h->dma) {
       if ((e = cudaMemcpyAsync(h->dstage[s] + lo * rb, h->stage[s] + lo * rb, (hi - lo) * rb,

@@ -33,6 +33,9 @@ def main():
     ap.add_argument("--spans", default="1.0,0.5,0.25,0.05")
     ap.add_argument("--bins", default="21,0")
     ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--region-fracs", default="",
+                    help="also draw the ids from a random subset (this fraction) of the 2 MB regions "
+                         "of the whole matrix: same span, fewer distinct regions per extract")
     args = ap.parse_args()
     import paper_conf_eurosys_yangtswycyz22_b200 as glb
     t0 = time.perf_counter()
@@ -70,6 +73,28 @@ def main():
                                   "span_gb": hi * args.D * 4 / 1e9, "input_order": order,
                                   "n": int(v.size), "row_bytes": 4 * args.D, "ms": ms,
                                   "gbs": v.size * 4 * args.D / (ms * 1e-3) / 1e9}), flush=True)
+        rows_per_region = (2 << 20) // (args.D * 4)
+        nreg = (args.V + rows_per_region - 1) // rows_per_region
+        for rf in [float(x) for x in args.region_fracs.split(",") if x]:
+            regs = rng.choice(nreg, size=max(1, int(nreg * rf)), replace=False)
+            cand = (regs[:, None] * rows_per_region + np.arange(rows_per_region)[None, :]).ravel()
+            cand = cand[cand < args.V]
+            ids = rng.choice(cand, size=args.n, replace=False).astype(np.int32)
+            dv = torch.from_numpy(np.sort(ids)).cuda()
+            ctx.extract(dv, out=out)
+            ts = []
+            for _ in range(args.reps):
+                e0 = torch.cuda.Event(enable_timing=True)
+                e1 = torch.cuda.Event(enable_timing=True)
+                e0.record(s)
+                ctx.extract(dv, out=out)
+                e1.record(s)
+                torch.cuda.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            ms = min(ts)
+            print(json.dumps({"miss_bin_log2": b, "region_frac": rf, "regions": int(len(regs)),
+                              "n": args.n, "ms": ms, "gbs": args.n * 4 * args.D / (ms * 1e-3) / 1e9}),
+                  flush=True)
         ctx.close()
         del out
         torch.cuda.empty_cache()
