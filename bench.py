@@ -104,11 +104,16 @@ def parse(argv=None):
                         "pipeline, is always among the timed ones)")
     p.add_argument("--host-gather", default="auto",
                    help="share of each batch's misses gathered by host threads "
-                        "(glb_set_host_gather): a fraction, or 'auto' = 0.25 when a feature "
-                        "row is <= 512 B and alpha < 1 (measured: 512-B zero-copy rows are "
-                        "bound by address translation, 1-KB rows are not; DESIGN.md §10)")
+                        "(glb_set_host_gather): a fraction, or 'auto' = 0.15 with the cold store "
+                        "(0.25 without) when a feature row is <= 512 B and alpha < 1 (measured: "
+                        "512-B zero-copy rows are bound by address translation, 1-KB rows are "
+                        "not; DESIGN.md §7)")
     p.add_argument("--host-gather-threads", type=int, default=0,
-                   help="host threads per rank (0: min(8, usable cores / local ranks - 1))")
+                   help="host threads per rank (0: min(4, usable cores / local ranks - 1))")
+    p.add_argument("--cold-store", default="auto", choices=["auto", "on", "off"],
+                   help="misses read a rank-ordered pinned copy of the non-cached rows "
+                        "(glb_set_cold_store); auto = on for <= 512-B rows at alpha < 1 with one "
+                        "rank per node (the copy is per process)")
     p.add_argument("--clock-ms", type=float, default=2.0,
                    help="NVML clock / throttle-reason sampling period during the timed regions")
     p.add_argument("--pipeline", type=int, default=2, choices=[1, 2],
@@ -672,6 +677,10 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
             t_counts.copy_(c)
     torch.cuda.synchronize()
     t_pre = time.perf_counter() - t0
+    small_rows = 4 * sh.D <= 512 and alpha < 1.0
+    cold = (small_rows and local_world == 1 and args.cache != "sharded"
+            if args.cold_store == "auto" else args.cold_store == "on")
+    ctx.set_cold_store(cold)
     t0 = time.perf_counter()
     if args.cache == "sharded":
         par.build_sharded_cache(ctx, alpha, rank, world)
@@ -679,14 +688,14 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
         ctx.build_cache(alpha)
     torch.cuda.synchronize()
     t_cache = time.perf_counter() - t0
-
     hg = args.host_gather
-    hg = (0.25 if 4 * sh.D <= 512 and alpha < 1.0 else 0.0) if hg == "auto" else float(hg)
+    hg = ((0.15 if cold else 0.25) if small_rows else 0.0) if hg == "auto" else float(hg)
     if hg > 0:
         nt = args.host_gather_threads
         if nt <= 0:  # share the node's cores between the local ranks
-            nt = min(8, max(2, host_info()["nproc"] // max(1, local_world) - 1))
+            nt = min(4, max(2, host_info()["nproc"] // max(1, local_world) - 1))
         ctx.set_host_gather(hg, threads=nt)
+
     ctx_cache_rows = ctx.cache_size
     ub = sh.batch
     for k in sh.fanouts:
@@ -881,6 +890,7 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
                             "presample": t_pre, "build_cache": t_cache},
            "cache": {"layout": args.cache, "rows_cached": ctx_cache_rows},
            "host_gather": ctx.host_gather,
+           "cold_store_rows": ctx.cold_store_rows,
            "relabel_table": ctx.relabel_mode, "relabel_l2_window_bytes": ctx.relabel_l2_window,
            "host_inputs": ("node-shared memfd, generated once by local rank 0 and mapped by "
                            f"{local_world} ranks") if shared else "private to this rank"}
@@ -1009,6 +1019,8 @@ def hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs, b
 
     per_epoch = []
     acc_sum = None
+    # the sweeps rebuild the cache ~15 times: without the cold store (a host copy per build)
+    ctx.set_cold_store(False)
     m0 = max([sh.K] + [int(x) for x in args.k_sweep.split(",") if x])
     for e in range(m0, m0 + args.measure_epochs):
         ctx.reset_counts(glb.COUNT_ACCESS)
@@ -1146,7 +1158,7 @@ def main(argv=None):
             "pr_alpha1": pr1,
             "host": host_info(), "gpu": gpu_info(local),
         }
-        for k in ("cache", "host_gather", "relabel_table", "relabel_l2_window_bytes", "host_inputs",
+        for k in ("cache", "host_gather", "cold_store_rows", "relabel_table", "relabel_l2_window_bytes", "host_inputs",
                   "host_wall_ms_timed_region", "host_enqueue_ms_timed_region", "hit_rate",
                   "alpha_sweep", "presc_k_sweep", "measured_epochs", "footprint_similarity",
                   "units", "preprocess_s"):

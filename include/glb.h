@@ -278,6 +278,15 @@ glb_status glb_extract_stream(glb_ctx* ctx, void** cuda_stream_out);
  * this ctx (not to handoff-received ones) and to caches with C < V.  Synchronous (creates the
  * thread pool).  Errors: EINVAL (fraction not in [0,1), threads > 256). */
 glb_status glb_set_host_gather(glb_ctx* ctx, uint32_t threads, double fraction);
+/* Cold store: at the next glb_build_cache (single-GPU cache), copy the rows NOT cached --
+ * ranks C..V-1 of the load_cache order (L301) -- into a pinned host buffer in rank order and
+ * read misses from it instead of the caller's gid-ordered matrix: a batch's misses then
+ * touch fewer 2 MB host regions, the unit the zero-copy link pays for.  Costs
+ * (V - C) x D x 4 bytes of pinned host memory and a host copy at build time (the load_cache
+ * phase, Table 6).  Results are identical.  enable 0 drops it.  Environment GLB_COLD_STORE=1.
+ * glb_cold_store_rows: rows held (0 = none).  Synchronous. */
+glb_status glb_set_cold_store(glb_ctx* ctx, int enable);
+glb_status glb_cold_store_rows(const glb_ctx* ctx, uint64_t* rows);
 glb_status glb_host_gather(const glb_ctx* ctx, uint32_t* threads, double* fraction);
 
 /* Timing of the extract kernel itself: CUDA events around every `period`-th

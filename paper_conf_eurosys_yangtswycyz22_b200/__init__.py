@@ -42,7 +42,7 @@ EXPORTS = [
     "glb_sample_async", "glb_extract_counts_device_ptr",
     "glb_handoff_create", "glb_handoff_attach", "glb_handoff_connect", "glb_handoff_send",
     "glb_handoff_recv", "glb_handoff_tag", "glb_handoff_release", "glb_relabel_l2_window",
-    "glb_set_host_gather", "glb_host_gather",
+    "glb_set_host_gather", "glb_host_gather", "glb_set_cold_store", "glb_cold_store_rows",
 ]
 MAX_SHARDS = 16
 IPC_HANDLE_BYTES = 64
@@ -149,6 +149,8 @@ def lib(auto_build: bool = True):
         "glb_handoff_tag": ([vp, ctypes.POINTER(u64)], i32),
         "glb_handoff_release": ([vp, u32], i32),
         "glb_set_host_gather": ([vp, u32, dbl], i32),
+        "glb_set_cold_store": ([vp, i32], i32),
+        "glb_cold_store_rows": ([vp, ctypes.POINTER(u64)], i32),
         "glb_host_gather": ([vp, ctypes.POINTER(u32), ctypes.POINTER(dbl)], i32),
         "glb_footprint_similarity": ([vp, vp, vp, dbl, ctypes.POINTER(u64), ctypes.POINTER(u64),
                                       ctypes.POINTER(dbl)], i32),
@@ -548,6 +550,17 @@ class Context:
         t, f = ctypes.c_uint32(), ctypes.c_double()
         self._ck(self._lib.glb_host_gather(self._h, ctypes.byref(t), ctypes.byref(f)))
         return {"threads": t.value, "fraction": f.value}
+
+    def set_cold_store(self, enable: bool = True):
+        """Misses read a rank-ordered pinned copy of the non-cached rows, built by the next
+        build_cache (include/glb.h glb_set_cold_store)."""
+        self._ck(self._lib.glb_set_cold_store(self._h, int(bool(enable))))
+
+    @property
+    def cold_store_rows(self) -> int:
+        n = ctypes.c_uint64()
+        self._ck(self._lib.glb_cold_store_rows(self._h, ctypes.byref(n)))
+        return n.value
 
     def set_pipeline(self, depth: int):
         """depth 2: double-buffered samples, extract on its own stream overlapping the

@@ -11,6 +11,7 @@
 #include <cstring>
 #include <new>
 #include <thread>
+#include <vector>
 
 #include "glb_internal.cuh"
 #include <nvtx3/nvToolsExt.h>
@@ -114,8 +115,21 @@ void close_shards(glb_ctx* c) {
   c->C_local = 0;
 }
 
+// Drop the cold store (host copy + map); callers synchronise first.
+void free_cold(glb_ctx* c) {
+  if (c->cold_h) {
+    cudaHostUnregister(c->cold_h);
+    free(c->cold_h);
+  }
+  c->cold_h = nullptr;
+  c->cold_d = nullptr;
+  c->cold_rows = 0;
+  dfree(c->cold_row);
+}
+
 void free_graph(glb_ctx* c) {
   close_shards(c);
+  free_cold(c);
   dfree(c->indptr); dfree(c->indices); dfree(c->wprefix); dfree(c->vmap); dfree(c->htab);
   c->hslot = nullptr;
   c->hmask = 0;
@@ -356,6 +370,7 @@ glb_status glb_create(int device, glb_ctx** out) {
   if (const char* g = getenv("GLB_GATHER_WARP")) c->gather_warp = atoi(g) != 0;
   if (const char* g = getenv("GLB_GATHER_LIDORDER")) c->gather_lidorder = atoi(g) != 0;
   if (const char* g = getenv("GLB_MISSES_FIRST")) c->misses_first = atoi(g) != 0;
+  if (const char* g = getenv("GLB_COLD_STORE")) c->cold_store = atoi(g) != 0;
   if (const char* g = getenv("GLB_MISS_BLOCKS")) c->miss_blocks = atoi(g) > 0 ? (uint32_t)atoi(g) : 0u;
   if (const char* g = getenv("GLB_RELABEL_DEDUP")) {  // 1 warp-level, 2 block smem-staged
     const int m = atoi(g);
@@ -846,6 +861,51 @@ static glb_status rank_vertices(glb_ctx* c, const uint32_t* hot, uint32_t* tmp, 
   return GLB_OK;
 }
 
+// Cold store (glb_set_cold_store): the rows of ranks C..V-1 copied, in rank order, into a
+// pinned host buffer the misses read instead of the caller's gid-ordered matrix.  A batch's
+// misses then fall in the non-cached part only and the warmer (more often missed) rows sit
+// together, so the zero-copy reads touch fewer 2 MB host regions (the host link's cost is
+// per region).  Bytes are the same rows, so results are unchanged.
+static glb_status build_cold_store(glb_ctx* c, const uint32_t* order, uint64_t C) {
+  const uint64_t V = c->V, n = V - C;
+  const size_t rb = 4ull * c->D;
+  std::vector<uint32_t> ord(n);
+  CK(cudaMemcpyAsync(ord.data(), order + C, sizeof(uint32_t) * n, cudaMemcpyDeviceToHost, c->stream));
+  CK(cudaStreamSynchronize(c->stream));
+  const size_t bytes = n * rb;
+  uint8_t* h = (uint8_t*)aligned_alloc(1 << 21, (bytes + (1 << 21) - 1) & ~(size_t)((1 << 21) - 1));
+  if (!h) return set_err(c, GLB_ENOMEM, "cold store: host alloc of %zu bytes", bytes);
+  const uint8_t* src = static_cast<const uint8_t*>(c->h_features);
+  unsigned T = std::thread::hardware_concurrency();
+  T = T ? T : 1;
+  std::vector<std::thread> th;
+  for (unsigned t = 0; t < T; ++t)
+    th.emplace_back([&, t] {
+      const uint64_t a = n * t / T, b = n * (t + 1) / T;
+      for (uint64_t i = a; i < b; ++i) memcpy(h + i * rb, src + (size_t)ord[i] * rb, rb);
+    });
+  for (auto& x : th) x.join();
+  cudaError_t e = cudaHostRegister(h, bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
+  if (e != cudaSuccess) {
+    (void)cudaGetLastError();
+    free(h);
+    return set_err(c, GLB_ENOMEM, "cold store: cudaHostRegister(%zu bytes): %s", bytes, cudaGetErrorString(e));
+  }
+  void* dp = nullptr;
+  if ((e = cudaHostGetDevicePointer(&dp, h, 0)) != cudaSuccess) {
+    cudaHostUnregister(h);
+    free(h);
+    return cuda_fail(c, e, "cold store device pointer");
+  }
+  c->cold_h = (float*)h;
+  c->cold_d = (const float*)dp;
+  c->cold_rows = n;
+  CK(dalloc(&c->cold_row, V));
+  CK(cudaMemsetAsync(c->cold_row, 0xFF, sizeof(uint32_t) * V, c->stream));
+  CK(launch_cold_rows(c, order, C));
+  return GLB_OK;
+}
+
 // load_cache (L301) for a cache of C global rows split over `world` shards: the
 // vertex of global rank i is cached iff i < C, slot[v] = i; shard i % world holds it
 // at row i / world (world == 1: the whole cache is local, row = rank).
@@ -863,6 +923,11 @@ static glb_status build_cache_impl(glb_ctx* c, uint64_t C, const uint32_t* hotne
   CK(cudaMemsetAsync(c->slot, 0xFF, sizeof(int32_t) * V, c->stream));
   CK(launch_assign_slots(c, order, C));
   CK(launch_vmap_reset(c));  // dense mode: copy the slots into the relabel entries
+  free_cold(c);
+  if (c->cold_store && world == 1 && c->features_mapped && C < V) {
+    glb_status cs = build_cold_store(c, order, C);
+    if (cs != GLB_OK) { cudaFree(tmp); return cs; }
+  }
   dfree(c->cache);
   c->C = C;
   c->shard_rank = rank;
@@ -1107,11 +1172,11 @@ glb_status glb_extract(glb_ctx* c, const uint32_t* vertices, uint64_t n, void* o
   CK(cudaMemsetAsync(&c->st_x->nhit, 0, 2 * sizeof(uint32_t), c->stream));
   if (n) CK(launch_mark(c, vertices, n));
   const uint2* misses = c->xb.miss_list;
-  if (n && c->C < c->V && c->miss_bin_log2) {  // rows may come over PCIe: order them by address
+  if (n && c->C < c->V && (c->miss_bin_log2 || c->cold_row)) {  // rows may come over PCIe: order them by address
     CK(launch_sort_misses(c, c->xb.miss_list, &c->st_x->nmiss, c->xb.miss_sorted));
     misses = c->xb.miss_sorted;
   }
-  CK(launch_gather(c, (float*)out, c->cache, c->features_mapped, c->xb.hit_list, misses,
+  CK(launch_gather(c, (float*)out, c->cache, miss_rows_dev(c), c->xb.hit_list, misses,
                    nullptr, &c->st_x->nhit, 0, 0));
   if (stats) {
     CK(cudaMemcpyAsync(c->h_xcount, c->xcount, 3 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, c->stream));
@@ -1157,7 +1222,7 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
   }
   const uint2* misses = c->sb.miss_list;
   cudaError_t e = cudaSuccess;
-  if (c->C < c->V && c->miss_bin_log2) {  // rows may come over PCIe: order them by address
+  if (c->C < c->V && (c->miss_bin_log2 || c->cold_row)) {  // rows may come over PCIe: order them by address
     e = launch_sort_misses(c, c->sb.miss_list, &c->st->nmiss, c->sb.miss_sorted);
     misses = c->sb.miss_sorted;
   }
@@ -1167,7 +1232,7 @@ glb_status glb_extract_sample(glb_ctx* c, void* out, glb_extract_stats* stats) {
   if (e == cudaSuccess && hg) e = hg_enqueue(c, (float*)out, misses, &dcnt);
   c->hg_inflight = hg && dcnt;
   if (e == cudaSuccess)
-    e = launch_gather(c, (float*)out, c->cache, c->features_mapped, c->sb.hit_list, misses,
+    e = launch_gather(c, (float*)out, c->cache, miss_rows_dev(c), c->sb.hit_list, misses,
                       nullptr, dcnt ? dcnt : &c->st->nhit, 0, 0,
                       c->gather_lidorder && !c->gather_warp ? c->sb.lidslot : nullptr,
                       &c->st->n[c->last_L]);
@@ -1248,6 +1313,22 @@ glb_status glb_set_host_gather(glb_ctx* c, uint32_t threads, double fraction) {
   CK(hg_configure(c, threads - 1));  // the host-function thread itself is the last worker
   c->hg_permille = pm;
   c->hg_threads = threads;
+  return GLB_OK;
+}
+
+glb_status glb_set_cold_store(glb_ctx* c, int enable) {
+  ENTER(c);
+  c->cold_store = enable != 0;
+  if (!c->cold_store) {
+    CK(sync_all(c));
+    free_cold(c);
+  }
+  return GLB_OK;
+}
+
+glb_status glb_cold_store_rows(const glb_ctx* c, uint64_t* rows) {
+  if (!c || !rows) return GLB_EINVAL;
+  *rows = c->cold_rows;
   return GLB_OK;
 }
 

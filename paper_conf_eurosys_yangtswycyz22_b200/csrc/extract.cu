@@ -402,11 +402,18 @@ __global__ void __launch_bounds__(kThreads)
 // ---- host-miss ordering: a one-pass counting sort of the miss list by the 2 MB
 // host page its source row lives in, so consecutive zero-copy reads share GPU
 // address translations (measured: random 512 B rows over 64 GB 35 -> 47 GB/s).
+// cold_row (nullable): the cold store's row of each vertex (rank-ordered host copy of the
+// non-cached rows, glb_set_cold_store) -- the misses are translated while they are ordered
+__device__ __forceinline__ uint32_t host_row(uint32_t gid, const uint32_t* cold_row) {
+  return cold_row ? __ldg(cold_row + gid) : gid;
+}
+
 __global__ void k_miss_hist(const uint2* __restrict__ miss, const uint32_t* __restrict__ nmiss,
-                            uint32_t page_shift, unsigned int* __restrict__ bins) {
+                            uint32_t page_shift, unsigned int* __restrict__ bins,
+                            const uint32_t* __restrict__ cold_row) {
   const uint32_t n = *nmiss;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x)
-    atomicAdd(&bins[miss[i].y >> page_shift], 1u);
+    atomicAdd(&bins[host_row(miss[i].y, cold_row) >> page_shift], 1u);
 }
 
 __global__ void __launch_bounds__(1024) k_miss_scan(unsigned int* bins, uint32_t nb) {
@@ -445,10 +452,11 @@ __global__ void __launch_bounds__(1024) k_miss_scan(unsigned int* bins, uint32_t
 
 __global__ void k_miss_scatter(const uint2* __restrict__ miss, const uint32_t* __restrict__ nmiss,
                                uint32_t page_shift, unsigned int* __restrict__ offs,
-                               uint2* __restrict__ sorted) {
+                               uint2* __restrict__ sorted, const uint32_t* __restrict__ cold_row) {
   const uint32_t n = *nmiss;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
-    const uint2 m = miss[i];
+    uint2 m = miss[i];
+    m.y = host_row(m.y, cold_row);
     sorted[atomicAdd(&offs[m.y >> page_shift], 1u)] = m;
   }
 }
@@ -567,16 +575,18 @@ __global__ void __launch_bounds__(64)
 
 cudaError_t launch_sort_misses(glb_ctx* c, const uint2* miss, const uint32_t* nmiss_dev,
                                uint2* sorted) {
-  // bins of 2^miss_bin_log2 bytes of the host matrix (rounded down to a power-of-2 row count)
+  // bins of 2^miss_bin_log2 bytes of the host matrix (rounded down to a power-of-2 row count);
+  // with a cold store the entries' host rows are cold-store rows, ordered the same way
   const uint64_t row_bytes = 4ull * c->D;
   uint32_t shift = 0;
-  while ((row_bytes << (shift + 1)) <= (1ull << c->miss_bin_log2)) ++shift;
+  const uint32_t lg = c->miss_bin_log2 ? c->miss_bin_log2 : 21;  // the cold store needs the pass
+  while ((row_bytes << (shift + 1)) <= (1ull << lg)) ++shift;
   const uint32_t nb = (uint32_t)((c->V >> shift) + 1);
   if (nb > c->miss_bins_cap) return cudaErrorInvalidValue;
   cudaError_t e = cudaMemsetAsync(c->miss_bins, 0, sizeof(unsigned int) * nb, c->stream);
   if (e != cudaSuccess) return e;
   const int grid = c->num_sms * 4;
-  k_miss_hist<<<grid, kThreads, 0, c->stream>>>(miss, nmiss_dev, shift, c->miss_bins);
+  k_miss_hist<<<grid, kThreads, 0, c->stream>>>(miss, nmiss_dev, shift, c->miss_bins, c->cold_row);
   count_launch(c);
   unsigned int* offs = c->miss_bins;
   if (nb <= 8192) {  // a few coarse bins: one block scans them in place
@@ -587,7 +597,7 @@ cudaError_t launch_sort_misses(glb_ctx* c, const uint2* miss, const uint32_t* nm
     e = scan_exclusive_u32(c, c->miss_bins, nb, offs, offs + c->miss_bins_cap);
     if (e != cudaSuccess) return e;
   }
-  k_miss_scatter<<<grid, kThreads, 0, c->stream>>>(miss, nmiss_dev, shift, offs, sorted);
+  k_miss_scatter<<<grid, kThreads, 0, c->stream>>>(miss, nmiss_dev, shift, offs, sorted, c->cold_row);
   count_launch(c);
   return cudaGetLastError();
 }

@@ -210,6 +210,13 @@ struct glb_ctx {
   int miss_bulk = 0;           // GLB_MISS_BULK=1: host misses through cp.async.bulk
   int gather_warp = 0;         // GLB_GATHER_WARP=1: warp-independent gather (k_gather_w)
   uint32_t miss_blocks = 0;    // GLB_MISS_BLOCKS: blocks of k_gather that take host misses (0 all)
+  // cold store (glb_set_cold_store): a rank-ordered, pinned host copy of the rows NOT in the
+  // HBM cache; misses read it instead of the caller's matrix (fewer host pages per batch)
+  int cold_store = 0;             // enabled for the next build_cache
+  float* cold_h = nullptr;        // host rows [V - C][D], registered mapped + portable
+  const float* cold_d = nullptr;  // device alias
+  uint64_t cold_rows = 0;
+  uint32_t* cold_row = nullptr;   // device u32[V]: the cold-store row of a non-cached vertex
   int misses_first = -1;       // miss-taking gather blocks start on the misses: -1 auto (on the
                                // extract stream), GLB_MISSES_FIRST=0/1 forces
   int gather_lidorder = 1;     // sample extracts gather hits in lid order from the marks
@@ -414,6 +421,10 @@ bool hg_active(const glb_ctx* c);
 cudaError_t hg_enqueue(glb_ctx* c, float* out, const uint2* miss_sorted, uint32_t** dcnt_out);
 cudaError_t hg_join(glb_ctx* c);
 cudaError_t hg_sync(glb_ctx* c);
+// host rows the misses read: the cold store when there is one, else the caller's matrix
+inline const void* miss_rows_host(const glb_ctx* c) { return c->cold_h ? (const void*)c->cold_h : c->h_features; }
+inline const float* miss_rows_dev(const glb_ctx* c) { return c->cold_d ? c->cold_d : c->features_mapped; }
+cudaError_t launch_cold_rows(glb_ctx* c, const uint32_t* order, uint64_t C);  // cold_row map
 
 inline void count_launch(glb_ctx* c, int n = 1) { c->launches += (uint64_t)n; }
 

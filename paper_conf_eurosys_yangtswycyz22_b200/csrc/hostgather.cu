@@ -249,7 +249,7 @@ void hg_gather(const HgJob* j) {
   if (hi > ncpu) hi = ncpu;
   if (hi <= lo) return;
   const size_t rb = 4ull * c->D;
-  const uint8_t* feats = static_cast<const uint8_t*>(c->h_features);
+  const uint8_t* feats = static_cast<const uint8_t*>(miss_rows_host(c));
   uint8_t* stage = h->stage[j->slot];
   const uint2* ent = h->ent[j->slot];
   const uint32_t ntask = (uint32_t)((hi - lo + kTaskRows - 1) / kTaskRows);

@@ -547,6 +547,19 @@ cudaError_t launch_assign_slots(glb_ctx* c, const uint32_t* order, uint64_t C) {
   return cudaGetLastError();
 }
 
+__global__ void k_cold_rows(const uint32_t* __restrict__ order, uint64_t C, uint64_t V,
+                            uint32_t* __restrict__ cold_row) {
+  for (uint64_t i = C + (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < V;
+       i += (uint64_t)gridDim.x * blockDim.x)
+    cold_row[order[i]] = (uint32_t)(i - C);  // rank C + j -> cold-store row j
+}
+
+cudaError_t launch_cold_rows(glb_ctx* c, const uint32_t* order, uint64_t C) {
+  k_cold_rows<<<c->num_sms * 8, kThreads, 0, c->stream>>>(order, C, c->V, c->cold_row);
+  count_launch(c);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_shard_rows(glb_ctx* c, const uint32_t* order, uint32_t W, uint32_t r,
                               uint64_t n, uint32_t* out) {
   if (n == 0) return cudaSuccess;

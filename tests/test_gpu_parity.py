@@ -271,6 +271,10 @@ GATHER_ENV = {"warp": {"GLB_GATHER_WARP": "1"}, "block": {"GLB_GATHER_WARP": "0"
               "hitlist": {"GLB_GATHER_LIDORDER": "0"},
               # the miss-taking blocks start on the misses (GLB_MISSES_FIRST)
               "missesfirst": {"GLB_MISSES_FIRST": "1", "GLB_MISS_BLOCKS": "3"},
+              # misses read from the rank-ordered cold store (glb_set_cold_store)
+              "coldstore": {"GLB_COLD_STORE": "1"},
+              "coldstore_host_nobins": {"GLB_COLD_STORE": "1", "GLB_HOST_GATHER": "400",
+                                        "GLB_HOST_GATHER_THREADS": "2", "GLB_MISS_BIN_LOG2": "0"},
               "missesfirst_host": {"GLB_MISSES_FIRST": "1", "GLB_HOST_GATHER": "300",
                                    "GLB_HOST_GATHER_THREADS": "2"},
               "lidorder_host": {"GLB_GATHER_LIDORDER": "1", "GLB_HOST_GATHER": "400",
@@ -541,3 +545,33 @@ def test_host_gather_every_batch(D, depth, fraction):
             assert st["misses"] == n - st["hits"]
     ctx.set_host_gather(0.0)
     assert ctx.host_gather["fraction"] == 0.0
+
+
+@pytest.mark.parametrize("alpha", [0.0, 0.3, 1.0])
+def test_cold_store(alpha):
+    """glb_set_cold_store: the non-cached rows copied in rank order into pinned host memory;
+    samples' and generic extracts give the oracle's bytes (pipelined, host-assisted too)."""
+    g = synth.small_graph(5000, 50000, 2.2, 24, 400, seed=21)
+    go = oracle.GraphOracle(g.indptr, g.indices, g.features)
+    sh = g.shape
+    ctx = make_ctx(g, fanouts=sh.fanouts, max_batch=sh.batch)
+    ctx.set_cold_store(True)
+    ctx.presample(1)
+    ctx.build_cache(alpha)
+    V = g.indptr.shape[0] - 1
+    assert ctx.cold_store_rows == (V - int(np.floor(alpha * V)) if alpha < 1.0 else 0)
+    ctx.set_host_gather(0.3, threads=2)
+    ctx.set_pipeline(2)
+    ob = oracle.epoch_batches(g.train, sh.batch, g.seed, 1)
+    for b in range(len(ob)):
+        ctx.sample_batch(1, b)
+        s = ctx.sample_result()
+        out = torch.full((s.sizes[-1], sh.D), float("nan"), device="cuda")
+        ctx.extract_sample(out, stats=True)
+        exp = go.sample_khop(ob[b], sh.fanouts, g.seed, 1, b)
+        assert np.array_equal(out.cpu().numpy().view(np.uint32), go.extract(exp.uniq).view(np.uint32))
+    ids = np.random.default_rng(3).integers(0, V, 3000).astype(np.uint32)
+    o, st = ctx.extract(torch.from_numpy(ids.view(np.int32)).cuda(), stats=True)
+    assert np.array_equal(o.cpu().numpy().view(np.uint32), go.extract(ids).view(np.uint32))
+    ctx.set_cold_store(False)
+    assert ctx.cold_store_rows == 0
