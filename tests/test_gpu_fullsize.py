@@ -156,7 +156,7 @@ def check_config(name, Ks=None, handoff=False, relabel_modes=("auto",)):
         ctx = make_sampler_ctx(g, sh, relabel=mode)
         ctx.set_pipeline(2)  # bench.py's launch configuration (extract stream, misses first)
         if 4 * sh.D <= 512:  # ... and its host-assisted misses for <= 512-byte rows
-            ctx.set_host_gather(0.25, threads=8)
+            ctx.set_host_gather(0.15, threads=4)
         if mode != "auto":
             assert ctx.relabel_mode == mode
         for K in (Ks or [sh.K]):
@@ -174,11 +174,13 @@ def check_config(name, Ks=None, handoff=False, relabel_modes=("auto",)):
         nb = -(-len(g.train) // sh.batch)
         rng = np.random.default_rng(0)
         a0 = sh.alphas[0]
+        ctx.set_cold_store(4 * sh.D <= 512)  # the bench's cold store for <= 512-byte rows
         ctx.build_cache(a0)
         slot_map = oracle.cache_slots(counts, a0)
         assert a0 < 1.0
         check_batches(ctx, g, sh, go, e, [0, 1, int(rng.integers(2, nb - 1)), nb - 1], out,
                       slot_map)
+        ctx.set_cold_store(False)
         ctx.build_cache(1.0)
         check_batches(ctx, g, sh, go, e, [int(rng.integers(0, nb))], out,
                       oracle.cache_slots(counts, 1.0))
