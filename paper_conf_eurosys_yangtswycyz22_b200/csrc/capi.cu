@@ -118,9 +118,13 @@ void close_shards(glb_ctx* c) {
 // Drop the cold store (host copy + map); callers synchronise first.
 void free_cold(glb_ctx* c) {
   if (c->cold_h) {
-    cudaHostUnregister(c->cold_h);
+    constexpr size_t kPiece = 4ull << 30;  // registered in pieces (build_cold_store)
+    for (size_t off = 0; off < c->cold_bytes; off += kPiece)
+      cudaHostUnregister(reinterpret_cast<uint8_t*>(c->cold_h) + off);
+    (void)cudaGetLastError();
     free(c->cold_h);
   }
+  c->cold_bytes = 0;
   c->cold_h = nullptr;
   c->cold_d = nullptr;
   c->cold_rows = 0;
@@ -885,21 +889,34 @@ static glb_status build_cold_store(glb_ctx* c, const uint32_t* order, uint64_t C
       for (uint64_t i = a; i < b; ++i) memcpy(h + i * rb, src + (size_t)ord[i] * rb, rb);
     });
   for (auto& x : th) x.join();
-  cudaError_t e = cudaHostRegister(h, bytes, cudaHostRegisterMapped | cudaHostRegisterPortable);
-  if (e != cudaSuccess) {
+  // register in 4 GB pieces (one huge registration has failed on a VM host that allows the
+  // same total in pieces); with unified addressing every piece maps at its host address, so
+  // the pieces form one device range.  Any failure: no cold store (misses read the caller's
+  // matrix, as without it) -- a cold store is an optimisation, not a requirement.
+  constexpr size_t kPiece = 4ull << 30;
+  size_t done = 0;
+  bool ok = true;
+  for (size_t off = 0; off < bytes && ok; off += kPiece) {
+    const size_t len = bytes - off < kPiece ? bytes - off : kPiece;
+    void* dp = nullptr;
+    ok = cudaHostRegister(h + off, len, cudaHostRegisterMapped | cudaHostRegisterPortable) == cudaSuccess;
+    if (ok) {
+      done = off + len;
+      ok = cudaHostGetDevicePointer(&dp, h + off, 0) == cudaSuccess && dp == (void*)(h + off);
+    }
+  }
+  (void)cudaGetLastError();
+  if (!ok) {
+    for (size_t off = 0; off < done; off += kPiece) cudaHostUnregister(h + off);
     (void)cudaGetLastError();
     free(h);
-    return set_err(c, GLB_ENOMEM, "cold store: cudaHostRegister(%zu bytes): %s", bytes, cudaGetErrorString(e));
-  }
-  void* dp = nullptr;
-  if ((e = cudaHostGetDevicePointer(&dp, h, 0)) != cudaSuccess) {
-    cudaHostUnregister(h);
-    free(h);
-    return cuda_fail(c, e, "cold store device pointer");
+    fprintf(stderr, "glb: cold store of %zu bytes could not be pinned; misses read the caller's matrix\n", bytes);
+    return GLB_OK;
   }
   c->cold_h = (float*)h;
-  c->cold_d = (const float*)dp;
+  c->cold_d = (const float*)h;  // unified addressing: the device address is the host address
   c->cold_rows = n;
+  c->cold_bytes = bytes;
   CK(dalloc(&c->cold_row, V));
   CK(cudaMemsetAsync(c->cold_row, 0xFF, sizeof(uint32_t) * V, c->stream));
   CK(launch_cold_rows(c, order, C));

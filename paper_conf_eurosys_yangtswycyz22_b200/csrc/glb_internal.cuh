@@ -216,6 +216,7 @@ struct glb_ctx {
   float* cold_h = nullptr;        // host rows [V - C][D], registered mapped + portable
   const float* cold_d = nullptr;  // device alias
   uint64_t cold_rows = 0;
+  size_t cold_bytes = 0;          // registered in 4 GB pieces
   uint32_t* cold_row = nullptr;   // device u32[V]: the cold-store row of a non-cached vertex
   int misses_first = -1;       // miss-taking gather blocks start on the misses: -1 auto (on the
                                // extract stream), GLB_MISSES_FIRST=0/1 forces
