@@ -843,7 +843,9 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
     tp = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tp):
         tj = json.load(open(tp))
-        traffic = tj.get(f"{sh.name}:{alpha}")
+        # the cold store changes the host-side layout the misses read: its own ncu entry
+        traffic = ((ctx.cold_store_rows and tj.get(f"{sh.name}:{alpha}:cold"))
+                   or tj.get(f"{sh.name}:{alpha}"))
     hbm_obj = {"achieved": ach_hbm, "peak": hbm_peak, "unit": "GB/s", "frac": ach_hbm / hbm_peak,
                "peak_source": hbm_src,
                "algorithmic_bytes_per_launch": statistics.mean(hbm_bytes[j] for j in sel)}
