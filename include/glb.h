@@ -284,6 +284,9 @@ glb_status glb_set_host_gather(glb_ctx* ctx, uint32_t threads, double fraction);
  * touch fewer 2 MB host regions, the unit the zero-copy link pays for.  Costs
  * (V - C) x D x 4 bytes of pinned host memory and a host copy at build time (the load_cache
  * phase, Table 6).  Results are identical.  enable 0 drops it.  Environment GLB_COLD_STORE=1.
+ * Best effort: when the copy would leave less than 16 GB of MemAvailable, or pinning it fails,
+ * no cold store is built (a note on stderr; glb_cold_store_rows reports 0) and the misses read
+ * the caller's matrix -- load_cache still returns GLB_OK.
  * glb_cold_store_rows: rows held (0 = none).  Synchronous. */
 glb_status glb_set_cold_store(glb_ctx* ctx, int enable);
 glb_status glb_cold_store_rows(const glb_ctx* ctx, uint64_t* rows);

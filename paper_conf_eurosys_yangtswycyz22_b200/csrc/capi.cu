@@ -870,6 +870,18 @@ static glb_status rank_vertices(glb_ctx* c, const uint32_t* hot, uint32_t* tmp, 
 // misses then fall in the non-cached part only and the warmer (more often missed) rows sit
 // together, so the zero-copy reads touch fewer 2 MB host regions (the host link's cost is
 // per region).  Bytes are the same rows, so results are unchanged.
+// MemAvailable of /proc/meminfo in bytes (0 if unreadable)
+static size_t host_mem_available() {
+  FILE* f = fopen("/proc/meminfo", "r");
+  if (!f) return 0;
+  char line[256];
+  size_t kb = 0;
+  while (fgets(line, sizeof line, f))
+    if (sscanf(line, "MemAvailable: %zu kB", &kb) == 1) break;
+  fclose(f);
+  return kb << 10;
+}
+
 static glb_status build_cold_store(glb_ctx* c, const uint32_t* order, uint64_t C) {
   const uint64_t V = c->V, n = V - C;
   const size_t rb = 4ull * c->D;
@@ -877,6 +889,15 @@ static glb_status build_cold_store(glb_ctx* c, const uint32_t* order, uint64_t C
   CK(cudaMemcpyAsync(ord.data(), order + C, sizeof(uint32_t) * n, cudaMemcpyDeviceToHost, c->stream));
   CK(cudaStreamSynchronize(c->stream));
   const size_t bytes = n * rb;
+  // a second host copy of up to most of the matrix: only when the host can hold it with room
+  // to spare (an over-committed copy is not a recoverable failure -- the kernel OOM-kills the
+  // process while the rows are copied); otherwise the misses read the caller's matrix
+  const size_t avail = host_mem_available();
+  if (avail && bytes + (16ull << 30) > avail) {
+    fprintf(stderr, "glb: cold store of %zu bytes skipped (%zu bytes of host memory available); "
+            "misses read the caller's matrix\n", bytes, avail);
+    return GLB_OK;
+  }
   uint8_t* h = (uint8_t*)aligned_alloc(1 << 21, (bytes + (1 << 21) - 1) & ~(size_t)((1 << 21) - 1));
   if (!h) return set_err(c, GLB_ENOMEM, "cold store: host alloc of %zu bytes", bytes);
   const uint8_t* src = static_cast<const uint8_t*>(c->h_features);
