@@ -93,6 +93,9 @@ def parse(argv=None):
                    help="host feature memory: pageable + cudaHostRegister, or cudaHostAlloc")
     p.add_argument("--shared-inputs", default="auto", choices=["auto", "on", "off"],
                    help="one copy of the host inputs per node, mapped by every local rank")
+    p.add_argument("--numa-replicas", default="auto", choices=["auto", "on", "off"],
+                   help="with shared inputs: one feature-matrix replica per NUMA node, each "
+                        "rank mapping the one on its GPU's node (auto = on with > 1 node)")
     p.add_argument("--cache", default="replicated", choices=["replicated", "sharded"],
                    help="sharded: each rank caches alpha*V distinct rows, peers read them over "
                         "NVLink (NEXT-3; glb_build_cache_sharded)")
@@ -194,6 +197,30 @@ def host_info():
     import glob
     nodes = len(glob.glob("/sys/devices/system/node/node[0-9]*")) or 1
     return {"cpu_model": model, "nproc": ncpu, "numa_nodes": nodes}
+
+
+def gpu_numa_node(index):
+    """NUMA node of local GPU `index`: NVML, else the PCI device's sysfs numa_node; 0 if
+    neither knows (a single-node host or a VM that hides it)."""
+    try:
+        import pynvml as nv
+        nv.nvmlInit()
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+        phys = int(vis.split(",")[index]) if vis and vis.split(",")[0].isdigit() else index
+        h = nv.nvmlDeviceGetHandleByIndex(phys)
+        try:
+            n = nv.nvmlDeviceGetNumaNodeId(h)
+            if n is not None and n >= 0:
+                return int(n)
+        except Exception:
+            pass
+        bus = nv.nvmlDeviceGetPciInfo(h).busId
+        bus = (bus.decode() if isinstance(bus, bytes) else bus).lower()
+        dom, rest = bus.split(":", 1)
+        n = int(open(f"/sys/bus/pci/devices/{dom[-4:]}:{rest}/numa_node").read())
+        return max(n, 0)
+    except Exception:
+        return 0
 
 
 def gpu_info(index):
@@ -630,12 +657,16 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
             dist.barrier()
 
     t0 = time.perf_counter()
-    shared = None
+    shared, numa = None, None
     use_shared = world > 1 and local_world > 1 and args.shared_inputs != "off"
     if use_shared:
         from synth import shm
         store = dist.distributed_c10d._get_default_store()
-        shared = shm.make_graph_shared(sh, local, local_world, store)
+        numa = None
+        if args.numa_replicas == "on" or (args.numa_replicas == "auto"
+                                          and host_info()["numa_nodes"] > 1):
+            numa = gpu_numa_node(local)
+        shared = shm.make_graph_shared(sh, local, local_world, store, numa_node=numa)
         g = shared.graph
     else:
         alloc = None
@@ -897,8 +928,11 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
            "host_gather": ctx.host_gather,
            "cold_store_rows": ctx.cold_store_rows,
            "relabel_table": ctx.relabel_mode, "relabel_l2_window_bytes": ctx.relabel_l2_window,
-           "host_inputs": ("node-shared memfd, generated once by local rank 0 and mapped by "
-                           f"{local_world} ranks") if shared else "private to this rank"}
+           "host_inputs": (("node-shared memfd, generated once by local rank 0 and mapped by "
+                            f"{local_world} ranks") + (f"; features replicated per NUMA node, this "
+                                                       f"rank's GPU on node {numa}"
+                                                       if numa is not None else "")
+                           if shared else "private to this rank")}
 
     # ---- hit rate vs Optimal (accesses recorded over measured epochs, untimed)
     if args.cache == "sharded":

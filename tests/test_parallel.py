@@ -370,3 +370,40 @@ def test_node_shared_graph(tmp_path, world):
         same, seen, owner, align = open(tmp_path / f"r{r}.txt").read().split()
         assert same == "1" and float(seen) == 1234.5 and int(align) == 0
         assert int(owner) == (r == 0)
+
+
+# ------------------------------------------- per-NUMA-node feature replicas
+def _numa_worker(rank, world, port, outdir, nodes):
+    import synth
+    from synth import shm
+    _init(rank, world, port)
+    store = dist.distributed_c10d._get_default_store()
+    sg = shm.make_graph_shared("tiny", rank, world, store, numa_node=nodes[rank])
+    g = sg.graph
+    ref = synth.make_graph("tiny")
+    same = all(np.array_equal(getattr(g, n), getattr(ref, n))
+               for n in ("indptr", "indices", "train", "features"))
+    dist.barrier()
+    # a write by the first rank of each node is seen by exactly the ranks of that node
+    if rank == min(r for r in range(world) if nodes[r] == nodes[rank]):
+        g.features[2, 1] = 100.0 + nodes[rank]
+    dist.barrier()
+    seen = float(g.features[2, 1])
+    with open(os.path.join(outdir, f"n{rank}.txt"), "w") as f:
+        f.write(f"{int(same)} {seen} {g.features.ctypes.data % 4096}")
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_numa_feature_replicas(tmp_path):
+    """Four local ranks on two NUMA nodes (0, 1, 0, 1): every rank sees the generator's
+    values; the ranks of a node share one feature copy and the two nodes' copies are
+    distinct memory (a write on one node's copy is invisible on the other's)."""
+    nodes = [0, 1, 0, 1]
+    world = len(nodes)
+    mp.spawn(_numa_worker, args=(world, free_port(), str(tmp_path), nodes), nprocs=world,
+             join=True)
+    for r in range(world):
+        same, seen, align = open(tmp_path / f"n{r}.txt").read().split()
+        assert same == "1" and int(align) == 0
+        assert float(seen) == 100.0 + nodes[r]
