@@ -5,12 +5,16 @@
 // time is "mainly dominated by loading features ... from host memory ... due
 // to the limited PCIe bandwidth" (L79 §2).
 //
-// One persistent launch serves both halves: every block first claims chunks of
-// cache hits (HBM) from one device counter and, once those run out, chunks of
-// misses read straight from the mapped pinned host matrix (zero copy over PCIe)
-// from a second counter -- all blocks drain the HBM work before any waits on the
-// host link.  Misses arrive ordered by host address (launch_sort_misses); a
-// share of them can be gathered by host threads instead (hostgather.cu).
+// One persistent launch serves both halves: chunks of cache hits (HBM) are handed
+// out by one device counter and chunks of misses, read straight from mapped pinned
+// host memory (zero copy over PCIe), by a second.  Which blocks take which: by
+// default every block drains the hits and then takes misses; with a miss-block cap
+// (one block per SM when host threads assist or on the pipelined extract stream)
+// only the first blocks take misses, and on the extract stream they start on them
+// ("misses first": the host link is the critical path) while the rest of the grid
+// gathers the hits.  Misses arrive ordered by host address (launch_sort_misses),
+// from the cold store when there is one (rank-ordered copy of the non-cached rows);
+// a share of them can be gathered by host threads instead (hostgather.cu).
 //
 // A block copies a chunk of R rows per iteration: the chunk's (dst, src)
 // work-list entries are staged in shared memory (double-buffered, the next
