@@ -200,25 +200,14 @@ def host_info():
 
 
 def gpu_numa_node(index):
-    """NUMA node of local GPU `index`: NVML, else the PCI device's sysfs numa_node; 0 if
-    neither knows (a single-node host or a VM that hides it)."""
+    """NUMA node of local CUDA device `index`: the sysfs numa_node of its PCI function (the
+    address from the CUDA device properties, so CUDA's and NVML's device orders cannot be
+    confused); 0 if unknown (a single-node host or a VM that hides it)."""
     try:
-        import pynvml as nv
-        nv.nvmlInit()
-        vis = os.environ.get("CUDA_VISIBLE_DEVICES")
-        phys = int(vis.split(",")[index]) if vis and vis.split(",")[0].isdigit() else index
-        h = nv.nvmlDeviceGetHandleByIndex(phys)
-        try:
-            n = nv.nvmlDeviceGetNumaNodeId(h)
-            if n is not None and n >= 0:
-                return int(n)
-        except Exception:
-            pass
-        bus = nv.nvmlDeviceGetPciInfo(h).busId
-        bus = (bus.decode() if isinstance(bus, bytes) else bus).lower()
-        dom, rest = bus.split(":", 1)
-        n = int(open(f"/sys/bus/pci/devices/{dom[-4:]}:{rest}/numa_node").read())
-        return max(n, 0)
+        import torch
+        p = torch.cuda.get_device_properties(index)
+        addr = f"{p.pci_domain_id:04x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0"
+        return max(int(open(f"/sys/bus/pci/devices/{addr}/numa_node").read()), 0)
     except Exception:
         return 0
 
