@@ -575,3 +575,34 @@ def test_cold_store(alpha):
     assert np.array_equal(o.cpu().numpy().view(np.uint32), go.extract(ids).view(np.uint32))
     ctx.set_cold_store(False)
     assert ctx.cold_store_rows == 0
+
+
+@pytest.mark.parametrize("D", [7, 100])
+def test_cold_store_rebuild(D):
+    """The cold store follows the cache: load_cache at another alpha (and with another
+    hotness map) replaces it; scalar (D % 4 != 0) and vector rows; depth 1 and 2; every
+    batch's bytes equal the oracle's after each rebuild."""
+    g = synth.small_graph(4000, 40000, 2.2, D, 500, seed=23)
+    go = oracle.GraphOracle(g.indptr, g.indices, g.features)
+    sh = g.shape
+    V = g.indptr.shape[0] - 1
+    ctx = make_ctx(g, fanouts=sh.fanouts, max_batch=sh.batch)
+    ctx.set_cold_store(True)
+    ctx.presample(1)
+    ob = oracle.epoch_batches(g.train, sh.batch, g.seed, 1)
+    for alpha, depth, degree in ((0.2, 1, False), (0.6, 2, False), (0.35, 2, True)):
+        if degree:
+            ctx.build_cache_policy(alpha, "degree")
+        else:
+            ctx.build_cache(alpha)
+        assert ctx.cold_store_rows == V - int(np.floor(alpha * V))
+        ctx.set_pipeline(depth)
+        for b in range(len(ob)):
+            ctx.sample_batch(1, b)
+            s = ctx.sample_result()
+            out = torch.full((s.sizes[-1], sh.D), float("nan"), device="cuda")
+            st = ctx.extract_sample(out, stats=True)
+            exp = go.sample_khop(ob[b], sh.fanouts, g.seed, 1, b)
+            assert np.array_equal(out.cpu().numpy().view(np.uint32),
+                                  go.extract(exp.uniq).view(np.uint32))
+            assert st["hits"] + st["misses"] == exp.uniq.shape[0]
