@@ -874,11 +874,18 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
                 "peak_source": "DMA H2D of 1 GiB pinned host memory, best of 5, measured in "
                                f"this run (PCIe Gen5 x16 nominal {PCIE_GEN5_X16_GBS:.0f} GB/s)",
                 "algorithmic_bytes_per_launch": statistics.mean(link_bytes[j] for j in sel)}
+    # `traffic`: ncu bytes per launch on the binding roof (sysmem reads for the host link,
+    # DRAM read + write for HBM), comparable with `algorithmic_bytes_per_launch`; the
+    # other counters of the same capture in `traffic_detail`
+    detail = traffic if isinstance(traffic, dict) else None
+    if detail is not None:
+        traffic = detail.get("sysmem_read_bytes") if host_bound else detail.get("dram_bytes")
     if host_bound:
         roof = {"kernel": "k_gather (extract a7)", "bound": "host-link", **link_obj,
-                "traffic": traffic, "hbm": hbm_obj}
+                "traffic": traffic, "traffic_detail": detail, "hbm": hbm_obj}
     else:
         roof = {"kernel": "k_gather (extract a7)", "bound": "hbm", **hbm_obj, "traffic": traffic,
+                "traffic_detail": detail,
                 "host_link": link_obj}
     roof.update({
         "extract_ms_per_step": x_mean,
