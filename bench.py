@@ -1075,18 +1075,8 @@ def hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs, b
         v, num, den = ctx.footprint_similarity(per_epoch[0], per_epoch[1], 0.1)
         similarity = {"epochs": [m0, m0 + 1], "top_frac": 0.1, "value": v,
                       "numerator": num, "denominator": den, "source": "Table 2 (L329)"}
-    sweep, result_hit = [], None
-    for a in sorted(set(sh.alphas) | {alpha}):
-        policies = {}
-        if 0.0 < a < 1.0:  # Fig 10 analog: Degree / Random vs PreSC vs Optimal
-            for pol in ("degree", "random"):
-                ctx.build_cache_policy(a, pol, seed=g.seed)
-                hs = ctx.hit_stats()
-                policies[pol] = hs["hits"] / hs["total"] if hs["total"] else 0.0
-        ctx.build_cache(a)
-        hs = ctx.hit_stats()
-        H = hs["hits"] / hs["total"] if hs["total"] else 0.0
-        Hs = hs["optimal_hits"] / hs["total"] if hs["total"] else 0.0
+    def sweep_rate():
+        """seeds/s of --sweep-steps pipelined steps with the cache as built (cold store off)"""
         torch.cuda.synchronize()
         s0 = torch.cuda.Event(enable_timing=True)
         s1 = torch.cuda.Event(enable_timing=True)
@@ -1099,13 +1089,26 @@ def hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs, b
             sd += n_seeds(b)
         s1.record(xs)
         torch.cuda.synchronize()
-        ms = s0.elapsed_time(s1)
+        return sd * world / (s0.elapsed_time(s1) / 1e3)
+
+    sweep, result_hit = [], None
+    for a in sorted(set(sh.alphas) | {alpha}):
+        policies = {}
+        if 0.0 < a < 1.0:  # Fig 10 analog: Degree / Random vs PreSC vs Optimal
+            for pol in ("degree", "random"):
+                ctx.build_cache_policy(a, pol, seed=g.seed)
+                hs = ctx.hit_stats()
+                policies[pol] = hs["hits"] / hs["total"] if hs["total"] else 0.0
+        ctx.build_cache(a)
+        hs = ctx.hit_stats()
+        H = hs["hits"] / hs["total"] if hs["total"] else 0.0
+        Hs = hs["optimal_hits"] / hs["total"] if hs["total"] else 0.0
         sweep.append({"alpha": a, "cache_rows": hs["cache_rows"], "hit_rate": H,
                       "optimal_hit_rate": Hs,
                       "presc_vs_optimal_pct": (100.0 * H / Hs) if Hs > 0 else None,
                       "degree_hit_rate": policies.get("degree"),
                       "random_hit_rate": policies.get("random"),
-                      "seeds_per_s": sd * world / (ms / 1e3)})
+                      "seeds_per_s": sweep_rate()})
         if a == alpha:
             result_hit = sweep[-1]
     k_sweep = []
@@ -1120,7 +1123,8 @@ def hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs, b
             H = hs["hits"] / hs["total"] if hs["total"] else 0.0
             Hs = hs["optimal_hits"] / hs["total"] if hs["total"] else 0.0
             k_sweep.append({"K": K, "alpha": a_k, "hit_rate": H, "optimal_hit_rate": Hs,
-                            "presc_vs_optimal_pct": 100.0 * H / Hs if Hs else None})
+                            "presc_vs_optimal_pct": 100.0 * H / Hs if Hs else None,
+                            "seeds_per_s": sweep_rate()})
     return {"hit_rate": result_hit, "alpha_sweep": sweep, "presc_k_sweep": k_sweep,
             "measured_epochs": [m0, m0 + args.measure_epochs - 1],
             "footprint_similarity": similarity}
