@@ -1126,6 +1126,8 @@ def hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs, b
                             "presc_vs_optimal_pct": 100.0 * H / Hs if Hs else None,
                             "seeds_per_s": sweep_rate()})
     return {"hit_rate": result_hit, "alpha_sweep": sweep, "presc_k_sweep": k_sweep,
+            "sweep_seeds_per_s_is": f"{args.sweep_steps} pipelined steps per point, cold store "
+                                    "off (the sweeps rebuild the cache per point)",
             "measured_epochs": [m0, m0 + args.measure_epochs - 1],
             "footprint_similarity": similarity}
 
