@@ -1123,8 +1123,7 @@ def hit_rate_sweeps(args, ctx, g, sh, alpha, world, rank, nb, out, stream, xs, b
             H = hs["hits"] / hs["total"] if hs["total"] else 0.0
             Hs = hs["optimal_hits"] / hs["total"] if hs["total"] else 0.0
             k_sweep.append({"K": K, "alpha": a_k, "hit_rate": H, "optimal_hit_rate": Hs,
-                            "presc_vs_optimal_pct": 100.0 * H / Hs if Hs else None,
-                            "seeds_per_s": sweep_rate()})
+                            "presc_vs_optimal_pct": 100.0 * H / Hs if Hs else None})
     return {"hit_rate": result_hit, "alpha_sweep": sweep, "presc_k_sweep": k_sweep,
             "sweep_seeds_per_s_is": f"{args.sweep_steps} pipelined steps per point, cold store "
                                     "off (the sweeps rebuild the cache per point)",
