@@ -2,7 +2,8 @@
 cache, extract with hits and misses, pipeline depth 2) for compute-sanitizer, under each
 library variant (environment knobs read at glb_create): default, warp / block-staged
 relabel pre-dedup, host-assisted misses, one miss bin per row (device scan), the
-warp-independent gather, a capped miss-block count."""
+warp-independent gather, a capped miss-block count, the cold store (with and without
+host-assisted misses)."""
 import os
 import sys
 
@@ -20,7 +21,9 @@ go = oracle.GraphOracle(g.indptr, g.indices, g.features)
 VARIANTS = [{}, {"GLB_RELABEL_DEDUP": "1"}, {"GLB_RELABEL_DEDUP": "2"},
             {"GLB_HOST_GATHER": "400", "GLB_HOST_GATHER_THREADS": "2"},
             {"GLB_MISS_BIN_LOG2": "7", "GLB_GATHER_WARP": "1"}, {"GLB_MISS_BLOCKS": "3"},
-            {"GLB_GATHER_LIDORDER": "0", "GLB_HOST_GATHER": "400", "GLB_HOST_GATHER_THREADS": "2"}]
+            {"GLB_GATHER_LIDORDER": "0", "GLB_HOST_GATHER": "400", "GLB_HOST_GATHER_THREADS": "2"},
+            {"GLB_COLD_STORE": "1", "GLB_HOST_GATHER": "150", "GLB_HOST_GATHER_THREADS": "2"},
+            {"GLB_COLD_STORE": "1"}]
 KEYS = {k for v in VARIANTS for k in v}
 for var, mode in [(v, m) for v in VARIANTS for m in ["dense", "hash"]]:
     for k in KEYS:
@@ -49,6 +52,9 @@ for var, mode in [(v, m) for v in VARIANTS for m in ["dense", "hash"]]:
     assert np.array_equal(s.uniq.cpu().numpy().view(np.uint32), exp.uniq)
     ids = torch.from_numpy(exp.uniq.view(np.int32)).cuda()
     o2 = ctx.extract(ids)
+    assert np.array_equal(o2.cpu().numpy().view(np.uint32), go.extract(exp.uniq).view(np.uint32))
+    if var.get("GLB_COLD_STORE") == "1":
+        assert ctx.cold_store_rows > 0
     ctx.set_sampler("rwalk", layers=2, max_batch=sh.batch)
     ctx.sample_batch(1, 2)
     ctx.sample_result()
