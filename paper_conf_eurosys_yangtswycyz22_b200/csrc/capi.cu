@@ -636,6 +636,7 @@ glb_status glb_set_sampler(glb_ctx* c, int kind, const uint32_t* fanouts, uint32
   c->rw_len = len;
   c->rw_topk = topk;
   c->sampler_set = true;
+  CK(hg_reserve(c));  // host-assisted staging for the new capacity (no-op when off)
   return GLB_OK;
 }
 
@@ -1351,6 +1352,7 @@ glb_status glb_set_host_gather(glb_ctx* c, uint32_t threads, double fraction) {
   CK(hg_configure(c, threads - 1));  // the host-function thread itself is the last worker
   c->hg_permille = pm;
   c->hg_threads = threads;
+  CK(hg_reserve(c));  // pinned staging now, not in the first extract
   return GLB_OK;
 }
 

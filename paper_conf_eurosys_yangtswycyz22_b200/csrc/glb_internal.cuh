@@ -417,6 +417,7 @@ cudaError_t launch_value_hist(glb_ctx* c, const uint32_t* a, uint64_t n, unsigne
 // hostgather.cu: a fraction of the misses gathered by host threads into pinned staging,
 // read back sequentially by the GPU (glb_set_host_gather)
 cudaError_t hg_configure(glb_ctx* c, uint32_t threads);
+cudaError_t hg_reserve(glb_ctx* c);  // size the host part's buffers for the sampler config
 void hg_free(glb_ctx* c);
 bool hg_active(const glb_ctx* c);
 cudaError_t hg_enqueue(glb_ctx* c, float* out, const uint2* miss_sorted, uint32_t** dcnt_out);

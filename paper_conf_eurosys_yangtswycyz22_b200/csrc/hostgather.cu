@@ -349,13 +349,15 @@ bool hg_active(const glb_ctx* c) {
          c->st == c->sts[c->cur];  // a sample of this ctx (not a handoff ring slot)
 }
 
-// Enqueue the host part of the current sample's extract (rows of the tail of
-// `miss_sorted`) and return the device counts {nh, n_zc, ...} the extract kernel takes.
-cudaError_t hg_enqueue(glb_ctx* c, float* out, const uint2* miss_sorted, uint32_t** dcnt_out) {
+// Size the host part's buffers (pinned work lists and staging, device counts) for the
+// current sampler config: the host part of the largest possible miss list.  Called when the
+// host-assisted share or the sampler changes (so the first extract does not pay the pinned
+// allocations) and again, as a no-op, by every hg_enqueue.
+cudaError_t hg_reserve(glb_ctx* c) {
   HostGather* h = c->hg;
-  const int s = c->cur;
-  // capacity: the host part of the largest possible miss list of this sampler config
+  if (!h || !c->hg_permille || !c->D) return cudaSuccess;
   const uint64_t ub = c->sb.ub[c->sb.L] > c->sb.cap_batch ? c->sb.ub[c->sb.L] : c->sb.cap_batch;
+  if (!ub) return cudaSuccess;  // no sampler yet
   const uint64_t cap = (ub * c->hg_permille + 999) / 1000;
   cudaError_t e;
   if (h->cap < cap || h->D != c->D) {
@@ -379,6 +381,16 @@ cudaError_t hg_enqueue(glb_ctx* c, float* out, const uint2* miss_sorted, uint32_
     h->cap = cap;
     h->D = c->D;
   }
+  return cudaSuccess;
+}
+
+// Enqueue the host part of the current sample's extract (rows of the tail of
+// `miss_sorted`) and return the device counts {nh, n_zc, ...} the extract kernel takes.
+cudaError_t hg_enqueue(glb_ctx* c, float* out, const uint2* miss_sorted, uint32_t** dcnt_out) {
+  HostGather* h = c->hg;
+  const int s = c->cur;
+  cudaError_t e = hg_reserve(c);
+  if (e != cudaSuccess) return e;
   // misses per batch from the pinned counts of recent batches (completed, or a benign
   // race with the copy that is writing them: either value is a miss count)
   for (int k = 0; k < kSlots; ++k) {
