@@ -276,7 +276,8 @@ glb_status glb_extract_stream(glb_ctx* ctx, void** cuda_stream_out);
  * for every fraction.  fraction 0 = off (default; environment GLB_HOST_GATHER = permille,
  * GLB_HOST_GATHER_THREADS); threads 0 = the usable cores minus two.  Applies to samples of
  * this ctx (not to handoff-received ones) and to caches with C < V.  Synchronous (creates the
- * thread pool).  Errors: EINVAL (fraction not in [0,1), threads > 256). */
+ * thread pool and sizes the pinned staging for the sampler config -- again at every
+ * glb_set_sampler -- so no extract allocates).  Errors: EINVAL (fraction not in [0,1), threads > 256). */
 glb_status glb_set_host_gather(glb_ctx* ctx, uint32_t threads, double fraction);
 /* Cold store: at the next glb_build_cache (single-GPU cache), copy the rows NOT cached --
  * ranks C..V-1 of the load_cache order (L301) -- into a pinned host buffer in rank order and
