@@ -712,7 +712,11 @@ def run_workload(args, sh, alpha, world, rank, local, local_world, dev, stream, 
     torch.cuda.synchronize()
     t_cache = time.perf_counter() - t0
     hg = args.host_gather
-    hg = ((0.15 if cold else 0.25) if small_rows else 0.0) if hg == "auto" else float(hg)
+    # the share the miss path measured best at (profiles/r02z, r02q2): smaller with the cold
+    # store (fewer host regions left for the host threads to win); the store may have been
+    # skipped (host memory), so ask the ctx whether it holds one
+    cold_on = ctx.cold_store_rows > 0
+    hg = ((0.15 if cold_on else 0.25) if small_rows else 0.0) if hg == "auto" else float(hg)
     if hg > 0:
         nt = args.host_gather_threads
         if nt <= 0:  # share the node's cores between the local ranks
