@@ -85,6 +85,24 @@ __device__ __forceinline__ uint32_t ld_csr(const uint32_t* p) {
 #endif
 }
 
+// The (indptr[v], indptr[v+1]) pair of a random frontier vertex.  A plain load of one random
+// 8-byte word pulls in a 128-byte line (ncu on PA's last random-walk hop: ~200 DRAM bytes
+// per walk step).  GLB_INDPTR_LD=1 (A/B builds) asks for a 64-byte fill like ld_csr: TW
+// 578.6 vs 580.2, UK 433.0 vs 433.4, PR 207.2 vs 207.0 us/step, but PA (random walks)
+// 595 vs 574 -- slower, so plain loads stay (profiles/r02t_indptr_ld_ab.txt).
+#ifndef GLB_INDPTR_LD
+#define GLB_INDPTR_LD 0
+#endif
+__device__ __forceinline__ uint64_t ld_indptr(const uint64_t* p) {
+#if GLB_INDPTR_LD == 1
+  uint64_t v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::64B.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+#else
+  return *p;
+#endif
+}
+
 // Insert one pick into the relabel table: keep the smallest position of this
 // generation.  Values only decrease over time, so a (possibly stale) read that
 // is already <= e proves the atomic would be a no-op.
@@ -313,8 +331,8 @@ __global__ void __launch_bounds__(kThreads)
     uint64_t lo = 0;
     if (active) {
       v = uniq[d];
-      lo = indptr[v];
-      deg = (uint32_t)(indptr[v + 1] - lo);
+      lo = ld_indptr(indptr + v);
+      deg = (uint32_t)(ld_indptr(indptr + v + 1) - lo);
       if (!HASH && hop == 0 && s == 0 && __ldcg(&T.e[v].gp) != enc_pos(gen, d))
         atomicOr(&st_w->err, kErrDupSeed);
     }
@@ -443,7 +461,7 @@ __global__ void __launch_bounds__(kThreads)
     const uint32_t d = w0 + gi;
     if (gi >= gpw || d >= n_l) continue;
     const uint32_t v = uniq[d];
-    const uint64_t lo = indptr[v], hi = indptr[v + 1];
+    const uint64_t lo = ld_indptr(indptr + v), hi = ld_indptr(indptr + v + 1);
     const unsigned long long pbase = lo ? wprefix[lo - 1] : 0ull;
     const unsigned long long W = hi > lo ? wprefix[hi - 1] - pbase : 0ull;
     for (uint32_t s = sl; s < k; s += G) {
@@ -494,8 +512,8 @@ __global__ void __launch_bounds__(kThreads)
   uint32_t* ch = chosen[wib];
   for (uint32_t d = warp_global; d < n_l; d += nwarps) {
     const uint32_t v = uniq[d];
-    const uint64_t lo = indptr[v];
-    const uint32_t deg = (uint32_t)(indptr[v + 1] - lo);
+    const uint64_t lo = ld_indptr(indptr + v);
+    const uint32_t deg = (uint32_t)(ld_indptr(indptr + v + 1) - lo);
     if (!HASH && hop == 0 && lane == 0 && __ldcg(&T.e[v].gp) != enc_pos(gen, d))
       atomicOr(&st_w->err, kErrDupSeed);
     if (deg > k) {
@@ -574,8 +592,8 @@ __global__ void __launch_bounds__(kThreads, GLB_RWALK_MINB)
 #pragma unroll
         for (int t = 0; t < LEN; ++t) {
           if ((uint32_t)t < len) {
-            const uint64_t b = indptr[cur];
-            const uint32_t deg = (uint32_t)(indptr[cur + 1] - b);
+            const uint64_t b = ld_indptr(indptr + cur);
+            const uint32_t deg = (uint32_t)(ld_indptr(indptr + cur + 1) - b);
             if (deg == 0) break;
             const uint64_t r = draw64(seed, v, (w << 8) | ((uint32_t)t >> 1), batch, c3, t & 1);
             cur = ld_csr(indices + b + bounded(r, deg));

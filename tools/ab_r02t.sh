@@ -1,2 +1,11 @@
+# r02t: 64-byte L2 fill on the sampler's random indptr loads (default build) vs plain loads
+# (GLB_INDPTR_LD=0 build), alpha = 1 on every shape (the sampler-heavy steps), alternating builds
 set -x
-GLB_MISS_BLOCKS=148 python tools/miss_probe.py --spans 1.0 --bins 21 --reps 3 --region-fracs 1.0,0.75,0.5,0.25,0.1 > gpurun_out/region_probe.jsonl 2>&1
+for C in "PR 1.0 200" "TW 1.0 60" "UK 1.0 60" "PA 1.0 60"; do
+  set -- $C
+  for L in default WT_ip0 default WT_ip0; do
+    if [ $L = default ]; then unset GLB_LIBRARY; else export GLB_LIBRARY=build/ab/libglb_$L.so; fi
+    python tools/ab_env.py --config $1 --alpha $2 --steps $3 --repeat 2 --variants "$L:" >> gpurun_out/indptr_ld_$1.jsonl 2>&1
+  done
+  unset GLB_LIBRARY
+done
