@@ -70,8 +70,8 @@ def _replicate_features(src: np.ndarray, node: int) -> tuple[_Mem, np.ndarray]:
     each page on the node of the CPU that writes it.  Bytes are copied, never computed."""
     m = _Mem(src.nbytes, f"glb_features_numa{node}")
     dst = m.array(src.dtype, src.shape)
-    cpus = node_cpus(node)
-    old = os.sched_getaffinity(0) if cpus else None
+    old = os.sched_getaffinity(0)
+    cpus = (node_cpus(node) or set()) & old  # only CPUs this process may run on
     try:
         if cpus:
             os.sched_setaffinity(0, cpus)
@@ -80,7 +80,7 @@ def _replicate_features(src: np.ndarray, node: int) -> tuple[_Mem, np.ndarray]:
         for i in range(0, flat_s.size, step):
             flat_d[i:i + step] = flat_s[i:i + step]
     finally:
-        if old is not None:
+        if cpus:
             os.sched_setaffinity(0, old)
     return m, dst
 
